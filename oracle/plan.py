@@ -1,0 +1,101 @@
+"""Oracle of the plan's integer outputs: stream tiles, row classes, hub chunks,
+hot prefix H, row-block partition bounds.
+
+The paper runs cuSPARSE and never describes scheduling (Alg. 1
+is a plain "parfor row"); these are build constants (reading c23), RE-DECLARED
+here from DESIGN.md §Plan, not imported from the library:
+
+  TILE_D      = 2048   stream tile "diagonal": row r (r < N) belongs to tile
+                        k = floor((row_ptr[r] + r) / TILE_D); tiles
+                        k = 0 .. K-1, K = ceil((NZ + N) / TILE_D);
+                        bounds b_k = lower_bound_{r in [0,N]}(row_ptr[r] + r >= k*TILE_D)
+  STREAM_MAX  = 2048   rows with L <= STREAM_MAX are computed inside their
+                        stream tile; longer rows are always the last row of
+                        their tile and are excluded from it
+  CTA_MAX     = 16384  STREAM_MAX < L <= CTA_MAX: one CTA per row
+  HUB_CHUNK   = 16384  L > CTA_MAX: hub row cut into ceil(L / HUB_CHUNK)
+                        chunks of HUB_CHUNK entries (merge-path split)
+
+H: the length of the leading run of columns j of B with
+colcnt_B[j] * N > NZ_B (the hot, hub-grouped prefix of x under RABBIT++).
+
+Partition: b_0 = 0, b_G = N,
+b_k = lower_bound(row_ptr_B, ceil(k * NZ / G)) for 0 < k < G.
+
+TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).
+"""
+from __future__ import annotations
+
+import numpy as np
+
+TILE_D = 2048
+STREAM_MAX = 2048
+CTA_MAX = 16384
+HUB_CHUNK = 16384
+
+
+def tile_bounds(row_ptr) -> np.ndarray:
+    row_ptr = np.asarray(row_ptr, np.int64)
+    n = len(row_ptr) - 1
+    nnz = int(row_ptr[-1])
+    if n == 0:
+        return np.zeros(1, np.int64)
+    K = -(-(nnz + n) // TILE_D)
+    c = row_ptr + np.arange(n + 1, dtype=np.int64)       # strictly increasing
+    b = np.empty(K + 1, np.int64)
+    for k in range(K + 1):
+        # lower_bound over r in [0, n]
+        lo, hi = 0, n
+        while lo < hi:
+            mid = (lo + hi) // 2
+            if c[mid] >= k * TILE_D:
+                hi = mid
+            else:
+                lo = mid + 1
+        b[k] = lo
+    return b
+
+
+def row_classes(row_ptr):
+    """(cta_rows, hub_rows, chunk_row, chunk_idx), all ascending."""
+    row_ptr = np.asarray(row_ptr, np.int64)
+    L = np.diff(row_ptr)
+    cta = [r for r in range(len(L)) if STREAM_MAX < L[r] <= CTA_MAX]
+    hub = [r for r in range(len(L)) if L[r] > CTA_MAX]
+    ch_r, ch_i = [], []
+    for r in hub:
+        for c in range(-(-int(L[r]) // HUB_CHUNK)):
+            ch_r.append(r)
+            ch_i.append(c)
+    return (np.array(cta, np.int64), np.array(hub, np.int64),
+            np.array(ch_r, np.int64), np.array(ch_i, np.int64))
+
+
+def stream_rows(row_ptr, b) -> np.ndarray:
+    """Flag of rows computed inside a stream tile (every row with L <= STREAM_MAX)."""
+    L = np.diff(np.asarray(row_ptr, np.int64))
+    return L <= STREAM_MAX
+
+
+def hot_prefix(n, col_B) -> int:
+    nnz = len(col_B)
+    if n == 0:
+        return 0
+    colcnt = np.bincount(np.asarray(col_B, np.int64), minlength=n).astype(np.int64)
+    hot = colcnt * np.int64(n) > nnz
+    H = 0
+    while H < n and hot[H]:
+        H += 1
+    return H
+
+
+def partition(row_ptr, G: int) -> np.ndarray:
+    row_ptr = np.asarray(row_ptr, np.int64)
+    n = len(row_ptr) - 1
+    nnz = int(row_ptr[-1])
+    b = np.zeros(G + 1, np.int64)
+    b[G] = n
+    for k in range(1, G):
+        target = -(-(k * nnz) // G)
+        b[k] = int(np.searchsorted(row_ptr, target, side="left"))
+    return b
