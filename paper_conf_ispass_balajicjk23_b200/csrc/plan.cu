@@ -1,0 +1,830 @@
+// spmv_plan / spmv_permute: validation, inverse permutation, B = P A P^T,
+// stream tiles, row classes, hub chunks, hot prefix H, row-block partition.
+//
+// PAPER.md:86 (§IV-A): reordering "assigns community members consecutive
+// IDs"; applied symmetrically B[perm[i], perm[j]] = A[i, j].
+// The paper does this on the CPU and never describes it; here it is a chain
+// of HBM-bound GPU kernels:
+//   validate rows/cols -> inverse perm (bijection check) -> len_B[perm[i]] =
+//   len_A[i] -> exclusive scan -> partition -> local row_ptr -> tiles/classes
+//   (plan, synchronous) ; relabel+scatter -> per-row stable sort (permute,
+//   stream-ordered).
+#include <algorithm>
+#include <cstring>
+
+#include "plan.cuh"
+
+namespace spmv {
+namespace {
+
+constexpr int TPB = 256;
+
+inline int grid_for(int64_t n, int tpb = TPB, int cap = 148 * 32) {
+  int64_t g = (n + tpb - 1) / tpb;
+  if (g < 1) g = 1;
+  if (g > cap) g = cap;
+  return (int)g;
+}
+
+#define GRID_STRIDE(i, n)                                                      \
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < (n); \
+       i += (int64_t)gridDim.x * blockDim.x)
+
+// ---------------------------------------------------------------- validation
+template <typename T>
+__global__ void k_validate_rp(const T* rp, int64_t n, int64_t nnz, int* flags) {
+  GRID_STRIDE(i, n) {
+    int64_t a = (int64_t)rp[i], b = (int64_t)rp[i + 1];
+    if (b < a || a < 0 || b > nnz) flags[0] = 1;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if ((int64_t)rp[0] != 0 || (int64_t)rp[n] != nnz) flags[0] = 1;
+  }
+}
+
+__global__ void k_validate_col(const int32_t* col, int64_t nnz, int64_t n, int* flags) {
+  GRID_STRIDE(k, nnz) {
+    int32_t c = col[k];
+    if (c < 0 || (int64_t)c >= n) flags[1] = 1;
+  }
+}
+
+__global__ void k_identity(int32_t* p, int64_t n) {
+  GRID_STRIDE(i, n) p[i] = (int32_t)i;
+}
+
+__global__ void k_fill_i32(int32_t* p, int64_t n, int32_t v) {
+  GRID_STRIDE(i, n) p[i] = v;
+}
+
+// inv[perm[i]] = i; a repeated or out-of-range target flags EPERM.
+__global__ void k_inverse(const int32_t* perm, int64_t n, int32_t* inv, int* flags) {
+  GRID_STRIDE(i, n) {
+    int32_t v = perm[i];
+    if (v < 0 || (int64_t)v >= n) {
+      flags[2] = 1;
+      continue;
+    }
+    int32_t old = atomicExch(&inv[v], (int32_t)i);
+    if (old != -1) flags[2] = 1;
+  }
+}
+
+template <typename T>
+__global__ void k_lenB(const T* rpA, const int32_t* perm, int64_t n, int64_t* lenB) {
+  GRID_STRIDE(i, n) lenB[perm[i]] = (int64_t)rpA[i + 1] - (int64_t)rpA[i];
+}
+
+// --------------------------------------------------------------------- scan
+constexpr int SCAN_T = 512, SCAN_I = 8, SCAN_B = SCAN_T * SCAN_I;
+
+__device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t* sw, int64_t* total) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  int64_t inc = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    int64_t t = __shfl_up_sync(0xffffffffu, inc, o);
+    if (lane >= o) inc += t;
+  }
+  if (lane == 31) sw[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    int64_t s = lane < nw ? sw[lane] : 0, si = s;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      int64_t t = __shfl_up_sync(0xffffffffu, si, o);
+      if (lane >= o) si += t;
+    }
+    if (lane < nw) sw[lane] = si - s;
+    if (lane == 31) sw[32] = si;
+  }
+  __syncthreads();
+  int64_t r = sw[w] + inc - v;
+  if (total) *total = sw[32];
+  __syncthreads();
+  return r;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(SCAN_T) k_scan_reduce(const T* in, int64_t n, int64_t* bsum) {
+  __shared__ int64_t sw[33];
+  int64_t base = (int64_t)blockIdx.x * SCAN_B + (int64_t)threadIdx.x * SCAN_I, s = 0;
+#pragma unroll
+  for (int j = 0; j < SCAN_I; ++j)
+    if (base + j < n) s += (int64_t)in[base + j];
+  int64_t tot;
+  block_excl_scan(s, sw, &tot);
+  if (threadIdx.x == 0) bsum[blockIdx.x] = tot;
+}
+
+// single CTA: exclusive scan of bsum[0..nb) in place, bsum[nb] = total
+__global__ void __launch_bounds__(1024) k_scan_top(int64_t* bsum, int64_t nb) {
+  __shared__ int64_t sw[33];
+  __shared__ int64_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (int64_t base = 0; base < nb; base += 1024) {
+    int64_t i = base + threadIdx.x;
+    int64_t v = i < nb ? bsum[i] : 0, tot;
+    int64_t e = block_excl_scan(v, sw, &tot);
+    if (i < nb) bsum[i] = carry + e;
+    __syncthreads();
+    if (threadIdx.x == 0) carry += tot;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) bsum[nb] = carry;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(SCAN_T)
+    k_scan_down(const T* in, int64_t n, const int64_t* bsum, int64_t nb, int64_t* out) {
+  __shared__ int64_t sw[33];
+  int64_t base = (int64_t)blockIdx.x * SCAN_B + (int64_t)threadIdx.x * SCAN_I, s = 0;
+  T v[SCAN_I];
+#pragma unroll
+  for (int j = 0; j < SCAN_I; ++j) {
+    v[j] = base + j < n ? in[base + j] : (T)0;
+    s += (int64_t)v[j];
+  }
+  int64_t e = block_excl_scan(s, sw, nullptr) + bsum[blockIdx.x];
+#pragma unroll
+  for (int j = 0; j < SCAN_I; ++j)
+    if (base + j < n) {
+      out[base + j] = e;
+      e += (int64_t)v[j];
+    }
+  if (blockIdx.x == 0 && threadIdx.x == 0) out[n] = bsum[nb];
+}
+
+// out[0..n] = exclusive scan of in[0..n), out[n] = total.  Returns nothing;
+// temp is a device buffer of >= nblocks+1 int64.
+template <typename T>
+void exclusive_scan(const T* in, int64_t n, int64_t* out, int64_t* temp, cudaStream_t s) {
+  int64_t nb = (n + SCAN_B - 1) / SCAN_B;
+  if (nb == 0) {
+    SPMV_CUDA(cudaMemsetAsync(out, 0, sizeof(int64_t), s));
+    return;
+  }
+  k_scan_reduce<T><<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, temp);
+  k_scan_top<<<1, 1024, 0, s>>>(temp, nb);
+  k_scan_down<T><<<(unsigned)nb, SCAN_T, 0, s>>>(in, n, temp, nb, out);
+  SPMV_LAUNCH_CHECK();
+}
+
+int64_t scan_temp_len(int64_t n) { return (n + SCAN_B - 1) / SCAN_B + 2; }
+
+// ---------------------------------------------------------------- partition
+__global__ void k_partition(const int64_t* rpB, int64_t n, int64_t nnz, int G, int64_t* b) {
+  int k = threadIdx.x;
+  if (k > G) return;
+  if (k == 0) { b[0] = 0; return; }
+  if (k == G) { b[G] = n; return; }
+  int64_t target = ((int64_t)k * nnz + G - 1) / G;
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    int64_t mid = (lo + hi) >> 1;
+    if (rpB[mid] >= target) hi = mid; else lo = mid + 1;
+  }
+  b[k] = lo;
+}
+
+template <typename OT>
+__global__ void k_local_rp(const int64_t* rpB, int64_t rb, int64_t nrows, OT* rp) {
+  int64_t base = rpB[rb];
+  GRID_STRIDE(i, nrows + 1) rp[i] = (OT)(rpB[rb + i] - base);
+}
+
+template <typename OT>
+__global__ void k_tiles(const OT* rp, int64_t nrows, int64_t K, int32_t* tiles) {
+  GRID_STRIDE(k, K + 1) {
+    int64_t target = k * (int64_t)TILE_D;
+    int64_t lo = 0, hi = nrows;
+    while (lo < hi) {
+      int64_t mid = (lo + hi) >> 1;
+      if ((int64_t)rp[mid] + mid >= target) hi = mid; else lo = mid + 1;
+    }
+    tiles[k] = (int32_t)lo;
+  }
+}
+
+// flags for a row-length predicate lo < L <= hi
+template <typename OT>
+__global__ void k_len_flag(const OT* rp, int64_t nrows, int64_t lo, int64_t hi, int32_t* f) {
+  GRID_STRIDE(r, nrows) {
+    int64_t L = (int64_t)rp[r + 1] - (int64_t)rp[r];
+    f[r] = (L > lo && L <= hi) ? 1 : 0;
+  }
+}
+
+__global__ void k_compact(const int32_t* f, const int64_t* pos, int64_t n, int32_t* out) {
+  GRID_STRIDE(i, n) if (f[i]) out[pos[i]] = (int32_t)i;
+}
+
+template <typename OT>
+__global__ void k_nchunks(const OT* rp, const int32_t* hub_rows, int64_t nh, int32_t* nch) {
+  GRID_STRIDE(h, nh) {
+    int r = hub_rows[h];
+    int64_t L = (int64_t)rp[r + 1] - (int64_t)rp[r];
+    nch[h] = (int32_t)((L + HUB_CHUNK - 1) / HUB_CHUNK);
+  }
+}
+
+template <typename OT>
+__global__ void k_row_len(const OT* rp, const int32_t* rows, int64_t nl, int64_t* len) {
+  GRID_STRIDE(t, nl) len[t] = (int64_t)rp[rows[t] + 1] - (int64_t)rp[rows[t]];
+}
+
+__global__ void k_chunks(const int32_t* hub_rows, const int32_t* nch, const int64_t* off,
+                         int64_t nh, int32_t* choff, int32_t* crow, int32_t* cidx) {
+  GRID_STRIDE(h, nh) {
+    int64_t o = off[h];
+    choff[h] = (int32_t)o;
+    for (int c = 0; c < nch[h]; ++c) {
+      crow[o + c] = hub_rows[h];
+      cidx[o + c] = c;
+    }
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) choff[nh] = (int32_t)off[nh];
+}
+
+// colcnt_B[perm[j]] = colcnt_A[j]: histogram of relabelled columns
+__global__ void k_colcnt(const int32_t* colA, const int32_t* perm, int64_t nnz, uint32_t* cnt) {
+  GRID_STRIDE(k, nnz) atomicAdd(&cnt[perm[colA[k]]], 1u);
+}
+
+__global__ void k_first_cold(const uint32_t* cnt, int64_t n, int64_t nnz,
+                             unsigned long long* H) {
+  GRID_STRIDE(j, n) {
+    if (!((int64_t)cnt[j] * n > nnz)) atomicMin(H, (unsigned long long)j);
+  }
+}
+
+// ------------------------------------------------------------- P A P^T data
+// warp per row for rows with L <= STREAM_MAX
+template <typename AT, typename OT>
+__global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* valA,
+                               const int32_t* perm, const int32_t* inv, int64_t rb,
+                               int64_t nrows, const OT* rpB, int32_t* colB, float* valB) {
+  const int lane = threadIdx.x & 31;
+  int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = w; r < nrows; r += nw) {
+    int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d;
+    if (L > STREAM_MAX) continue;
+    int64_t i = inv[rb + r];
+    int64_t a = (int64_t)rpA[i];
+    for (int64_t k = lane; k < L; k += 32) {
+      colB[d + k] = perm[colA[a + k]];
+      valB[d + k] = valA[a + k];
+    }
+  }
+}
+
+// CTA per long row (list)
+template <typename AT, typename OT>
+__global__ void k_relabel_cta(const AT* rpA, const int32_t* colA, const float* valA,
+                              const int32_t* perm, const int32_t* inv, int64_t rb,
+                              const int32_t* rows, int64_t nrows_list, const OT* rpB,
+                              int32_t* colB, float* valB) {
+  for (int64_t t = blockIdx.x; t < nrows_list; t += gridDim.x) {
+    int64_t r = rows[t];
+    int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d;
+    int64_t i = inv[rb + r];
+    int64_t a = (int64_t)rpA[i];
+    for (int64_t k = threadIdx.x; k < L; k += blockDim.x) {
+      colB[d + k] = perm[colA[a + k]];
+      valB[d + k] = valA[a + k];
+    }
+  }
+}
+
+// ----------------------------------------------------------------- row sort
+// Key (col_B << 32 | position in row) is unique inside a row, so any correct
+// sort by key is the stable sort by col_B (duplicates keep A's order).
+__device__ __forceinline__ uint64_t mkkey(int32_t c, int64_t rel) {
+  return ((uint64_t)(uint32_t)c << 32) | (uint64_t)(uint32_t)rel;
+}
+
+template <typename OT>
+__global__ void k_sort_warp(const OT* rp, int64_t nrows, int32_t* col, float* val) {
+  const int lane = threadIdx.x & 31;
+  int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = w; r < nrows; r += nw) {
+    int64_t d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d;
+    if (L < 2 || L > 32) continue;
+    uint64_t key = lane < L ? mkkey(col[d + lane], lane) : ~0ull;
+    float v = lane < L ? val[d + lane] : 0.f;
+#pragma unroll
+    for (int k = 2; k <= 32; k <<= 1) {
+#pragma unroll
+      for (int j = k >> 1; j > 0; j >>= 1) {
+        uint64_t ok = __shfl_xor_sync(0xffffffffu, key, j);
+        float ov = __shfl_xor_sync(0xffffffffu, v, j);
+        bool take_min = ((lane & j) == 0) == ((lane & k) == 0);
+        bool other_smaller = ok < key;
+        if (take_min == other_smaller) {
+          key = ok;
+          v = ov;
+        }
+      }
+    }
+    if (lane < L) {
+      col[d + lane] = (int32_t)(key >> 32);
+      val[d + lane] = v;
+    }
+  }
+}
+
+// CTA bitonic sort of one row of length L <= P held in shared memory.
+template <int P>
+__device__ void smem_bitonic(uint64_t* keys, float* vals) {
+#pragma unroll 1
+  for (int k = 2; k <= P; k <<= 1) {
+#pragma unroll 1
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < P; i += blockDim.x) {
+        int ixj = i ^ j;
+        if (ixj > i) {
+          uint64_t a = keys[i], b = keys[ixj];
+          bool asc = (i & k) == 0;
+          if ((a > b) == asc) {
+            keys[i] = b;
+            keys[ixj] = a;
+            float t = vals[i];
+            vals[i] = vals[ixj];
+            vals[ixj] = t;
+          }
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+
+template <int P, typename OT>
+__global__ void k_sort_cta(const OT* rp, const int32_t* rows, int64_t nlist, int32_t* col,
+                           float* val) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  uint64_t* keys = (uint64_t*)sm;
+  float* vals = (float*)(keys + P);
+  for (int64_t t = blockIdx.x; t < nlist; t += gridDim.x) {
+    int64_t r = rows[t];
+    int64_t d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d;
+    for (int i = threadIdx.x; i < P; i += blockDim.x) {
+      keys[i] = i < L ? mkkey(col[d + i], i) : ~0ull;
+      vals[i] = i < L ? val[d + i] : 0.f;
+    }
+    __syncthreads();
+    smem_bitonic<P>(keys, vals);
+    for (int i = threadIdx.x; i < L; i += blockDim.x) {
+      col[d + i] = (int32_t)(keys[i] >> 32);
+      val[d + i] = vals[i];
+    }
+    __syncthreads();
+  }
+}
+
+constexpr int BIG_CHUNK = 4096;
+
+// big rows: load keys into a scratch buffer at big_off[b]
+template <typename OT>
+__global__ void k_big_load(const OT* rp, const int32_t* rows, const int64_t* boff, int64_t nb,
+                           const int32_t* col, const float* val, uint64_t* K, float* V) {
+  for (int64_t b = blockIdx.x; b < nb; b += gridDim.x) {
+    int64_t r = rows[b], d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d, o = boff[b];
+    for (int64_t i = threadIdx.x; i < L; i += blockDim.x) {
+      K[o + i] = mkkey(col[d + i], i);
+      V[o + i] = val[d + i];
+    }
+  }
+}
+
+// sort every BIG_CHUNK-run of every big row in shared memory
+__global__ void k_big_chunk_sort(const int64_t* boff, int64_t nb, uint64_t* K, float* V) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  uint64_t* keys = (uint64_t*)sm;
+  float* vals = (float*)(keys + BIG_CHUNK);
+  int64_t b = blockIdx.x;
+  if (b >= nb) return;
+  int64_t o = boff[b], L = boff[b + 1] - o;
+  int64_t c0 = (int64_t)blockIdx.y * BIG_CHUNK;
+  if (c0 >= L) return;
+  int64_t m = min((int64_t)BIG_CHUNK, L - c0);
+  for (int i = threadIdx.x; i < BIG_CHUNK; i += blockDim.x) {
+    keys[i] = i < m ? K[o + c0 + i] : ~0ull;
+    vals[i] = i < m ? V[o + c0 + i] : 0.f;
+  }
+  __syncthreads();
+  smem_bitonic<BIG_CHUNK>(keys, vals);
+  for (int i = threadIdx.x; i < m; i += blockDim.x) {
+    K[o + c0 + i] = keys[i];
+    V[o + c0 + i] = vals[i];
+  }
+}
+
+// one merge pass of width w over all big rows: element-wise rank merge
+__global__ void k_big_merge(const int64_t* boff, int64_t nb, int64_t total, int64_t w,
+                            const uint64_t* K, const float* V, uint64_t* K2, float* V2) {
+  GRID_STRIDE(e, total) {
+    int64_t lo = 0, hi = nb;  // find b with boff[b] <= e < boff[b+1]
+    while (hi - lo > 1) {
+      int64_t mid = (lo + hi) >> 1;
+      if (boff[mid] <= e) lo = mid; else hi = mid;
+    }
+    int64_t o = boff[lo], L = boff[lo + 1] - o, rel = e - o;
+    int64_t run = rel / w, base = (run & ~1ll) * w;
+    uint64_t key = K[e];
+    int64_t out;
+    if ((run & 1) == 0) {
+      int64_t b0 = base + w, b1 = min(base + 2 * w, L);
+      int64_t cnt = 0;
+      if (b0 < b1) {  // count keys in B less than key
+        int64_t l = b0, h = b1;
+        while (l < h) {
+          int64_t mid = (l + h) >> 1;
+          if (K[o + mid] < key) l = mid + 1; else h = mid;
+        }
+        cnt = l - b0;
+      }
+      out = base + (rel - base) + cnt;
+    } else {
+      int64_t a0 = base, a1 = base + w;
+      int64_t l = a0, h = a1;
+      while (l < h) {
+        int64_t mid = (l + h) >> 1;
+        if (K[o + mid] < key) l = mid + 1; else h = mid;
+      }
+      out = base + (rel - base - w) + (l - a0);
+    }
+    K2[o + out] = key;
+    V2[o + out] = V[e];
+  }
+}
+
+template <typename OT>
+__global__ void k_big_store(const OT* rp, const int32_t* rows, const int64_t* boff, int64_t nb,
+                            const uint64_t* K, const float* V, int32_t* col, float* val) {
+  for (int64_t b = blockIdx.x; b < nb; b += gridDim.x) {
+    int64_t r = rows[b], d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d, o = boff[b];
+    for (int64_t i = threadIdx.x; i < L; i += blockDim.x) {
+      col[d + i] = (int32_t)(K[o + i] >> 32);
+      val[d + i] = V[o + i];
+    }
+  }
+}
+
+// world > 1: global column -> padded x layout (monotone, keeps row order)
+__global__ void k_pad_cols(int32_t* col, int64_t nnz, const int64_t* part, int G, int64_t M) {
+  GRID_STRIDE(k, nnz) {
+    int64_t c = col[k];
+    int lo = 0, hi = G;  // owner: part[o] <= c < part[o+1]
+    while (hi - lo > 1) {
+      int mid = (lo + hi) >> 1;
+      if (part[mid] <= c) lo = mid; else hi = mid;
+    }
+    col[k] = (int32_t)(lo * M + (c - part[lo]));
+  }
+}
+
+__global__ void k_permute_vec(const int32_t* perm, int64_t n, const float* in, float* out,
+                              int inverse) {
+  GRID_STRIDE(i, n) {
+    if (inverse) out[i] = in[perm[i]];
+    else out[perm[i]] = in[i];
+  }
+}
+
+__global__ void k_pad_vec(const int64_t* part, int G, int64_t M, int64_t n, const float* in,
+                          float* out, int to_padded) {
+  GRID_STRIDE(i, n) {
+    int lo = 0, hi = G;
+    while (hi - lo > 1) {
+      int mid = (lo + hi) >> 1;
+      if (part[mid] <= i) lo = mid; else hi = mid;
+    }
+    int64_t j = lo * M + (i - part[lo]);
+    if (to_padded) out[j] = in[i];
+    else out[i] = in[j];
+  }
+}
+
+// ------------------------------------------------------------- host helpers
+template <typename T>
+T* dalloc(int64_t n) {
+  void* p = nullptr;
+  size_t bytes = sizeof(T) * (size_t)std::max<int64_t>(n, 1);
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    SPMV_FAIL(SPMV_ENOMEM, "cudaMalloc of " + std::to_string(bytes) + " bytes failed: " +
+                               cudaGetErrorString(e));
+  }
+  return (T*)p;
+}
+
+template <typename T>
+void dfree(T*& p) {
+  if (p) cudaFree((void*)p);
+  p = nullptr;
+}
+
+template <typename T>
+T d2h_one(const T* d, cudaStream_t s) {
+  T h;
+  SPMV_CUDA(cudaMemcpyAsync(&h, d, sizeof(T), cudaMemcpyDeviceToHost, s));
+  SPMV_CUDA(cudaStreamSynchronize(s));
+  return h;
+}
+
+// flags -> ascending list of rows; returns count
+template <typename OT>
+int64_t class_list(const OT* rp, int64_t nrows, int64_t lo, int64_t hi, int32_t** out,
+                   int32_t* f, int64_t* pos, int64_t* tmp, cudaStream_t s) {
+  k_len_flag<OT><<<grid_for(nrows), TPB, 0, s>>>(rp, nrows, lo, hi, f);
+  exclusive_scan<int32_t>(f, nrows, pos, tmp, s);
+  int64_t cnt = d2h_one(pos + nrows, s);
+  *out = dalloc<int32_t>(cnt);
+  if (cnt) k_compact<<<grid_for(nrows), TPB, 0, s>>>(f, pos, nrows, *out);
+  SPMV_LAUNCH_CHECK();
+  return cnt;
+}
+
+}  // namespace
+
+template <typename AT, typename OT>
+static void build_typed(spmv_plan_s* p, const AT* rpA) {
+  cudaStream_t s = p->s;
+  const int64_t n = p->n, nnz = p->nnz;
+  int* d_flags = dalloc<int>(4);
+  SPMV_CUDA(cudaMemsetAsync(d_flags, 0, 4 * sizeof(int), s));
+  k_validate_rp<AT><<<grid_for(n), TPB, 0, s>>>(rpA, n, nnz, d_flags);
+  k_validate_col<<<grid_for(nnz), TPB, 0, s>>>(p->A_col, nnz, n, d_flags);
+  SPMV_LAUNCH_CHECK();
+  int h_flags[4];
+  SPMV_CUDA(cudaMemcpyAsync(h_flags, d_flags, sizeof(h_flags), cudaMemcpyDeviceToHost, s));
+  SPMV_CUDA(cudaStreamSynchronize(s));
+  if (h_flags[0]) { dfree(d_flags); SPMV_FAIL(SPMV_EINVAL, "row_ptr is not a valid CSR row pointer (row_ptr[0]=0, non-decreasing, row_ptr[n]=nnz)"); }
+  if (h_flags[1]) { dfree(d_flags); SPMV_FAIL(SPMV_EINVAL, "column index out of range [0, n)"); }
+
+  // inverse permutation + bijection check
+  k_fill_i32<<<grid_for(n), TPB, 0, s>>>(p->d_inv, n, -1);
+  k_inverse<<<grid_for(n), TPB, 0, s>>>(p->d_perm, n, p->d_inv, d_flags);
+  SPMV_LAUNCH_CHECK();
+  int eperm = d2h_one(d_flags + 2, s);
+  dfree(d_flags);
+  if (eperm) SPMV_FAIL(SPMV_EPERM, "perm is not a bijection on [0, n)");
+
+  // full row pointer of B
+  int64_t* lenB = dalloc<int64_t>(n);
+  int64_t* rpB = dalloc<int64_t>(n + 1);
+  int64_t* tmp = dalloc<int64_t>(scan_temp_len(std::max<int64_t>(n, 1)));
+  k_lenB<AT><<<grid_for(n), TPB, 0, s>>>(rpA, p->d_perm, n, lenB);
+  exclusive_scan<int64_t>(lenB, n, rpB, tmp, s);
+  dfree(lenB);
+
+  // partition: b_k = lower_bound(row_ptr_B, ceil(k NZ / G))
+  int64_t* d_part = dalloc<int64_t>(p->world + 1);
+  k_partition<<<1, 1024, 0, s>>>(rpB, n, nnz, p->world, d_part);
+  p->part.assign(p->world + 1, 0);
+  SPMV_CUDA(cudaMemcpyAsync(p->part.data(), d_part, sizeof(int64_t) * (p->world + 1),
+                            cudaMemcpyDeviceToHost, s));
+  SPMV_CUDA(cudaStreamSynchronize(s));
+  dfree(d_part);
+  p->row_begin = p->part[p->rank];
+  p->row_end = p->part[p->rank + 1];
+  p->nrows = p->row_end - p->row_begin;
+  int64_t lo_nz, hi_nz;
+  SPMV_CUDA(cudaMemcpyAsync(&lo_nz, rpB + p->row_begin, 8, cudaMemcpyDeviceToHost, s));
+  SPMV_CUDA(cudaMemcpyAsync(&hi_nz, rpB + p->row_end, 8, cudaMemcpyDeviceToHost, s));
+  SPMV_CUDA(cudaStreamSynchronize(s));
+  p->nnz_before = lo_nz;
+  p->nnz_local = hi_nz - lo_nz;
+  if (p->world > 1) {
+    int64_t M = 0;
+    for (int k = 0; k < p->world; ++k) M = std::max<int64_t>(M, p->part[k + 1] - p->part[k]);
+    M = (M + 31) / 32 * 32;
+    if ((int64_t)p->world * M > (int64_t)INT32_MAX)
+      SPMV_FAIL(SPMV_EUNSUPPORTED, "padded x layout exceeds int32 column range");
+    p->x_stride = M;
+    p->x_len = (int64_t)p->world * M;
+    p->y_offset = (int64_t)p->rank * M;
+  } else {
+    p->x_stride = n;
+    p->x_len = n;
+    p->y_offset = 0;
+  }
+
+  // local row pointer
+  const int64_t nr = p->nrows;
+  OT* rp = dalloc<OT>(nr + 1);
+  p->d_rp = rp;
+  k_local_rp<OT><<<grid_for(nr + 1), TPB, 0, s>>>(rpB, p->row_begin, nr, rp);
+  SPMV_LAUNCH_CHECK();
+
+  // hot prefix H over the full B
+  uint32_t* cnt = (uint32_t*)dalloc<uint32_t>(n);
+  SPMV_CUDA(cudaMemsetAsync(cnt, 0, sizeof(uint32_t) * std::max<int64_t>(n, 1), s));
+  unsigned long long* dH = dalloc<unsigned long long>(1);
+  unsigned long long hinit = (unsigned long long)n;
+  SPMV_CUDA(cudaMemcpyAsync(dH, &hinit, 8, cudaMemcpyHostToDevice, s));
+  if (nnz) k_colcnt<<<grid_for(nnz), TPB, 0, s>>>(p->A_col, p->d_perm, nnz, cnt);
+  if (n) k_first_cold<<<grid_for(n), TPB, 0, s>>>(cnt, n, nnz, dH);
+  SPMV_LAUNCH_CHECK();
+  p->H = (int64_t)d2h_one(dH, s);
+  dfree(dH);
+  dfree(cnt);
+  dfree(rpB);
+
+  // tiles
+  p->K = nr ? (p->nnz_local + nr + TILE_D - 1) / TILE_D : 0;
+  p->d_tiles = dalloc<int32_t>(p->K + 1);
+  k_tiles<OT><<<grid_for(p->K + 1), TPB, 0, s>>>(rp, nr, p->K, p->d_tiles);
+  SPMV_LAUNCH_CHECK();
+
+  // row classes + sort buckets
+  int32_t* f = dalloc<int32_t>(nr);
+  int64_t* pos = dalloc<int64_t>(nr + 1);
+  dfree(tmp);
+  tmp = dalloc<int64_t>(scan_temp_len(std::max<int64_t>(nr, 1)));
+  p->n_cta = class_list<OT>(rp, nr, STREAM_MAX, CTA_MAX, &p->d_cta_rows, f, pos, tmp, s);
+  p->n_hub = class_list<OT>(rp, nr, CTA_MAX, INT64_MAX, &p->d_hub_rows, f, pos, tmp, s);
+  spmv_plan_s* ps = p;
+  ps->n1 = class_list<OT>(rp, nr, 32, 128, &ps->s1, f, pos, tmp, s);
+  ps->n2 = class_list<OT>(rp, nr, 128, 1024, &ps->s2, f, pos, tmp, s);
+  ps->n3 = class_list<OT>(rp, nr, 1024, BIG_CHUNK, &ps->s3, f, pos, tmp, s);
+  ps->nbig = class_list<OT>(rp, nr, BIG_CHUNK, INT64_MAX, &ps->big, f, pos, tmp, s);
+  ps->nlong = class_list<OT>(rp, nr, STREAM_MAX, INT64_MAX, &ps->longrows, f, pos, tmp, s);
+  // big row offsets in the key scratch
+  ps->boff = dalloc<int64_t>(ps->nbig + 1);
+  if (ps->nbig) {
+    int64_t* blen = dalloc<int64_t>(ps->nbig);
+    int64_t* t3 = dalloc<int64_t>(scan_temp_len(ps->nbig));
+    k_row_len<OT><<<grid_for(ps->nbig), TPB, 0, s>>>(rp, ps->big, ps->nbig, blen);
+    exclusive_scan<int64_t>(blen, ps->nbig, ps->boff, t3, s);
+    std::vector<int64_t> hl(ps->nbig);
+    SPMV_CUDA(cudaMemcpyAsync(hl.data(), blen, 8 * ps->nbig, cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA(cudaStreamSynchronize(s));
+    for (int64_t L : hl) { ps->big_total += L; ps->big_max = std::max(ps->big_max, L); }
+    dfree(blen);
+    dfree(t3);
+  } else {
+    SPMV_CUDA(cudaMemsetAsync(ps->boff, 0, 8, s));
+  }
+  // hub chunks
+  p->d_hub_choff = dalloc<int32_t>(p->n_hub + 1);
+  if (p->n_hub) {
+    int32_t* nch = dalloc<int32_t>(p->n_hub);
+    int64_t* off = dalloc<int64_t>(p->n_hub + 1);
+    int64_t* t2 = dalloc<int64_t>(scan_temp_len(p->n_hub));
+    k_nchunks<OT><<<grid_for(p->n_hub), TPB, 0, s>>>(rp, p->d_hub_rows, p->n_hub, nch);
+    exclusive_scan<int32_t>(nch, p->n_hub, off, t2, s);
+    p->n_chunks = d2h_one(off + p->n_hub, s);
+    p->d_chunk_row = dalloc<int32_t>(p->n_chunks);
+    p->d_chunk_idx = dalloc<int32_t>(p->n_chunks);
+    k_chunks<<<grid_for(p->n_hub), TPB, 0, s>>>(p->d_hub_rows, nch, off, p->n_hub,
+                                                  p->d_hub_choff, p->d_chunk_row, p->d_chunk_idx);
+    SPMV_LAUNCH_CHECK();
+    dfree(nch);
+    dfree(off);
+    dfree(t2);
+  } else {
+    SPMV_CUDA(cudaMemsetAsync(p->d_hub_choff, 0, 4, s));
+  }
+  dfree(f);
+  dfree(pos);
+  dfree(tmp);
+
+  // local B storage (+8 elements of zero padding for 16-byte bulk copies)
+  p->d_col = dalloc<int32_t>(p->nnz_local + 8);
+  p->d_val = dalloc<float>(p->nnz_local + 8);
+  SPMV_CUDA(cudaMemsetAsync(p->d_col + p->nnz_local, 0, 32, s));
+  SPMV_CUDA(cudaMemsetAsync(p->d_val + p->nnz_local, 0, 32, s));
+  // exec scratch
+  p->d_chunk_part = dalloc<double>(p->n_chunks);
+  p->d_tile_ss = dalloc<double>(p->K);
+  p->d_cta_ss = dalloc<double>(p->n_cta);
+  p->d_hub_ss = dalloc<double>(p->n_hub);
+  p->d_ss = dalloc<double>(4);
+  SPMV_CUDA(cudaStreamSynchronize(s));
+}
+
+template <typename AT, typename OT>
+static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
+  OT* rp = (OT*)p->d_rp;
+  spmv_plan_s* ps = p;
+  const int64_t nr = p->nrows;
+  if (nr) {
+    k_relabel_warp<AT, OT><<<grid_for(nr * 32), TPB, 0, s>>>(
+        rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, nr, rp, p->d_col, p->d_val);
+    if (ps->nlong)
+      k_relabel_cta<AT, OT><<<(unsigned)std::min<int64_t>(ps->nlong, 148 * 8), 512, 0, s>>>(
+          rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, ps->longrows, ps->nlong,
+          rp, p->d_col, p->d_val);
+    k_sort_warp<OT><<<grid_for(nr * 32), TPB, 0, s>>>(rp, nr, p->d_col, p->d_val);
+    SPMV_LAUNCH_CHECK();
+    if (ps->n1) {
+      k_sort_cta<128, OT><<<(unsigned)std::min<int64_t>(ps->n1, 148 * 64), 64, 128 * 12, s>>>(
+          rp, ps->s1, ps->n1, p->d_col, p->d_val);
+    }
+    if (ps->n2) {
+      k_sort_cta<1024, OT><<<(unsigned)std::min<int64_t>(ps->n2, 148 * 16), 256, 1024 * 12, s>>>(
+          rp, ps->s2, ps->n2, p->d_col, p->d_val);
+    }
+    if (ps->n3) {
+      k_sort_cta<4096, OT><<<(unsigned)std::min<int64_t>(ps->n3, 148 * 4), 512, 4096 * 12, s>>>(
+          rp, ps->s3, ps->n3, p->d_col, p->d_val);
+    }
+    SPMV_LAUNCH_CHECK();
+    if (ps->nbig) {
+      uint64_t* K1 = dalloc<uint64_t>(ps->big_total);
+      uint64_t* K2 = dalloc<uint64_t>(ps->big_total);
+      float* V1 = dalloc<float>(ps->big_total);
+      float* V2 = dalloc<float>(ps->big_total);
+      unsigned nb = (unsigned)std::min<int64_t>(ps->nbig, 148 * 8);
+      k_big_load<OT><<<nb, 512, 0, s>>>(rp, ps->big, ps->boff, ps->nbig, p->d_col, p->d_val, K1, V1);
+      dim3 g((unsigned)ps->nbig, (unsigned)((ps->big_max + BIG_CHUNK - 1) / BIG_CHUNK));
+      k_big_chunk_sort<<<g, 512, BIG_CHUNK * 12, s>>>(ps->boff, ps->nbig, K1, V1);
+      SPMV_LAUNCH_CHECK();
+      for (int64_t w = BIG_CHUNK; w < ps->big_max; w *= 2) {
+        k_big_merge<<<grid_for(ps->big_total), TPB, 0, s>>>(ps->boff, ps->nbig, ps->big_total, w,
+                                                            K1, V1, K2, V2);
+        std::swap(K1, K2);
+        std::swap(V1, V2);
+      }
+      k_big_store<OT><<<nb, 512, 0, s>>>(rp, ps->big, ps->boff, ps->nbig, K1, V1, p->d_col, p->d_val);
+      SPMV_LAUNCH_CHECK();
+      SPMV_CUDA(cudaStreamSynchronize(s));  // scratch lifetime
+      dfree(K1); dfree(K2); dfree(V1); dfree(V2);
+    }
+  }
+  if (p->world > 1 && p->nnz_local) {
+    int64_t* d_part = dalloc<int64_t>(p->world + 1);
+    SPMV_CUDA(cudaMemcpyAsync(d_part, p->part.data(), 8 * (p->world + 1), cudaMemcpyHostToDevice, s));
+    k_pad_cols<<<grid_for(p->nnz_local), TPB, 0, s>>>(p->d_col, p->nnz_local, d_part, p->world,
+                                                      p->x_stride);
+    SPMV_LAUNCH_CHECK();
+    SPMV_CUDA(cudaStreamSynchronize(s));
+    dfree(d_part);
+  }
+}
+
+// ------------------------------------------------------------------ public
+void plan_build(spmv_plan_s* p, const spmv_csr_t* A, const int32_t* perm) {
+  const int64_t n = p->n;
+  p->d_perm = dalloc<int32_t>(n);
+  p->d_inv = dalloc<int32_t>(n);
+  if (perm) {
+    SPMV_CUDA(cudaMemcpyAsync(p->d_perm, perm, 4 * std::max<int64_t>(n, 0), cudaMemcpyDeviceToDevice, p->s));
+  } else {
+    k_identity<<<grid_for(n), TPB, 0, p->s>>>(p->d_perm, n);
+    SPMV_LAUNCH_CHECK();
+  }
+  if (A->row_ptr64) {
+    if (p->off64) build_typed<int64_t, int64_t>(p, A->row_ptr64);
+    else build_typed<int64_t, int32_t>(p, A->row_ptr64);
+  } else {
+    if (p->off64) build_typed<int32_t, int64_t>(p, A->row_ptr32);
+    else build_typed<int32_t, int32_t>(p, A->row_ptr32);
+  }
+}
+
+void plan_permute(spmv_plan_s* p, cudaStream_t s) {
+  if (p->A_rp64) {
+    if (p->off64) permute_typed<int64_t, int64_t>(p, p->A_rp64, s);
+    else permute_typed<int64_t, int32_t>(p, p->A_rp64, s);
+  } else {
+    if (p->off64) permute_typed<int32_t, int64_t>(p, p->A_rp32, s);
+    else permute_typed<int32_t, int32_t>(p, p->A_rp32, s);
+  }
+  p->permuted = true;
+}
+
+void permute_vec(spmv_plan_s* p, const float* in, float* out, int inverse, cudaStream_t s) {
+  if (p->n == 0) return;
+  k_permute_vec<<<grid_for(p->n), TPB, 0, s>>>(p->d_perm, p->n, in, out, inverse);
+  SPMV_LAUNCH_CHECK();
+}
+
+void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStream_t s) {
+  if (p->n == 0) return;
+  int64_t* d_part = dalloc<int64_t>(p->world + 1);
+  SPMV_CUDA(cudaMemcpyAsync(d_part, p->part.data(), 8 * (p->world + 1), cudaMemcpyHostToDevice, s));
+  k_pad_vec<<<grid_for(p->n), TPB, 0, s>>>(d_part, p->world, p->x_stride, p->n, in, out, to_padded);
+  SPMV_LAUNCH_CHECK();
+  SPMV_CUDA(cudaStreamSynchronize(s));
+  dfree(d_part);
+}
+
+void plan_free(spmv_plan_s* p) {
+  dfree(p->s1); dfree(p->s2); dfree(p->s3); dfree(p->big); dfree(p->boff);
+  dfree(p->longrows);
+  dfree(p->d_perm); dfree(p->d_inv);
+  if (p->d_rp) { cudaFree(p->d_rp); p->d_rp = nullptr; }
+  dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows);
+  dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
+  dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
+  dfree(p->d_ss); dfree(p->d_u);
+}
+
+}  // namespace spmv

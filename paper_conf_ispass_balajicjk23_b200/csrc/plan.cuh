@@ -1,0 +1,79 @@
+// Plan object (owned device buffers) — internal.
+#pragma once
+#include <vector>
+
+#include "common.cuh"
+
+struct spmv_plan_s {
+  int device = 0;
+  spmv_opts_t opts{};
+  cudaStream_t s = nullptr;  // internal stream for the synchronous plan phase
+
+  // global problem
+  int64_t n = 0, nnz = 0;
+  bool off64 = false;  // local row_ptr stored as int64 (global nnz >= 2^31)
+
+  // borrowed input (valid until spmv_permute completes)
+  const int32_t* A_rp32 = nullptr;
+  const int64_t* A_rp64 = nullptr;
+  const int32_t* A_col = nullptr;
+  const float* A_val = nullptr;
+
+  // owned: permutation
+  int32_t* d_perm = nullptr;  // perm[old] = new (identity if none given)
+  int32_t* d_inv = nullptr;   // inv[new] = old
+
+  // partition
+  int world = 1, rank = 0;
+  std::vector<int64_t> part;  // b_0..b_world (global rows)
+  int64_t row_begin = 0, row_end = 0, nrows = 0, nnz_local = 0, nnz_before = 0;
+  int64_t x_len = 0, x_stride = 0, y_offset = 0;
+
+  // owned: local block of B
+  void* d_rp = nullptr;        // int32 or int64 [nrows+1], local offsets
+  int32_t* d_col = nullptr;    // [nnz_local + pad]
+  float* d_val = nullptr;      // [nnz_local + pad]
+
+  // bins
+  int64_t K = 0, n_cta = 0, n_hub = 0, n_chunks = 0, H = 0, max_hub_len = 0;
+  int32_t* d_tiles = nullptr;      // [K+1]
+  int32_t* d_cta_rows = nullptr;   // [n_cta]
+  int32_t* d_hub_rows = nullptr;   // [n_hub]
+  int32_t* d_hub_choff = nullptr;  // [n_hub+1] first chunk of each hub row
+  int32_t* d_chunk_row = nullptr;  // [n_chunks]
+  int32_t* d_chunk_idx = nullptr;  // [n_chunks]
+
+  // exec scratch
+  double* d_chunk_part = nullptr;  // [n_chunks]
+  double* d_tile_ss = nullptr;     // [K]
+  double* d_cta_ss = nullptr;      // [n_cta]
+  double* d_hub_ss = nullptr;      // [n_hub]
+  double* d_ss = nullptr;          // [4] iterate scalars
+  float* d_u = nullptr;            // iterate ping-pong [x_len]
+
+  // permute-phase sort buckets (ascending local rows)
+  int32_t* s1 = nullptr; int64_t n1 = 0;        // 32 < L <= 128
+  int32_t* s2 = nullptr; int64_t n2 = 0;        // 128 < L <= 1024
+  int32_t* s3 = nullptr; int64_t n3 = 0;        // 1024 < L <= 4096
+  int32_t* big = nullptr; int64_t nbig = 0;     // L > 4096 (chunk sort + merges)
+  int64_t* boff = nullptr; int64_t big_total = 0, big_max = 0;
+  int32_t* longrows = nullptr; int64_t nlong = 0;  // L > STREAM_MAX
+
+  // state
+  bool permuted = false;
+  int64_t l2_window_bytes = 0;
+  const void* win_ptr = nullptr;
+  cudaStream_t win_stream = nullptr;
+};
+
+namespace spmv {
+void plan_build(spmv_plan_s* p, const spmv_csr_t* A, const int32_t* perm);
+void plan_permute(spmv_plan_s* p, cudaStream_t s);
+void plan_free(spmv_plan_s* p);
+void permute_vec(spmv_plan_s* p, const float* in, float* out, int inverse, cudaStream_t s);
+void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStream_t s);
+void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
+          cudaStream_t s);
+void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s);
+void scale_vec(const float* u, float* x, int64_t n, const double* ss, cudaStream_t s);
+}  // namespace spmv

@@ -1,0 +1,409 @@
+// spmv_reorder: host reordering (input preparation, timed separately).
+//
+// RABBIT (PAPER.md:86 §IV-A, :130 §V-A; Rabbit Order, ref [1] PAPER.md:259):
+// modularity-maximising incremental aggregation, then community members get
+// consecutive IDs by a DFS of the merge dendrogram.  The paper gives no
+// algorithm; the deterministic reading (DESIGN.md
+// §Readings) is implemented here sequentially so that it is reproducible bit
+// for bit:
+//   S = Bp + Bp^T over the off-diagonal 0/1 pattern; visit vertices in
+//   ascending (deg, id); for u: aggregate u's S-row with the lists of the
+//   children merged so far, map neighbours to their union-find roots, sum
+//   weights per root, drop u; dQ' = 2m w_uv - tot_u tot_v (exact __int128);
+//   merge into argmax (ties -> smallest root) iff dQ' > 0; else top level.
+//   IDs: pre-order DFS from each top-level root in append order, children
+//   in merge order.
+// RABBIT++ (§VI-A): insular nodes (all S-neighbours in the
+// same top-level community) grouped last, non-insular hubs (colcount*N > NZ)
+// grouped first, RABBIT's relative order kept inside each group.
+#include <omp.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "../../include/spmv.h"
+
+namespace spmv {
+void set_error(const std::string& m);
+}
+
+namespace {
+
+struct Sym {  // S = Bp + Bp^T in CSR, weights 1 or 2
+  int64_t n = 0;
+  std::vector<int64_t> ptr;
+  std::vector<int32_t> idx;
+  std::vector<uint8_t> w;
+};
+
+void scan_inplace(std::vector<int64_t>& v) {  // exclusive, v has n+1 slots
+  int64_t acc = 0;
+  for (auto& x : v) {
+    int64_t t = x;
+    x = acc;
+    acc += t;
+  }
+}
+
+Sym symmetrize(int64_t n, const int64_t* rp, const int32_t* col) {
+  // Bp: per row sorted unique off-diagonal columns
+  std::vector<int64_t> bl(n + 1, 0);
+  std::vector<int32_t> bidx((size_t)rp[n]);
+#pragma omp parallel for schedule(dynamic, 1024)
+  for (int64_t i = 0; i < n; ++i) {
+    int32_t* b = bidx.data() + rp[i];
+    int64_t m = 0;
+    for (int64_t k = rp[i]; k < rp[i + 1]; ++k)
+      if (col[k] != i) b[m++] = col[k];
+    std::sort(b, b + m);
+    bl[i] = std::unique(b, b + m) - b;
+  }
+  // transpose counts
+  std::vector<int64_t> tcnt(n + 1, 0);
+  for (int64_t i = 0; i < n; ++i)
+    for (int64_t k = 0; k < bl[i]; ++k) tcnt[bidx[rp[i] + k]]++;
+  std::vector<int64_t> tptr(tcnt);
+  scan_inplace(tptr);
+  std::vector<int32_t> tidx((size_t)tptr[n]);
+  {
+    std::vector<int64_t> cur(tptr.begin(), tptr.end() - 1);
+    for (int64_t i = 0; i < n; ++i)  // rows ascending -> transposed rows sorted
+      for (int64_t k = 0; k < bl[i]; ++k) tidx[cur[bidx[rp[i] + k]]++] = (int32_t)i;
+  }
+  // merge row i of Bp and Bp^T
+  Sym S;
+  S.n = n;
+  S.ptr.assign(n + 1, 0);
+#pragma omp parallel for schedule(dynamic, 1024)
+  for (int64_t i = 0; i < n; ++i) {
+    const int32_t *a = bidx.data() + rp[i], *ae = a + bl[i];
+    const int32_t *b = tidx.data() + tptr[i], *be = tidx.data() + tptr[i + 1];
+    int64_t m = 0;
+    while (a < ae || b < be) {
+      if (b == be || (a < ae && *a < *b)) ++a;
+      else if (a == ae || *b < *a) ++b;
+      else { ++a; ++b; }
+      ++m;
+    }
+    S.ptr[i] = m;
+  }
+  scan_inplace(S.ptr);
+  S.idx.resize((size_t)S.ptr[n]);
+  S.w.resize((size_t)S.ptr[n]);
+#pragma omp parallel for schedule(dynamic, 1024)
+  for (int64_t i = 0; i < n; ++i) {
+    const int32_t *a = bidx.data() + rp[i], *ae = a + bl[i];
+    const int32_t *b = tidx.data() + tptr[i], *be = tidx.data() + tptr[i + 1];
+    int64_t o = S.ptr[i];
+    while (a < ae || b < be) {
+      if (b == be || (a < ae && *a < *b)) { S.idx[o] = *a++; S.w[o++] = 1; }
+      else if (a == ae || *b < *a) { S.idx[o] = *b++; S.w[o++] = 1; }
+      else { S.idx[o] = *a; S.w[o++] = 2; ++a; ++b; }
+    }
+  }
+  return S;
+}
+
+struct Edge {
+  int32_t v;
+  int64_t w;
+};
+
+struct Rabbit {
+  std::vector<int32_t> perm, comm;
+  int64_t two_m = 0, n_merges = 0, n_top = 0;
+};
+
+Rabbit rabbit_detect(const Sym& S) {
+  const int64_t n = S.n;
+  std::vector<int64_t> deg(n);
+#pragma omp parallel for schedule(static)
+  for (int64_t v = 0; v < n; ++v) {
+    int64_t d = 0;
+    for (int64_t k = S.ptr[v]; k < S.ptr[v + 1]; ++k) d += S.w[k];
+    deg[v] = d;
+  }
+  int64_t two_m = 0;
+  for (int64_t v = 0; v < n; ++v) two_m += deg[v];
+  // ascending (deg, id): stable counting sort by degree
+  int64_t maxd = 0;
+  for (int64_t v = 0; v < n; ++v) maxd = std::max(maxd, deg[v]);
+  std::vector<int64_t> order(n);
+  {
+    std::vector<int64_t> c(maxd + 2, 0);
+    for (int64_t v = 0; v < n; ++v) c[deg[v] + 1]++;
+    for (int64_t d = 0; d <= maxd; ++d) c[d + 1] += c[d];
+    for (int64_t v = 0; v < n; ++v) order[c[deg[v]]++] = v;
+  }
+  std::vector<int32_t> parent(n);
+  std::iota(parent.begin(), parent.end(), 0);
+  auto find = [&](int32_t v) {
+    int32_t r = v;
+    while (parent[r] != r) r = parent[r];
+    while (parent[v] != r) {
+      int32_t nx = parent[v];
+      parent[v] = r;
+      v = nx;
+    }
+    return r;
+  };
+  std::vector<int64_t> tot(deg);
+  std::vector<int32_t> first_child(n, -1), last_child(n, -1), next_sib(n, -1);
+  std::vector<std::vector<Edge>> agg(n);
+  std::vector<int64_t> acc(n, 0);
+  std::vector<int32_t> touched;
+  std::vector<int32_t> top;
+  Rabbit R;
+  R.two_m = two_m;
+  for (int64_t oi = 0; oi < n; ++oi) {
+    const int32_t u = (int32_t)order[oi];
+    touched.clear();
+    auto add = [&](int32_t w, int64_t wt) {
+      int32_t r = find(w);
+      if (r == u) return;
+      if (acc[r] == 0) touched.push_back(r);
+      acc[r] += wt;
+    };
+    for (int64_t k = S.ptr[u]; k < S.ptr[u + 1]; ++k) add(S.idx[k], S.w[k]);
+    for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) {
+      for (const Edge& e : agg[c]) add(e.v, e.w);
+      std::vector<Edge>().swap(agg[c]);
+    }
+    int32_t best = -1;
+    __int128 bestdq = 0;
+    for (int32_t r : touched) {
+      __int128 dq = (__int128)two_m * acc[r] - (__int128)tot[u] * tot[r];
+      if (best == -1 || dq > bestdq || (dq == bestdq && r < best)) {
+        best = r;
+        bestdq = dq;
+      }
+    }
+    if (best != -1 && bestdq > 0) {
+      parent[u] = best;
+      tot[best] += tot[u];
+      if (last_child[best] == -1) first_child[best] = u;
+      else next_sib[last_child[best]] = u;
+      last_child[best] = u;
+      agg[u].reserve(touched.size());
+      for (int32_t r : touched) agg[u].push_back({r, acc[r]});
+      R.n_merges++;
+    } else {
+      top.push_back(u);
+    }
+    for (int32_t r : touched) acc[r] = 0;
+  }
+  // pre-order DFS of the dendrogram
+  R.perm.assign(n, -1);
+  R.comm.assign(n, -1);
+  int32_t nxt = 0;
+  std::vector<int32_t> st;
+  for (int32_t r : top) {
+    st.push_back(r);
+    while (!st.empty()) {
+      int32_t x = st.back();
+      st.pop_back();
+      R.perm[x] = nxt++;
+      R.comm[x] = r;
+      // push children in reverse merge order so they pop in merge order
+      size_t mark = st.size();
+      for (int32_t c = first_child[x]; c != -1; c = next_sib[c]) st.push_back(c);
+      std::reverse(st.begin() + mark, st.end());
+    }
+  }
+  R.n_top = (int64_t)top.size();
+  return R;
+}
+
+inline uint64_t mix64(uint64_t z) {
+  z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+  z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+  return z ^ (z >> 31);
+}
+
+void random_order(int64_t n, uint64_t seed, int32_t* perm) {
+  std::vector<int32_t> p(n);
+  std::iota(p.begin(), p.end(), 0);
+  for (int64_t i = n - 1; i > 0; --i) {
+    uint64_t h = mix64(seed + 0x9E3779B97F4A7C15ull * (uint64_t)(i + 1));
+    int64_t j = (int64_t)(h % (uint64_t)(i + 1));
+    std::swap(p[i], p[j]);
+  }
+  std::memcpy(perm, p.data(), sizeof(int32_t) * n);
+}
+
+}  // namespace
+
+static thread_local std::vector<int32_t> g_last_comm;
+
+extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, const int32_t* col,
+                                    int method, uint64_t seed, int32_t* perm_out,
+                                    spmv_reorder_stats_t* st) {
+  try {
+    auto t0 = std::chrono::steady_clock::now();
+    if (n < 0 || nnz < 0 || !rp || (nnz && !col) || (n && !perm_out)) {
+      spmv::set_error("spmv_reorder: bad argument");
+      return SPMV_EINVAL;
+    }
+    if (n > (int64_t)INT32_MAX - 1) {
+      spmv::set_error("spmv_reorder: n must fit int32");
+      return SPMV_EUNSUPPORTED;
+    }
+    if (rp[0] != 0 || rp[n] != nnz) {
+      spmv::set_error("spmv_reorder: row_ptr inconsistent with nnz");
+      return SPMV_EINVAL;
+    }
+    for (int64_t i = 0; i < n; ++i)
+      if (rp[i + 1] < rp[i]) {
+        spmv::set_error("spmv_reorder: row_ptr not monotone");
+        return SPMV_EINVAL;
+      }
+    for (int64_t k = 0; k < nnz; ++k)
+      if (col[k] < 0 || col[k] >= n) {
+        spmv::set_error("spmv_reorder: column out of range");
+        return SPMV_EINVAL;
+      }
+    spmv_reorder_stats_t S0;
+    std::memset(&S0, 0, sizeof(S0));
+    // skew: top ceil(0.1 N) row lengths / NZ
+    {
+      std::vector<int64_t> L(n);
+      for (int64_t i = 0; i < n; ++i) L[i] = rp[i + 1] - rp[i];
+      int64_t top = (int64_t)std::ceil(0.1 * (double)n);
+      if (top > 0 && n > 0) {
+        std::nth_element(L.begin(), L.begin() + (top - 1), L.end(), std::greater<int64_t>());
+        int64_t s = 0;
+        for (int64_t i = 0; i < top; ++i) s += L[i];
+        S0.skew = nnz ? (double)s / (double)nnz : 0.0;
+      }
+    }
+    // in-degree (column counts, diagonal and duplicates included: reading c13)
+    std::vector<int64_t> colcnt(n, 0);
+    for (int64_t k = 0; k < nnz; ++k) colcnt[col[k]]++;
+    std::vector<uint8_t> hub(n);
+    for (int64_t v = 0; v < n; ++v) {
+      hub[v] = (__int128)colcnt[v] * n > (__int128)nnz;
+      S0.n_hubs += hub[v];
+    }
+
+    if (method == SPMV_ORDER_ORIGINAL) {
+      for (int64_t i = 0; i < n; ++i) perm_out[i] = (int32_t)i;
+    } else if (method == SPMV_ORDER_RANDOM) {
+      random_order(n, seed, perm_out);
+    } else if (method == SPMV_ORDER_DEGSORT) {
+      std::vector<int32_t> seq(n);
+      std::iota(seq.begin(), seq.end(), 0);
+      std::stable_sort(seq.begin(), seq.end(),
+                       [&](int32_t a, int32_t b) { return colcnt[a] > colcnt[b]; });
+      for (int64_t i = 0; i < n; ++i) perm_out[seq[i]] = (int32_t)i;
+    } else if (method >= SPMV_ORDER_RABBIT && method <= SPMV_ORDER_HUBGROUP) {
+      Sym S = symmetrize(n, rp, col);
+      auto td = std::chrono::steady_clock::now();
+      Rabbit R = rabbit_detect(S);
+      S0.seconds_detect = std::chrono::duration<double>(std::chrono::steady_clock::now() - td).count();
+      S0.two_m = R.two_m;
+      S0.n_merges = R.n_merges;
+      S0.n_communities = R.n_top;
+      // community sizes
+      {
+        std::vector<int64_t> sz(n, 0);
+        for (int64_t v = 0; v < n; ++v) sz[R.comm[v]]++;
+        int64_t mx = 0;
+        for (int64_t v = 0; v < n; ++v) mx = std::max(mx, sz[v]);
+        S0.largest_comm_frac = n ? (double)mx / (double)n : 0.0;
+      }
+      // modularity Q' = sum_c (2m in_c - tot_c^2) and insular flags
+      std::vector<uint8_t> ins(n, 1);
+      {
+        std::vector<__int128> inc(n, 0), totc(n, 0);
+        for (int64_t v = 0; v < n; ++v) {
+          int32_t c = R.comm[v];
+          for (int64_t k = S.ptr[v]; k < S.ptr[v + 1]; ++k) {
+            totc[c] += S.w[k];
+            if (R.comm[S.idx[k]] == c) inc[c] += S.w[k];
+            else ins[v] = 0;
+          }
+        }
+        __int128 q = 0;
+        for (int64_t c = 0; c < n; ++c)
+          if (totc[c] || inc[c]) q += (__int128)R.two_m * inc[c] - totc[c] * totc[c];
+        S0.modularity_num = (double)q;
+        S0.modularity = R.two_m ? (double)q / ((double)R.two_m * (double)R.two_m) : 0.0;
+      }
+      // insularity over distinct off-diagonal pairs of A (reading c12)
+      {
+        int64_t intra = 0, total = 0;
+        std::vector<int32_t> tmp;
+        for (int64_t i = 0; i < n; ++i) {
+          tmp.assign(col + rp[i], col + rp[i + 1]);
+          std::sort(tmp.begin(), tmp.end());
+          tmp.erase(std::unique(tmp.begin(), tmp.end()), tmp.end());
+          for (int32_t j : tmp)
+            if (j != i) {
+              total++;
+              intra += R.comm[j] == R.comm[i];
+            }
+        }
+        S0.insularity = total ? (double)intra / (double)total : 1.0;
+        int64_t ni = 0;
+        for (int64_t v = 0; v < n; ++v) ni += ins[v];
+        S0.insular_frac = n ? (double)ni / (double)n : 0.0;
+      }
+      if (method == SPMV_ORDER_RABBIT) {
+        std::memcpy(perm_out, R.perm.data(), sizeof(int32_t) * n);
+      } else {
+        std::vector<int32_t> seq(n);
+        for (int64_t v = 0; v < n; ++v) seq[R.perm[v]] = (int32_t)v;
+        std::vector<int32_t> out;
+        out.reserve(n);
+        auto take = [&](auto pred) {
+          for (int32_t v : seq)
+            if (pred(v)) out.push_back(v);
+        };
+        if (method == SPMV_ORDER_RABBITPP || method == SPMV_ORDER_HUBSORT) {
+          take([&](int32_t v) { return !ins[v] && hub[v]; });
+          S0.n_group0 = (int64_t)out.size();
+          if (method == SPMV_ORDER_HUBSORT)
+            std::stable_sort(out.begin(), out.end(),
+                             [&](int32_t a, int32_t b) { return colcnt[a] > colcnt[b]; });
+          take([&](int32_t v) { return !ins[v] && !hub[v]; });
+          take([&](int32_t v) { return (bool)ins[v]; });
+        } else if (method == SPMV_ORDER_INSULAR) {
+          take([&](int32_t v) { return !ins[v]; });
+          take([&](int32_t v) { return (bool)ins[v]; });
+        } else {  // HUBGROUP only
+          take([&](int32_t v) { return (bool)hub[v]; });
+          S0.n_group0 = (int64_t)out.size();
+          take([&](int32_t v) { return !hub[v]; });
+        }
+        for (int64_t i = 0; i < n; ++i) perm_out[out[i]] = (int32_t)i;
+      }
+      g_last_comm = R.comm;
+    } else {
+      spmv::set_error("spmv_reorder: unknown method");
+      return SPMV_EINVAL;
+    }
+    S0.seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    if (st) *st = S0;
+    return SPMV_OK;
+  } catch (const std::bad_alloc&) {
+    spmv::set_error("spmv_reorder: out of host memory");
+    return SPMV_ENOMEM;
+  } catch (...) {
+    spmv::set_error("spmv_reorder: internal error");
+    return SPMV_EINVAL;
+  }
+}
+
+extern "C" spmv_status spmv_reorder_last_comm(int64_t n, int32_t* comm_out) {
+  if ((int64_t)g_last_comm.size() != n || (n && !comm_out)) {
+    spmv::set_error("spmv_reorder_last_comm: no RABBIT result of this size on this thread");
+    return SPMV_EINVAL;
+  }
+  std::memcpy(comm_out, g_last_comm.data(), sizeof(int32_t) * n);
+  return SPMV_OK;
+}

@@ -1,0 +1,68 @@
+"""Row-block power iteration across ranks (reading c22).
+
+One process per GPU.  Rank k owns rows [b_k, b_{k+1}) of B (nnz-balanced
+partition computed by spmv_plan), a full replica of x in the padded layout
+x[k*M + (i - b_k)] (M = plan x_stride), and writes its y slice straight into
+its own segment of the next x buffer.  Per iteration:
+
+    exec_scaled   y_k = (B_k u_{t-1}) / s_{t-1},  partial sum y_k^2   (libspmv)
+    all_reduce    s_t^2 = sum_k partial                               (NCCL, 8 B)
+    all_gather    in place, equal-size segments of M floats           (NCCL over NVLink)
+
+The padded layout turns NCCL's missing all-gatherv into an in-place
+equal-count all-gather with zero copies.  The
+collectives go through torch.distributed (plumbing); all arithmetic runs in
+libspmv.  ``local`` may be any object with the Plan interface below, which is
+how the gloo/CPU tests drive this exact code with a stand-in local SpMV.
+"""
+from __future__ import annotations
+
+import math
+
+
+def iterate(local, x, iters: int, group=None):
+    """Run `iters` normalised steps from x (padded layout, every rank the same).
+
+    local: object with attributes world, rank, x_stride, y_offset, nrows and
+    methods exec_scaled(x, y, ss_in, ss_out) and scale(u, x, ss).
+    Returns (x_iters normalised, padded layout; lambda = s_iters).
+    """
+    import torch
+    import torch.distributed as dist
+
+    if iters < 1:
+        raise ValueError("iters must be >= 1")
+    M, off, nr = local.x_stride, local.y_offset, local.nrows
+    xa, xb = x, torch.empty_like(x)
+    ss = torch.zeros(2, dtype=torch.float64, device=x.device)
+    ss_in = None
+    for t in range(iters):
+        ss_out = ss[t & 1:(t & 1) + 1]
+        local.exec_scaled(xa, xb[off:off + nr], ss_in, ss_out)
+        if local.world > 1:
+            dist.all_reduce(ss_out, op=dist.ReduceOp.SUM, group=group)
+            dist.all_gather_into_tensor(xb, xb[off:off + M].clone() if not xb.is_cuda
+                                        else xb[off:off + M], group=group)
+        ss_in = ss_out
+        xa, xb = xb, xa
+    local.scale(xa, xa, ss_in)
+    return xa, math.sqrt(float(ss_in.item()))
+
+
+class PlanLocal:
+    """Adapter: a libspmv Plan as the `local` of iterate()."""
+
+    def __init__(self, plan):
+        from . import spmv
+        self._spmv = spmv
+        self.plan = plan
+        i = plan.info()
+        self.world, self.rank = i["world"], i["rank"]
+        self.x_stride, self.y_offset = i["x_stride"], i["y_offset"]
+        self.nrows = i["row_end"] - i["row_begin"]
+
+    def exec_scaled(self, x, y, ss_in, ss_out):
+        self.plan.exec_scaled(x, y, ss_in, ss_out)
+
+    def scale(self, u, x, ss):
+        self._spmv.scale_vec(u, x, ss)

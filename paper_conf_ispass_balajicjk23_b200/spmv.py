@@ -1,0 +1,295 @@
+"""Thin ctypes binding of include/spmv.h (argument marshalling only).
+
+Every step of the path runs in libspmv.so; torch supplies device memory and
+streams.  There is no fallback: if the library is missing or a call fails,
+an exception is raised.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+SO_PATH = os.path.join(_HERE, "libspmv.so")
+HEADER = os.path.join(os.path.dirname(_HERE), "include", "spmv.h")
+
+ORIGINAL, RANDOM, RABBIT, RABBITPP, HUBSORT, INSULAR, HUBGROUP, DEGSORT = range(8)
+METHODS = {"original": ORIGINAL, "random": RANDOM, "rabbit": RABBIT, "rabbitpp": RABBITPP,
+           "hubsort": HUBSORT, "insular": INSULAR, "hubgroup": HUBGROUP, "degsort": DEGSORT}
+STATUS = {0: "SPMV_OK", 1: "SPMV_EINVAL", 2: "SPMV_EPERM", 3: "SPMV_ENOMEM", 4: "SPMV_ECUDA",
+          5: "SPMV_ENCCL", 6: "SPMV_EUNSUPPORTED", 7: "SPMV_ESTATE"}
+
+
+class SpmvError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class _Csr(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("nnz", ctypes.c_int64), ("row_ptr32", ctypes.c_void_p),
+                ("row_ptr64", ctypes.c_void_p), ("col_idx", ctypes.c_void_p),
+                ("vals", ctypes.c_void_p)]
+
+
+class _Opts(ctypes.Structure):
+    _fields_ = [("l2_window", ctypes.c_int32), ("evict_first", ctypes.c_int32),
+                ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("device", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+                ("l2_hit_ratio", ctypes.c_double), ("reserved", ctypes.c_int64 * 8)]
+
+
+class _Info(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int64) for n in (
+        "n", "nnz", "row_begin", "row_end", "nnz_local", "x_len", "x_stride", "y_offset",
+        "n_tiles", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "hot_prefix", "ideal_bytes")] + \
+        [(n, ctypes.c_int32) for n in ("offset_bytes", "world", "rank", "permuted",
+                                       "l2_window_bytes", "r0", "r1", "r2")]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [("n_communities", ctypes.c_int64), ("largest_comm_frac", ctypes.c_double),
+                ("modularity", ctypes.c_double), ("modularity_num", ctypes.c_double),
+                ("two_m", ctypes.c_int64), ("n_merges", ctypes.c_int64),
+                ("insularity", ctypes.c_double), ("insular_frac", ctypes.c_double),
+                ("n_hubs", ctypes.c_int64), ("n_group0", ctypes.c_int64),
+                ("skew", ctypes.c_double), ("seconds", ctypes.c_double),
+                ("seconds_detect", ctypes.c_double)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libspmv.so (built in-tree by build.py / __graft_entry__.build())."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(SO_PATH):
+            raise ImportError(f"{SO_PATH} is missing: run `python -m paper_conf_ispass_balajicjk23_b200.build`")
+        L = ctypes.CDLL(SO_PATH)
+        vp, i64, i32, dp = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_void_p
+        sig = {
+            "spmv_opts_default": (None, [ctypes.POINTER(_Opts)]),
+            "spmv_plan": (i32, [ctypes.POINTER(_Csr), vp, ctypes.POINTER(_Opts), ctypes.POINTER(vp)]),
+            "spmv_permute": (i32, [vp, vp]),
+            "spmv_permute_vec": (i32, [vp, vp, vp, i32, vp]),
+            "spmv_pad_vec": (i32, [vp, vp, vp, i32, vp]),
+            "spmv_exec": (i32, [vp, vp, vp, vp]),
+            "spmv_exec_scaled": (i32, [vp, vp, vp, dp, dp, vp]),
+            "spmv_iterate": (i32, [vp, vp, i32, ctypes.POINTER(ctypes.c_double), vp]),
+            "spmv_scale_vec": (i32, [vp, vp, i64, dp, vp]),
+            "spmv_plan_info": (i32, [vp, ctypes.POINTER(_Info)]),
+            "spmv_export_csr": (i32, [vp, vp, vp, vp, vp]),
+            "spmv_export_bins": (i32, [vp, vp, vp, vp, vp, vp, vp]),
+            "spmv_export_partition": (i32, [vp, vp]),
+            "spmv_export_inverse": (i32, [vp, vp, vp]),
+            "spmv_destroy": (None, [vp]),
+            "spmv_reorder": (i32, [i64, i64, vp, vp, i32, ctypes.c_uint64, vp, ctypes.POINTER(_Stats)]),
+            "spmv_reorder_last_comm": (i32, [i64, vp]),
+            "spmv_last_error": (ctypes.c_char_p, []),
+            "spmv_version": (ctypes.c_char_p, []),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def declared_symbols() -> list[str]:
+    """Every function include/spmv.h declares."""
+    txt = open(HEADER).read()
+    return sorted(set(re.findall(r"^\s*(?:spmv_status|void|const char\*)\s+(spmv_\w+)\s*\(", txt, re.M)))
+
+
+def _check(st: int):
+    if st != 0:
+        raise SpmvError(st, lib().spmv_last_error().decode())
+
+
+def version() -> str:
+    return lib().spmv_version().decode()
+
+
+def _stream_ptr(stream=None) -> int:
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+def _ptr(t) -> int | None:
+    return None if t is None else int(t.data_ptr())
+
+
+class Plan:
+    """spmv_plan + spmv_permute over device CSR tensors (torch, cuda).
+
+    row_ptr: int32 or int64 [n+1]; col: int32 [nnz]; val: float32 [nnz];
+    perm: int32 [n] (perm[old] = new) or None for identity.
+    """
+
+    def __init__(self, row_ptr, col, val, perm=None, *, world=1, rank=0, l2_window=True,
+                 evict_first=True, l2_hit_ratio=1.0, permute=True, stream=None):
+        import torch
+        assert row_ptr.is_cuda and col.is_cuda and val.is_cuda
+        assert col.dtype == torch.int32 and val.dtype == torch.float32
+        n = row_ptr.numel() - 1
+        self._keep = (row_ptr, col, val, perm)  # A must outlive permute
+        A = _Csr(n, col.numel(), None, None, _ptr(col), _ptr(val))
+        if row_ptr.dtype == torch.int64:
+            A.row_ptr64 = _ptr(row_ptr)
+        elif row_ptr.dtype == torch.int32:
+            A.row_ptr32 = _ptr(row_ptr)
+        else:
+            raise TypeError("row_ptr must be int32 or int64")
+        if perm is not None:
+            assert perm.is_cuda and perm.dtype == torch.int32 and perm.numel() == n
+        o = _Opts()
+        lib().spmv_opts_default(ctypes.byref(o))
+        o.world, o.rank = world, rank
+        o.l2_window, o.evict_first = int(l2_window), int(evict_first)
+        o.l2_hit_ratio = l2_hit_ratio
+        o.device = row_ptr.device.index if row_ptr.device.index is not None else -1
+        h = ctypes.c_void_p()
+        _check(lib().spmv_plan(ctypes.byref(A), _ptr(perm), ctypes.byref(o), ctypes.byref(h)))
+        self._h = h
+        self.device = row_ptr.device
+        if permute:
+            self.permute(stream)
+
+    # ------------------------------------------------------------------ calls
+    def permute(self, stream=None):
+        _check(lib().spmv_permute(self._h, _stream_ptr(stream)))
+        return self
+
+    def info(self) -> dict:
+        i = _Info()
+        _check(lib().spmv_plan_info(self._h, ctypes.byref(i)))
+        return {f: getattr(i, f) for f, _ in _Info._fields_ if f not in ("r0", "r1", "r2")}
+
+    def permute_vec(self, x, inverse=False, out=None, stream=None):
+        import torch
+        out = torch.empty_like(x) if out is None else out
+        _check(lib().spmv_permute_vec(self._h, _ptr(x), _ptr(out), int(inverse), _stream_ptr(stream)))
+        return out
+
+    def pad_vec(self, x, to_padded=True, out=None, stream=None):
+        import torch
+        if out is None:
+            info = self.info()
+            out = torch.zeros(info["x_len"] if to_padded else info["n"], dtype=torch.float32,
+                              device=x.device)
+        _check(lib().spmv_pad_vec(self._h, _ptr(x), _ptr(out), int(to_padded), _stream_ptr(stream)))
+        return out
+
+    def exec(self, x, y=None, stream=None):
+        import torch
+        if y is None:
+            info = self.info()
+            y = torch.empty(info["row_end"] - info["row_begin"], dtype=torch.float32, device=x.device)
+        _check(lib().spmv_exec(self._h, _ptr(x), _ptr(y), _stream_ptr(stream)))
+        return y
+
+    def exec_scaled(self, x, y, sumsq_in=None, sumsq_out=None, stream=None):
+        _check(lib().spmv_exec_scaled(self._h, _ptr(x), _ptr(y), _ptr(sumsq_in), _ptr(sumsq_out),
+                                      _stream_ptr(stream)))
+        return y
+
+    def iterate(self, x, iters: int, stream=None) -> float:
+        lam = ctypes.c_double(0.0)
+        _check(lib().spmv_iterate(self._h, _ptr(x), iters, ctypes.byref(lam), _stream_ptr(stream)))
+        return lam.value
+
+    def export_csr(self, stream=None):
+        import torch
+        i = self.info()
+        nr = i["row_end"] - i["row_begin"]
+        rp = torch.empty(nr + 1, dtype=torch.int64, device=self.device)
+        col = torch.empty(max(i["nnz_local"], 0), dtype=torch.int32, device=self.device)
+        val = torch.empty(max(i["nnz_local"], 0), dtype=torch.float32, device=self.device)
+        _check(lib().spmv_export_csr(self._h, _ptr(rp), _ptr(col), _ptr(val), _stream_ptr(stream)))
+        return rp, col, val
+
+    def export_bins(self, stream=None) -> dict:
+        import torch
+        i = self.info()
+        mk = lambda m: torch.empty(max(m, 0), dtype=torch.int32, device=self.device)  # noqa: E731
+        d = {"tiles": mk(i["n_tiles"] + 1), "cta_rows": mk(i["n_cta_rows"]),
+             "hub_rows": mk(i["n_hub_rows"]), "chunk_row": mk(i["n_hub_chunks"]),
+             "chunk_idx": mk(i["n_hub_chunks"])}
+        _check(lib().spmv_export_bins(self._h, _ptr(d["tiles"]), _ptr(d["cta_rows"]),
+                                      _ptr(d["hub_rows"]), _ptr(d["chunk_row"]),
+                                      _ptr(d["chunk_idx"]), _stream_ptr(stream)))
+        return d
+
+    def export_partition(self) -> list[int]:
+        w = self.info()["world"]
+        b = (ctypes.c_int64 * (w + 1))()
+        _check(lib().spmv_export_partition(self._h, ctypes.cast(b, ctypes.c_void_p)))
+        return list(b)
+
+    def export_inverse(self, stream=None):
+        import torch
+        inv = torch.empty(self.info()["n"], dtype=torch.int32, device=self.device)
+        _check(lib().spmv_export_inverse(self._h, _ptr(inv), _stream_ptr(stream)))
+        return inv
+
+    def close(self):
+        if getattr(self, "_h", None):
+            import torch
+            torch.cuda.synchronize(self.device)
+            lib().spmv_destroy(self._h)
+            self._h = None
+            self._keep = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def scale_vec(u, x, sumsq=None, stream=None):
+    _check(lib().spmv_scale_vec(_ptr(u), _ptr(x), u.numel(), _ptr(sumsq), _stream_ptr(stream)))
+    return x
+
+
+@dataclass
+class ReorderStats:
+    n_communities: int
+    largest_comm_frac: float
+    modularity: float
+    modularity_num: float
+    two_m: int
+    n_merges: int
+    insularity: float
+    insular_frac: float
+    n_hubs: int
+    n_group0: int
+    skew: float
+    seconds: float
+    seconds_detect: float
+
+
+def reorder(row_ptr: np.ndarray, col: np.ndarray, method="rabbitpp", seed: int = 0):
+    """Host reordering (spmv_reorder).  Returns (perm int32[n], ReorderStats)."""
+    m = METHODS[method] if isinstance(method, str) else int(method)
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    c = np.ascontiguousarray(col, dtype=np.int32)
+    n = len(rp) - 1
+    perm = np.empty(n, np.int32)
+    st = _Stats()
+    _check(lib().spmv_reorder(n, int(rp[-1]) if n >= 0 else 0, rp.ctypes.data, c.ctypes.data, m,
+                              seed, perm.ctypes.data, ctypes.byref(st)))
+    return perm, ReorderStats(**{f: getattr(st, f) for f, _ in _Stats._fields_})
+
+
+def reorder_last_comm(n: int) -> np.ndarray:
+    out = np.empty(n, np.int32)
+    _check(lib().spmv_reorder_last_comm(n, out.ctypes.data))
+    return out

@@ -1,0 +1,290 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle.
+
+Bars (BASELINE.json north_star):
+  * integer outputs bit-exact: permuted CSR (row_ptr, col, value bits), stream
+    tiles, row classes, hub chunks, partition bounds, H, inverse perm;
+  * y within |y_gpu - y_ref| <= 1e-5 * sum_j |a_rj x_j| per row (TOL below);
+  * y bitwise repeatable and independent of the row partition (world).
+"""
+import math
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import cref, permute, plan as oplan, power, rabbit, spmv as ospmv
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+TOL = 1e-5
+
+
+def _skip_no_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+
+
+@pytest.fixture(scope="module")
+def dev():
+    _skip_no_gpu()
+    from paper_conf_ispass_balajicjk23_b200 import spmv  # noqa: F401  (fails loudly if missing)
+    return torch.device("cuda:0")
+
+
+def to_dev(A, dev, rp_dtype=torch.int64):
+    return (torch.from_numpy(np.asarray(A.row_ptr)).to(dev, rp_dtype),
+            torch.from_numpy(np.asarray(A.col)).to(dev),
+            torch.from_numpy(np.asarray(A.val)).to(dev))
+
+
+def mk_plan(A, perm, dev, **kw):
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    rp, c, v = to_dev(A, dev, kw.pop("rp_dtype", torch.int64))
+    p = None if perm is None else torch.from_numpy(np.asarray(perm, np.int32)).to(dev)
+    return spmv.Plan(rp, c, v, p, **kw)
+
+
+class Mat:
+    def __init__(self, n, row_ptr, col, val):
+        self.n, self.row_ptr, self.col, self.val = n, np.asarray(row_ptr, np.int64), \
+            np.asarray(col, np.int32), np.asarray(val, np.float32)
+
+    @property
+    def nnz(self):
+        return int(self.row_ptr[-1])
+
+
+def long_rows_matrix(seed=0):
+    """Rows of every class: empty, short, medium, CTA, hub (> 16384), with
+    duplicates and unsorted columns."""
+    rng = np.random.default_rng(seed)
+    n = 30000
+    L = rng.integers(0, 20, n)
+    L[rng.random(n) < 0.3] = 0
+    special = {5: 40000, 17: 16385, 99: 16384, 1000: 9000, 1001: 2049, 1002: 2048, 2500: 700,
+               2501: 33, 2502: 32, 29999: 70000}
+    for r, l in special.items():
+        L[r] = l
+    rp = np.concatenate([[0], np.cumsum(L)])
+    col = rng.integers(0, n, rp[-1]).astype(np.int32)
+    col[rp[5]:rp[5] + 100] = 7                       # duplicates in a hub row
+    val = rng.uniform(-1, 1, rp[-1]).astype(np.float32)
+    return Mat(n, rp, col, val)
+
+
+def _cases():
+    yield "rmat12", lambda: synth.config(1, small=True).A
+    yield "sbm16x1024", lambda: synth.config(2, small=True).A
+    yield "stencil24", lambda: synth.config(4, small=True).A
+    yield "kron14", lambda: synth.config(5, small=True).A
+    yield "longrows", long_rows_matrix
+
+
+CASES = list(_cases())
+
+
+def _perms(A, which):
+    if which == "identity":
+        return None
+    if which == "random":
+        return rabbit.random_perm(A.n, 77)
+    if which == "rabbitpp":
+        from paper_conf_ispass_balajicjk23_b200 import spmv
+        return spmv.reorder(A.row_ptr, A.col, "rabbitpp")[0]
+    raise ValueError(which)
+
+
+@pytest.mark.parametrize("name,make", CASES)
+@pytest.mark.parametrize("which", ["identity", "random", "rabbitpp"])
+def test_permute_and_bins_bitexact(dev, name, make, which):
+    A = make()
+    if which == "rabbitpp" and name == "longrows":
+        which = "random"
+    perm = _perms(A, which)
+    P = mk_plan(A, perm, dev)
+    pm = np.arange(A.n) if perm is None else np.asarray(perm, np.int64)
+    Bp, Bc, Bv = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, pm)
+    rp, c, v = (t.cpu().numpy() for t in P.export_csr())
+    assert np.array_equal(rp, Bp)
+    assert np.array_equal(c, Bc)
+    assert np.array_equal(v.view(np.int32), Bv.view(np.int32))
+    bins = {k: t.cpu().numpy() for k, t in P.export_bins().items()}
+    assert np.array_equal(bins["tiles"], oplan.tile_bounds(Bp))
+    cta, hub, cr, ci = oplan.row_classes(Bp)
+    assert np.array_equal(bins["cta_rows"], cta)
+    assert np.array_equal(bins["hub_rows"], hub)
+    assert np.array_equal(bins["chunk_row"], cr) and np.array_equal(bins["chunk_idx"], ci)
+    info = P.info()
+    assert info["hot_prefix"] == oplan.hot_prefix(A.n, Bc)
+    assert np.array_equal(P.export_inverse().cpu().numpy(), permute.inverse(pm))
+    P.close()
+
+
+def _check_y(y, ref, absrow, what=""):
+    err = np.abs(y.astype(np.float64) - ref.astype(np.float64))
+    bad = err > TOL * absrow + 1e-37
+    assert not bad.any(), f"{what}: {bad.sum()} rows out of tolerance, worst {err[bad].max()}"
+
+
+@pytest.mark.parametrize("name,make", CASES)
+def test_exec_matches_oracle(dev, name, make):
+    A = make()
+    perm = rabbit.random_perm(A.n, 5)
+    P = mk_plan(A, perm, dev)
+    x = synth.vector(A.n, 99)
+    Bp, Bc, Bv = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
+    xB = permute.permute_vec(x, perm)
+    xB_dev = P.permute_vec(torch.from_numpy(x).to(dev))
+    assert np.array_equal(xB_dev.cpu().numpy(), xB)
+    y = P.exec(xB_dev).cpu().numpy()
+    ref = ospmv.spmv(Bp, Bc, Bv, xB)
+    _check_y(y, ref, ospmv.abs_rowsum(Bp, Bc, Bv, xB), name)
+    # empty rows give exactly +-0
+    L = np.diff(Bp)
+    assert np.all(y[L == 0] == 0)
+    # bitwise repeatable
+    y2 = P.exec(xB_dev).cpu().numpy()
+    assert np.array_equal(y.view(np.int32), y2.view(np.int32))
+    # P^T y_B == A x  (inverse relabel on the device)
+    yA = P.permute_vec(torch.from_numpy(y).to(dev), inverse=True).cpu().numpy()
+    _check_y(yA, ospmv.spmv(A.row_ptr, A.col, A.val, x), ospmv.abs_rowsum(A.row_ptr, A.col, A.val, x))
+    P.close()
+
+
+@pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("rmat12", "longrows", "kron14")])
+@pytest.mark.parametrize("world", [2, 3, 4])
+def test_partitioned_equals_single_bitwise(dev, name, make, world):
+    A = make()
+    perm = rabbit.random_perm(A.n, 11)
+    P1 = mk_plan(A, perm, dev)
+    x = torch.from_numpy(synth.vector(A.n, 3)).to(dev)
+    xB = P1.permute_vec(x)
+    y1 = P1.exec(xB).cpu().numpy()
+    Bp, _, _ = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
+    bounds = oplan.partition(Bp, world)
+    parts = []
+    for r in range(world):
+        Pr = mk_plan(A, perm, dev, world=world, rank=r)
+        assert Pr.export_partition() == bounds.tolist()
+        info = Pr.info()
+        assert (info["row_begin"], info["row_end"]) == (bounds[r], bounds[r + 1])
+        xpad = Pr.pad_vec(xB, to_padded=True)
+        assert xpad.numel() == info["x_len"] == world * info["x_stride"]
+        back = Pr.pad_vec(xpad, to_padded=False)
+        assert torch.equal(back, xB)
+        parts.append(Pr.exec(xpad).cpu().numpy())
+        Pr.close()
+    yc = np.concatenate(parts)
+    assert np.array_equal(yc.view(np.int32), y1.view(np.int32))
+    P1.close()
+
+
+def test_int32_and_int64_row_ptr_agree(dev):
+    A = synth.config(1, small=True).A
+    perm = rabbit.random_perm(A.n, 2)
+    x = torch.from_numpy(synth.vector(A.n, 1)).to(dev)
+    ys = []
+    for dt in (torch.int32, torch.int64):
+        P = mk_plan(A, perm, dev, rp_dtype=dt)
+        ys.append(P.exec(P.permute_vec(x)).cpu().numpy())
+        P.close()
+    assert np.array_equal(ys[0].view(np.int32), ys[1].view(np.int32))
+
+
+def test_errors(dev):
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = synth.rmat(8, 4, 1)
+    bad = np.arange(A.n, dtype=np.int32)
+    bad[3] = 4
+    with pytest.raises(spmv.SpmvError) as e:
+        mk_plan(A, bad, dev)
+    assert e.value.status == 2  # EPERM
+    Abad = Mat(A.n, A.row_ptr, np.where(A.col == 0, A.n, A.col), A.val)
+    with pytest.raises(spmv.SpmvError) as e:
+        mk_plan(Abad, None, dev)
+    assert e.value.status == 1
+    P = mk_plan(A, None, dev, permute=False)
+    with pytest.raises(spmv.SpmvError) as e:
+        P.exec(torch.zeros(A.n, device=dev))
+    assert e.value.status == 7  # ESTATE
+    P.close()
+
+
+def test_degenerate_shapes(dev):
+    for A in (Mat(1, [0, 0], [], []), Mat(5, [0] * 6, [], []),
+              Mat(3, [0, 1, 1, 2], [2, 0], [2.5, -1.0]),
+              Mat(2, [0, 70000, 70000], np.zeros(70000), np.ones(70000))):
+        P = mk_plan(A, None, dev)
+        x = np.arange(1, A.n + 1, dtype=np.float32)
+        y = P.exec(torch.from_numpy(x).to(dev)).cpu().numpy()
+        ref = ospmv.spmv(A.row_ptr, A.col, A.val, x)
+        _check_y(y, ref, ospmv.abs_rowsum(A.row_ptr, A.col, A.val, x))
+        P.close()
+
+
+def test_iterate_regular_fixed_point(dev):
+    # periodic 27-point stencil, unit values: lambda = 27, x0 = 1/sqrt(N) fixed
+    A = synth.stencil27(12, periodic=True, relabel=True, seed_scr=5, valmode=synth.VAL_ONES)
+    perm, _ = __import__("paper_conf_ispass_balajicjk23_b200").spmv.reorder(A.row_ptr, A.col, "rabbitpp")
+    P = mk_plan(A, perm, dev)
+    x0 = np.full(A.n, np.float32(1 / math.sqrt(A.n)))
+    x = torch.from_numpy(x0).to(dev)
+    lam = P.iterate(x, 10)
+    assert math.isclose(lam, 27.0, rel_tol=1e-5)
+    assert np.allclose(x.cpu().numpy(), x0, rtol=1e-5)
+    P.close()
+
+
+def test_iterate_matches_oracle_recurrence(dev):
+    w = synth.config(5, small=True)          # Kronecker, positive values
+    A = w.A
+    perm, _ = __import__("paper_conf_ispass_balajicjk23_b200").spmv.reorder(A.row_ptr, A.col, "rabbitpp")
+    P = mk_plan(A, perm, dev)
+    Bp, Bc, Bv = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
+    x0 = permute.permute_vec(w.x, perm)
+    x = torch.from_numpy(x0.copy()).to(dev)
+    iters = 20
+    lam = P.iterate(x, iters)
+    xr, lr = power.power_iteration(Bp, Bc, Bv, x0, iters)
+    assert abs(lam - lr) <= 1e-5 * lr
+    assert np.max(np.abs(x.cpu().numpy() - xr)) <= 1e-5 * np.max(np.abs(xr)) * 10
+    # step-wise parity: one scaled step from the GPU's own x
+    xt = x.cpu().numpy()
+    y = torch.empty(A.n, device=dev)
+    ss = torch.zeros(1, dtype=torch.float64, device=dev)
+    P.exec_scaled(x, y, None, ss)
+    yr, sr = power.power_step(Bp, Bc, Bv, xt)
+    _check_y(y.cpu().numpy(), yr, ospmv.abs_rowsum(Bp, Bc, Bv, xt))
+    assert abs(math.sqrt(ss.item()) - sr) <= 1e-5 * sr
+    P.close()
+
+
+def test_bench_config_full_size(dev):
+    """BASELINE config 2 (SBM 4M/64M) at full size in the launch configuration
+    bench.py times: every row against the compensated C oracle, sampled rows
+    against the exact fsum oracle."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    w = synth.config(2)
+    A = w.A
+    perm, _ = spmv.reorder(A.row_ptr, A.col, "rabbitpp")
+    P = mk_plan(A, perm, dev)
+    xB = P.permute_vec(torch.from_numpy(w.x).to(dev))
+    y = P.exec(xB).cpu().numpy()
+    rp, c, v = (t.cpu().numpy() for t in P.export_csr())
+    # integer structure on sampled rows vs the oracle's own relabelling
+    inv = permute.inverse(perm)
+    rng = np.random.default_rng(0)
+    rows = np.sort(rng.choice(A.n, 2000, replace=False))
+    for r, (cc, vv) in zip(rows, permute.permute_rows(A.row_ptr, A.col, A.val, perm, inv, rows)):
+        assert np.array_equal(c[rp[r]:rp[r + 1]], cc)
+        assert np.array_equal(v[rp[r]:rp[r + 1]].view(np.int32), vv.view(np.int32))
+    xBh = permute.permute_vec(w.x, perm)
+    oracle_rows = permute.permute_rows(A.row_ptr, A.col, A.val, perm, inv, rows)
+    ys = np.array([ospmv.spmv_rows([0, len(cc)], cc, vv, xBh, [0])[0] for cc, vv in oracle_rows])
+    ab = np.array([np.abs(vv.astype(np.float64) * xBh[cc].astype(np.float64)).sum()
+                   for cc, vv in oracle_rows])
+    _check_y(y[rows], ys, ab, "sampled")
+    # every row: compensated C oracle on A itself, relabelled (y_B = P (A x))
+    yA, absA = cref.spmv_neumaier(A.row_ptr, A.col, A.val, w.x)
+    _check_y(y, permute.permute_vec(yA, perm), permute.permute_vec(absA, perm), "all rows")
+    P.close()
