@@ -53,6 +53,19 @@ def permute_csr(n, row_ptr, col, val, perm):
     return B_ptr, B_col, B_val
 
 
+def permute_csr_scipy(n, row_ptr, col, val, perm):
+    """B = P A P^T through scipy fancy indexing (B = A[inv][:, inv]) with
+    sorted rows: a fast library route used only to prepare the input of the
+    timed CPU baseline (duplicate order is not guaranteed stable)."""
+    import scipy.sparse as sp
+    inv = inverse(perm)
+    M = sp.csr_matrix((np.asarray(val, np.float32), np.asarray(col), np.asarray(row_ptr)),
+                      shape=(n, n))
+    B = M[inv][:, inv]
+    B.sort_indices()
+    return B.indptr.astype(np.int64), B.indices.astype(np.int32), B.data.astype(np.float32)
+
+
 def permute_rows(row_ptr, col, val, perm, inv, rows):
     """Rows `rows` of B = P A P^T only (large-size sampled parity):
     row r of B is row inv[r] of A relabelled by perm and stably sorted."""

@@ -5,14 +5,17 @@ The paper runs cuSPARSE and never describes scheduling (Alg. 1
 is a plain "parfor row"); these are build constants (reading c23), RE-DECLARED
 here from DESIGN.md §Plan, not imported from the library:
 
-  TILE_D      = 2048   stream tile "diagonal": row r (r < N) belongs to tile
+  TILE_D      = 8192   stream tile "diagonal": row r (r < N) belongs to tile
                         k = floor((row_ptr[r] + r) / TILE_D); tiles
                         k = 0 .. K-1, K = ceil((NZ + N) / TILE_D);
                         bounds b_k = lower_bound_{r in [0,N]}(row_ptr[r] + r >= k*TILE_D)
-  STREAM_MAX  = 2048   rows with L <= STREAM_MAX are computed inside their
-                        stream tile; longer rows are always the last row of
-                        their tile and are excluded from it
-  CTA_MAX     = 16384  STREAM_MAX < L <= CTA_MAX: one CTA per row
+  STREAM_MAX  = 1024   a stream tile computes its rows with L <= WARP_MAX,
+                        except its LAST row when that row has L > STREAM_MAX
+                        (the tile buffer holds < TILE_D + STREAM_MAX entries);
+                        rows with L >= TILE_D are always last
+  WARP_MAX    = 2048   last-in-tile rows with STREAM_MAX < L <= WARP_MAX: one
+                        warp per row
+  CTA_MAX     = 16384  WARP_MAX < L <= CTA_MAX (any position): one CTA per row
   HUB_CHUNK   = 16384  L > CTA_MAX: hub row cut into ceil(L / HUB_CHUNK)
                         chunks of HUB_CHUNK entries (merge-path split)
 
@@ -28,8 +31,9 @@ from __future__ import annotations
 
 import numpy as np
 
-TILE_D = 2048
-STREAM_MAX = 2048
+TILE_D = 8192
+STREAM_MAX = 1024
+WARP_MAX = 2048
 CTA_MAX = 16384
 HUB_CHUNK = 16384
 
@@ -56,25 +60,35 @@ def tile_bounds(row_ptr) -> np.ndarray:
     return b
 
 
+def _last_in_tile(row_ptr, r):
+    n = len(row_ptr) - 1
+    if r + 1 >= n:
+        return True
+    return (int(row_ptr[r]) + r) // TILE_D != (int(row_ptr[r + 1]) + r + 1) // TILE_D
+
+
 def row_classes(row_ptr):
-    """(cta_rows, hub_rows, chunk_row, chunk_idx), all ascending."""
+    """(warp_rows, cta_rows, hub_rows, chunk_row, chunk_idx), all ascending."""
     row_ptr = np.asarray(row_ptr, np.int64)
     L = np.diff(row_ptr)
-    cta = [r for r in range(len(L)) if STREAM_MAX < L[r] <= CTA_MAX]
+    warp = [r for r in range(len(L)) if STREAM_MAX < L[r] <= WARP_MAX and _last_in_tile(row_ptr, r)]
+    cta = [r for r in range(len(L)) if WARP_MAX < L[r] <= CTA_MAX]
     hub = [r for r in range(len(L)) if L[r] > CTA_MAX]
     ch_r, ch_i = [], []
     for r in hub:
         for c in range(-(-int(L[r]) // HUB_CHUNK)):
             ch_r.append(r)
             ch_i.append(c)
-    return (np.array(cta, np.int64), np.array(hub, np.int64),
+    return (np.array(warp, np.int64), np.array(cta, np.int64), np.array(hub, np.int64),
             np.array(ch_r, np.int64), np.array(ch_i, np.int64))
 
 
-def stream_rows(row_ptr, b) -> np.ndarray:
-    """Flag of rows computed inside a stream tile (every row with L <= STREAM_MAX)."""
-    L = np.diff(np.asarray(row_ptr, np.int64))
-    return L <= STREAM_MAX
+def stream_rows(row_ptr) -> np.ndarray:
+    """Flag of rows computed inside their stream tile."""
+    row_ptr = np.asarray(row_ptr, np.int64)
+    L = np.diff(row_ptr)
+    return np.array([L[r] <= WARP_MAX and not (L[r] > STREAM_MAX and _last_in_tile(row_ptr, r))
+                     for r in range(len(L))], bool)
 
 
 def hot_prefix(n, col_B) -> int:

@@ -42,6 +42,7 @@ void spmv_opts_default(spmv_opts_t* o) {
   o->world = 1;
   o->device = -1;
   o->l2_hit_ratio = 1.0;
+  o->smem_window = 1;
 }
 
 const char* spmv_last_error(void) { return spmv::get_error(); }
@@ -173,6 +174,7 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->x_stride = p->x_stride;
   info->y_offset = p->y_offset;
   info->n_tiles = p->K;
+  info->n_warp_rows = p->n_warp;
   info->n_cta_rows = p->n_cta;
   info->n_hub_rows = p->n_hub;
   info->n_hub_chunks = p->n_chunks;
@@ -219,13 +221,16 @@ spmv_status spmv_export_csr(spmv_plan_t p, int64_t* row_ptr, int32_t* col, float
   API_END
 }
 
-spmv_status spmv_export_bins(spmv_plan_t p, int32_t* tiles, int32_t* cta_rows, int32_t* hub_rows,
-                             int32_t* chunk_row, int32_t* chunk_idx, void* stream) {
+spmv_status spmv_export_bins(spmv_plan_t p, int32_t* tiles, int32_t* warp_rows, int32_t* cta_rows,
+                             int32_t* hub_rows, int32_t* chunk_row, int32_t* chunk_idx,
+                             void* stream) {
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_export_bins: NULL plan");
   use_device(p);
   cudaStream_t s = S(stream);
   if (tiles) SPMV_CUDA(cudaMemcpyAsync(tiles, p->d_tiles, 4 * (p->K + 1), cudaMemcpyDeviceToDevice, s));
+  if (warp_rows && p->n_warp)
+    SPMV_CUDA(cudaMemcpyAsync(warp_rows, p->d_warp_rows, 4 * p->n_warp, cudaMemcpyDeviceToDevice, s));
   if (cta_rows && p->n_cta)
     SPMV_CUDA(cudaMemcpyAsync(cta_rows, p->d_cta_rows, 4 * p->n_cta, cudaMemcpyDeviceToDevice, s));
   if (hub_rows && p->n_hub)

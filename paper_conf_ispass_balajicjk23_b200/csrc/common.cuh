@@ -11,13 +11,14 @@ namespace spmv {
 
 // Build constants (reading c23; declared in include/spmv.h and DESIGN.md §Plan;
 // re-declared independently in oracle/plan.py).
-constexpr int TILE_D = 2048;        // stream tile: rows + entries
-constexpr int STREAM_MAX = 2048;    // longest row computed inside a stream tile
+constexpr int TILE_D = 8192;        // stream tile: rows + entries
+constexpr int STREAM_MAX = 1024;    // longest row computed inside a stream tile
 constexpr int SHORT_MAX = 32;       // canonical order: sequential up to here
+constexpr int WARP_MAX = 2048;      // warp-per-row class upper bound (canonical W = 32)
 constexpr int CTA_MAX = 16384;      // CTA-per-row class upper bound
 constexpr int HUB_CHUNK = 16384;    // merge-path chunk of a hub row
 constexpr int CTA_THREADS = 256;    // canonical width of CTA / hub-chunk sums
-constexpr int TILE_BUF = 2 * TILE_D + 8;  // smem elements per tile (+ alignment slack)
+constexpr int TILE_BUF = TILE_D + STREAM_MAX + 8;  // max entries of a tile (+ alignment slack)
 
 void set_error(const std::string& msg);
 const char* get_error();

@@ -1,22 +1,22 @@
 // spmv_exec / spmv_exec_scaled / spmv_iterate: the hot path.
 //
 // Alg. 1 of the paper:  Y[row] += values[i] * X[coords[i]].
-// B200 design (DESIGN.md §Kernels):
-//   k_stream     one CTA per stream tile (TILE_D = 2048 rows+entries, row
-//                aligned).  One elected thread moves the tile's col/val slice
-//                global->shared with two cp.async.bulk copies (TMA bulk engine)
-//                carrying an L2 evict_first policy and completing on an
-//                mbarrier; all threads then gather x through L2 (__ldg),
-//                form the fp32 products into a bank-padded product array, and
-//                reduce rows in the canonical order of include/spmv.h: thread
-//                per row (L <= 32, sequential) or warp per row (32 < L <=
-//                2048, 32 strided partials + xor tree).  y is written once,
-//                coalesced.
+// B200 design (DESIGN.md §6):
+//   k_panel      persistent CTAs over contiguous row panels of stream tiles
+//                (TILE_D = 8192 rows+entries, row aligned); a 2-stage ring of
+//                cp.async.bulk (TMA bulk engine) + mbarrier copies of tile
+//                col/val (L2 evict_first); a sliding
+//                shared-memory x window follows the diagonal, so
+//                community-local gathers are shared-memory reads; rows reduced
+//                in the canonical order of include/spmv.h (thread per row
+//                L <= 32, warp per row 32 < L <= 1024); y written once.
+//   k_warp_rows  one warp per row, 1024 < L <= 2048 (32 strided partials + tree),
+//                col/val streamed with 4 independent 128-B warp loads in flight.
 //   k_cta_rows   one CTA per row, 2048 < L <= 16384 (256 strided partials + tree).
 //   k_hub_chunk  one CTA per 16384-entry chunk of a hub row (merge-path split);
 //   k_hub_fix    fp64 combine of the chunk sums in chunk order.
 //   k_ss_final   fixed-order fp64 sum of per-tile / per-row y^2 partials
-//                (power iteration norm; deterministic).
+//                (power-iteration norm; deterministic).
 // No tensor cores: SpMV is not a dense contraction (AI <= 0.25 flop/B).
 #include <cmath>
 
@@ -41,13 +41,24 @@ __device__ __forceinline__ uint64_t l2_policy(int evict_first) {
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count)
                : "memory");
+}
+
+__device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
                "r"(bytes)
                : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes,
@@ -75,132 +86,331 @@ __device__ __forceinline__ float alpha_of(const double* ss_in) {
   return v > 0.0 ? (float)(1.0 / sqrt(v)) : 1.f;
 }
 
-// bank-padded index of the product array (one pad word per 32)
-__device__ __forceinline__ int pidx(int j) { return j + (j >> 5); }
-
-constexpr int ST_THREADS = 256;
-constexpr int PROD_LEN = TILE_BUF + TILE_BUF / 32 + 1;
-
-template <bool SS>
-__device__ __forceinline__ void block_sum_store(double acc, double* out) {
-  __shared__ double wss[32];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+__device__ __forceinline__ float warp_tree(float s) {
 #pragma unroll
-  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-  if (lane == 0) wss[w] = acc;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double s = 0.0;
-    for (int i = 0; i < (int)(blockDim.x >> 5); ++i) s += wss[i];
-    *out = s;
+  for (int o = 16; o > 0; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+  return s;
+}
+
+__device__ __forceinline__ double warp_sum_d(double s) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  return s;
+}
+
+// ------------------------------------------------------------ stream tiles
+// k_panel: persistent CTAs, each over a contiguous range of stream tiles (a
+// panel of consecutive rows), one CTA of 16 warps per SM.  Thread 0 keeps the
+// next tile in flight while the current one is computed (2-stage ring) with
+// cp.async.bulk copies (TMA bulk engine) of the tile's col / val (L2
+// evict_first), completing on per-stage mbarriers; tile descriptors are
+// precomputed by the plan and prefetched, so the producer has no dependent
+// loads on its path.  Tiles are large (TILE_D = 8192 rows+entries, ~64 KB of
+// matrix) so per-tile bookkeeping is amortised over ~16 entries per thread.
+// x is read through a SLIDING WINDOW: a shared-memory ring of XWIN floats that
+// holds x[c] at slot c % XWIN for c in [whi(t) - XWIN, whi(t)), whi(t) =
+// (last row of tile t) + XLEAD.  Community-ordered matrices put most columns
+// of a row near its diagonal (Fig. 1), so most gathers become
+// shared-memory reads instead of one L1/L2 request per scattered line; other
+// columns fall back to __ldg through L2.  The CTA advances the ring after the
+// tile's last window read (prefetched into registers during the tile, ordered
+// by __syncthreads), so no two writers ever race on a slot.  Rows are reduced
+// in the canonical order of include/spmv.h, so where x came from never
+// changes y.
+constexpr int PT_THREADS = 512;
+constexpr int PT_STAGES = 2;
+constexpr int XWIN = 4096;   // x window ring (floats, power of two)
+constexpr int XLEAD = 1536;  // window leads the tile's end row by this many columns
+constexpr int PROD_LEN = TILE_BUF + TILE_BUF / 16 + 1;
+constexpr int MID_CAP = (TILE_D + STREAM_MAX) / (SHORT_MAX + 1) + 2;
+
+struct alignas(16) PanelSmem {
+  int32_t col[PT_STAGES][TILE_BUF];
+  float val[PT_STAGES][TILE_BUF];
+  float win[XWIN];
+  float prod[PROD_LEN];
+  uint64_t bar[PT_STAGES];
+  int32_t mid[MID_CAP];
+  int mid_n;
+  double wss[PT_THREADS / 32];
+};
+static_assert((TILE_BUF * 4) % 16 == 0, "stage buffers must stay 16-byte aligned");
+static_assert(TILE_D <= TILE_BUF, "row results reuse a col stage");
+
+// padded index of the product array: one pad word per 16, which makes the
+// thread-per-row pass bank-conflict free for rows of 16 (and light otherwise)
+__device__ __forceinline__ int pidx(int j) { return j + (j >> 4); }
+
+struct TileView {
+  int64_t e0;
+  int r0, rend, r1, cnt;
+};
+
+__device__ __forceinline__ TileView view(const TileDesc& d) {
+  TileView v;
+  v.e0 = d.e0;
+  v.r0 = d.r0;
+  v.cnt = (int)(d.packed & 0x3fffu);
+  v.rend = v.r0 + (int)((d.packed >> 14) & 0x3fffu);
+  v.r1 = v.rend + (int)((d.packed >> 28) & 1u);
+  return v;
+}
+
+__device__ __forceinline__ void issue_panel_tile(const TileView& v,
+                                                 const int32_t* __restrict__ col,
+                                                 const float* __restrict__ val, PanelSmem& S,
+                                                 int s, uint64_t pol) {
+  const int64_t a0 = v.e0 & ~3ll, a1 = (v.e0 + v.cnt + 3) & ~3ll;
+  const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
+  mbar_expect_tx(&S.bar[s], 2 * bytes);
+  if (bytes) {
+    bulk_g2s(S.col[s], col + a0, bytes, &S.bar[s], pol);
+    bulk_g2s(S.val[s], val + a0, bytes, &S.bar[s], pol);
   }
 }
 
 template <typename OT, bool SS>
-__global__ void __launch_bounds__(ST_THREADS)
-    k_stream(const OT* __restrict__ rp, const int32_t* __restrict__ col,
-             const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
-             const int32_t* __restrict__ tiles, const double* __restrict__ ss_in,
-             double* __restrict__ tile_ss, int evict_first) {
+__global__ void __launch_bounds__(PT_THREADS, 1)
+    k_panel(const OT* __restrict__ rp, const int32_t* __restrict__ col,
+            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
+            const TileDesc* __restrict__ desc, int64_t K, int64_t diag, int64_t xlen,
+            int use_win_i, const double* __restrict__ ss_in, double* __restrict__ tile_ss,
+            int evict_first) {
+  constexpr int SEGW = 2;  // window advance prefetched per thread (2 x 512 floats)
+  constexpr int RPF = 2;   // row pointers prefetched per thread
   extern __shared__ __align__(16) unsigned char smraw[];
-  int32_t* col_s = (int32_t*)smraw;                 // [TILE_BUF], reused as res_s
-  float* val_s = (float*)(col_s + TILE_BUF);        // [TILE_BUF]
-  float* prod_s = val_s + TILE_BUF;                 // [PROD_LEN]
-  __shared__ __align__(8) uint64_t bar;
-  __shared__ int mid_n;
-  __shared__ int32_t mid_s[TILE_D / (SHORT_MAX + 1) + 2];
-  float* res_s = (float*)col_s;
-
-  const int k = blockIdx.x, tid = threadIdx.x;
-  const int r0 = tiles[k], r1 = tiles[k + 1];
-  if (r0 == r1) {
-    if (SS && tid == 0) tile_ss[k] = 0.0;
-    return;
-  }
+  PanelSmem& S = *reinterpret_cast<PanelSmem*>(smraw);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t k0 = (K * (int64_t)blockIdx.x) / gridDim.x;
+  const int64_t k1 = (K * (int64_t)(blockIdx.x + 1)) / gridDim.x;
+  if (k0 >= k1) return;
+  const bool use_win = use_win_i != 0;
+  const int xl = (int)xlen, dg = (int)diag;  // columns are int32 (n < 2^31)
   const float alpha = alpha_of(ss_in);
-  const int64_t e0 = (int64_t)rp[r0];
-  const int64_t lastb = (int64_t)rp[r1 - 1], eend = (int64_t)rp[r1];
-  const bool last_long = (eend - lastb) > STREAM_MAX;
-  const int rend = last_long ? r1 - 1 : r1;
-  const int64_t e1 = last_long ? lastb : eend;
-  const int64_t a0 = e0 & ~3ll, a1 = (e1 + 3) & ~3ll;
-  const int cnt = (int)(e1 - e0), sh = (int)(e0 - a0);
+  uint64_t pol = 0;
+  TileView v = view(desc[k0]);
+  TileView vn = v;
+  if (k0 + 1 < k1) vn = view(desc[k0 + 1]);
   if (tid == 0) {
-    mid_n = 0;
-    if (a1 > a0) {
-      mbar_init(&bar, 1);
-      const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
-      const uint64_t pol = l2_policy(evict_first);
-      mbar_expect_tx(&bar, 2 * bytes);
-      bulk_g2s(col_s, col + a0, bytes, &bar, pol);
-      bulk_g2s(val_s, val + a0, bytes, &bar, pol);
+    pol = l2_policy(evict_first);
+    for (int s = 0; s < PT_STAGES; ++s) mbar_init(&S.bar[s], 1);
+    fence_mbar_init();
+    issue_panel_tile(v, col, val, S, 0, pol);
+  }
+  // initial window [whi(k0) - XWIN, whi(k0))
+  int whi = 0;
+  if (use_win) {
+    const int h = v.r1 + dg + XLEAD;
+    whi = h < xl ? h : xl;
+    for (int u = tid; u < XWIN; u += PT_THREADS) {
+      const int c = whi - XWIN + u;
+      if (c >= 0) S.win[c & (XWIN - 1)] = __ldg(x + c);
     }
   }
   __syncthreads();
-  if (a1 > a0) mbar_wait(&bar, 0);
-
-  // products p_j = val_j * x[col_j] (fp32, rounded once)
-  int i = tid;
-  for (; i + 3 * ST_THREADS < cnt; i += 4 * ST_THREADS) {
-    int c0 = col_s[sh + i], c1 = col_s[sh + i + ST_THREADS];
-    int c2 = col_s[sh + i + 2 * ST_THREADS], c3 = col_s[sh + i + 3 * ST_THREADS];
-    float x0 = __ldg(x + c0), x1 = __ldg(x + c1), x2 = __ldg(x + c2), x3 = __ldg(x + c3);
-    prod_s[pidx(i)] = __fmul_rn(val_s[sh + i], x0);
-    prod_s[pidx(i + ST_THREADS)] = __fmul_rn(val_s[sh + i + ST_THREADS], x1);
-    prod_s[pidx(i + 2 * ST_THREADS)] = __fmul_rn(val_s[sh + i + 2 * ST_THREADS], x2);
-    prod_s[pidx(i + 3 * ST_THREADS)] = __fmul_rn(val_s[sh + i + 3 * ST_THREADS], x3);
-  }
-  for (; i < cnt; i += ST_THREADS) prod_s[pidx(i)] = __fmul_rn(val_s[sh + i], __ldg(x + col_s[sh + i]));
-  __syncthreads();
-
-  // short rows: thread per row, sequential (canonical W = 1)
-  for (int r = r0 + tid; r < rend; r += ST_THREADS) {
-    const int b = (int)((int64_t)rp[r] - e0);
-    const int L = (int)((int64_t)rp[r + 1] - (int64_t)rp[r]);
-    if (L <= SHORT_MAX) {
-      float s = 0.f;
-      for (int t = 0; t < L; ++t) s = __fadd_rn(s, prod_s[pidx(b + t)]);
-      res_s[r - r0] = s;
-    } else {
-      mid_s[atomicAdd(&mid_n, 1)] = r;
+  float* __restrict__ pr = S.prod;
+  float* __restrict__ win = S.win;
+  int s = 0;
+  uint32_t ph = 0;
+  for (int64_t t = k0; t < k1; ++t) {
+    const bool has_next = t + 1 < k1;
+    if (tid == 0) {
+      S.mid_n = 0;
+      if (has_next) {  // the other stage held tile t-1, finished before the last barrier
+        fence_proxy_async();
+        issue_panel_tile(vn, col, val, S, s ^ 1, pol);
+      }
     }
-  }
-  __syncthreads();
-  // medium rows: warp per row (canonical W = 32)
-  const int warp = tid >> 5, lane = tid & 31;
-  for (int q = warp; q < mid_n; q += ST_THREADS / 32) {
-    const int r = mid_s[q];
-    const int b = (int)((int64_t)rp[r] - e0);
-    const int L = (int)((int64_t)rp[r + 1] - (int64_t)rp[r]);
-    float s = 0.f;
-    for (int t = lane; t < L; t += 32) s = __fadd_rn(s, prod_s[pidx(b + t)]);
+    const int nr = v.rend - v.r0;
+    // row pointers of this tile (prefetch)
+    OT rb[RPF], re[RPF];
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
-    if (lane == 0) res_s[r - r0] = s;
+    for (int u = 0; u < RPF; ++u) {
+      const int q = tid + u * PT_THREADS;
+      rb[u] = q < nr ? rp[v.r0 + q] : (OT)0;
+      re[u] = q < nr ? rp[v.r0 + q + 1] : (OT)0;
+    }
+    // window of this tile: [vlo, whi); warp 0 prefetches the advance for t+1
+    const int vlo = whi - XWIN > 0 ? whi - XWIN : 0;
+    const uint32_t span = use_win ? (uint32_t)(whi - vlo) : 0u;
+    int whi_next = whi, seg_lo = whi;
+    float segv[SEGW];
+    if (use_win && has_next) {
+      const int h = vn.r1 + dg + XLEAD;
+      whi_next = h < xl ? h : xl;
+      seg_lo = whi_next - whi > XWIN ? whi_next - XWIN : whi;
+#pragma unroll
+      for (int u = 0; u < SEGW; ++u) {
+        const int c = seg_lo + tid + PT_THREADS * u;
+        segv[u] = c < whi_next ? __ldg(x + c) : 0.f;
+      }
+    }
+    mbar_wait(&S.bar[s], ph);
+    const int cnt = v.cnt, sh = (int)(v.e0 & 3);
+    const int32_t* __restrict__ cs = S.col[s] + sh;
+    const float* __restrict__ vs = S.val[s] + sh;
+    // products p_j = val_j * x[col_j] (fp32, rounded once); window hits from smem
+    int j = tid;
+    for (; j + 3 * PT_THREADS < cnt; j += 4 * PT_THREADS) {
+      int c[4];
+      float xv[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) c[u] = cs[j + u * PT_THREADS];
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        xv[u] = (uint32_t)(c[u] - vlo) < span ? win[c[u] & (XWIN - 1)] : __ldg(x + c[u]);
+      const int pj = pidx(j);  // pidx(j + 512u) = pidx(j) + 544u
+#pragma unroll
+      for (int u = 0; u < 4; ++u) pr[pj + 544 * u] = __fmul_rn(vs[j + u * PT_THREADS], xv[u]);
+    }
+    for (; j < cnt; j += PT_THREADS) {
+      const int c = cs[j];
+      const float xv = (uint32_t)(c - vlo) < span ? win[c & (XWIN - 1)] : __ldg(x + c);
+      pr[pidx(j)] = __fmul_rn(vs[j], xv);
+    }
+    __syncthreads();
+    // advance the window to tile t+1 (tile t no longer reads it)
+    if (use_win && has_next) {
+#pragma unroll
+      for (int u = 0; u < SEGW; ++u) {
+        const int c = seg_lo + tid + PT_THREADS * u;
+        if (c < whi_next) win[c & (XWIN - 1)] = segv[u];
+      }
+      for (int c = seg_lo + PT_THREADS * SEGW + tid; c < whi_next; c += PT_THREADS)
+        win[c & (XWIN - 1)] = __ldg(x + c);
+    }
+    whi = whi_next;
+    float* res = reinterpret_cast<float*>(S.col[s]);  // col of this stage is dead now
+    // short rows: thread per row, sequential (canonical W = 1)
+    auto row_pass = [&](int q, OT p0, OT p1) {
+      const int b = (int)((int64_t)p0 - v.e0);
+      const int L = (int)(p1 - p0);
+      if (L <= SHORT_MAX) {
+        float acc = 0.f;
+        int jj = b;
+        const float* P = pr + pidx(b);
+        for (int w = 0; w < L; ++w) {
+          acc = __fadd_rn(acc, *P);
+          ++jj;
+          P += 1 + ((jj & 15) == 0);
+        }
+        res[q] = acc;
+      } else if (L <= WARP_MAX) {  // longer rows belong to k_cta_rows / k_hub_chunk
+        S.mid[atomicAdd(&S.mid_n, 1)] = q;
+      }
+    };
+#pragma unroll
+    for (int u = 0; u < RPF; ++u) {
+      const int q = tid + u * PT_THREADS;
+      if (q < nr) row_pass(q, rb[u], re[u]);
+    }
+    for (int q = tid + RPF * PT_THREADS; q < nr; q += PT_THREADS)
+      row_pass(q, rp[v.r0 + q], rp[v.r0 + q + 1]);
+    __syncthreads();
+    // medium rows: warp per row (canonical W = 32)
+    const int nmid = S.mid_n;
+    for (int m = warp; m < nmid; m += PT_THREADS / 32) {
+      const int q = S.mid[m];
+      const int64_t p0 = (int64_t)rp[v.r0 + q];
+      const int b = (int)(p0 - v.e0);
+      const int L = (int)((int64_t)rp[v.r0 + q + 1] - p0);
+      float acc = 0.f;
+      for (int u = lane; u < L; u += 32) acc = __fadd_rn(acc, pr[pidx(b + u)]);
+      acc = warp_tree(acc);
+      if (lane == 0) res[q] = acc;
+    }
+    __syncthreads();
+    double ssacc = 0.0;
+    auto emit = [&](int q, OT p0, OT p1) {
+      if ((int64_t)(p1 - p0) > WARP_MAX) return;  // written by k_cta_rows / k_hub_fix
+      const float o = __fmul_rn(res[q], alpha);
+      y[v.r0 + q] = o;
+      if (SS) ssacc += (double)o * (double)o;
+    };
+#pragma unroll
+    for (int u = 0; u < RPF; ++u) {
+      const int q = tid + u * PT_THREADS;
+      if (q < nr) emit(q, rb[u], re[u]);
+    }
+    for (int q = tid + RPF * PT_THREADS; q < nr; q += PT_THREADS)
+      emit(q, rp[v.r0 + q], rp[v.r0 + q + 1]);
+    if (SS) {
+      ssacc = warp_sum_d(ssacc);
+      if (lane == 0) S.wss[warp] = ssacc;
+      __syncthreads();
+      if (tid == 0) {
+        double a = 0.0;
+        for (int w = 0; w < PT_THREADS / 32; ++w) a += S.wss[w];
+        tile_ss[t] = a;
+      }
+    }
+    __syncthreads();
+    v = vn;
+    if (t + 2 < k1) vn = view(desc[t + 2]);
+    s ^= 1;
+    if (s == 0) ph ^= 1u;
   }
-  __syncthreads();
-  double acc = 0.0;
-  for (int r = r0 + tid; r < rend; r += ST_THREADS) {
-    const float v = __fmul_rn(res_s[r - r0], alpha);
-    y[r] = v;
-    if (SS) acc += (double)v * (double)v;
-  }
-  if (SS) block_sum_store<SS>(acc, tile_ss + k);
 }
 
-// canonical W = 256 sum of entries [b, b + L) of a row (L >= 256 assumed by class)
+// ------------------------------------------------------------- long rows
+template <typename OT, bool SS>
+__global__ void __launch_bounds__(256)
+    k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
+                const float* __restrict__ val, const float* __restrict__ x,
+                float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
+                const double* __restrict__ ss_in, double* __restrict__ row_ss) {
+  const int lane = threadIdx.x & 31;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const float alpha = alpha_of(ss_in);
+  for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < nrows; q += W) {
+    const int r = rows[q];
+    const int64_t b = (int64_t)rp[r];
+    const int L = (int)((int64_t)rp[r + 1] - b);
+    const int32_t* cc = col + b;
+    const float* vv = val + b;
+    float s = 0.f;
+    int j = lane;
+    for (; j + 96 < L; j += 128) {
+      const int c0 = __ldcs(cc + j), c1 = __ldcs(cc + j + 32), c2 = __ldcs(cc + j + 64),
+                c3 = __ldcs(cc + j + 96);
+      const float v0 = __ldcs(vv + j), v1 = __ldcs(vv + j + 32), v2 = __ldcs(vv + j + 64),
+                  v3 = __ldcs(vv + j + 96);
+      const float x0 = __ldg(x + c0), x1 = __ldg(x + c1), x2 = __ldg(x + c2), x3 = __ldg(x + c3);
+      s = __fadd_rn(s, __fmul_rn(v0, x0));
+      s = __fadd_rn(s, __fmul_rn(v1, x1));
+      s = __fadd_rn(s, __fmul_rn(v2, x2));
+      s = __fadd_rn(s, __fmul_rn(v3, x3));
+    }
+    for (; j < L; j += 32) s = __fadd_rn(s, __fmul_rn(__ldcs(vv + j), __ldg(x + __ldcs(cc + j))));
+    s = warp_tree(s);
+    if (lane == 0) {
+      const float v = __fmul_rn(s, alpha);
+      y[r] = v;
+      if (SS) row_ss[q] = (double)v * (double)v;
+    }
+  }
+}
+
+// canonical W = 256 sum of entries [b, b + L) of a row
 __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             const float* __restrict__ val,
                                             const float* __restrict__ x, int64_t b, int64_t L,
                                             float* red) {
   const int tid = threadIdx.x;
   float s = 0.f;
-#pragma unroll 8
-  for (int64_t t = tid; t < L; t += 256) {
-    const int c = __ldcs(col + b + t);
-    const float v = __ldcs(val + b + t);
-    s = __fadd_rn(s, __fmul_rn(v, __ldg(x + c)));
+  int64_t t = tid;
+  for (; t + 768 < L; t += 1024) {
+    const int c0 = __ldcs(col + b + t), c1 = __ldcs(col + b + t + 256),
+              c2 = __ldcs(col + b + t + 512), c3 = __ldcs(col + b + t + 768);
+    const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256),
+                v2 = __ldcs(val + b + t + 512), v3 = __ldcs(val + b + t + 768);
+    const float x0 = __ldg(x + c0), x1 = __ldg(x + c1), x2 = __ldg(x + c2), x3 = __ldg(x + c3);
+    s = __fadd_rn(s, __fmul_rn(v0, x0));
+    s = __fadd_rn(s, __fmul_rn(v1, x1));
+    s = __fadd_rn(s, __fmul_rn(v2, x2));
+    s = __fadd_rn(s, __fmul_rn(v3, x3));
   }
+  for (; t < L; t += 256) s = __fadd_rn(s, __fmul_rn(__ldcs(val + b + t), __ldg(x + __ldcs(col + b + t))));
   red[tid] = s;
   __syncthreads();
 #pragma unroll
@@ -209,11 +419,7 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
     __syncthreads();
   }
   float r = 0.f;
-  if (tid < 32) {
-    r = red[tid];
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) r = __fadd_rn(r, __shfl_xor_sync(0xffffffffu, r, o));
-  }
+  if (tid < 32) r = warp_tree(red[tid]);
   return r;  // valid in thread 0
 }
 
@@ -266,12 +472,23 @@ __global__ void k_hub_fix(const int32_t* __restrict__ hub_rows, const int32_t* _
 
 __global__ void __launch_bounds__(1024)
     k_ss_final(const double* __restrict__ a, int64_t na, const double* __restrict__ b, int64_t nb,
-               const double* __restrict__ c, int64_t nc, double* __restrict__ out) {
+               const double* __restrict__ c, int64_t nc, const double* __restrict__ d,
+               int64_t nd, double* __restrict__ out) {
+  __shared__ double wss[32];
   double acc = 0.0;
   for (int64_t i = threadIdx.x; i < na; i += 1024) acc += a[i];
   for (int64_t i = threadIdx.x; i < nb; i += 1024) acc += b[i];
   for (int64_t i = threadIdx.x; i < nc; i += 1024) acc += c[i];
-  block_sum_store<true>(acc, out);
+  for (int64_t i = threadIdx.x; i < nd; i += 1024) acc += d[i];
+  acc = warp_sum_d(acc);
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  if (lane == 0) wss[w] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int i = 0; i < 32; ++i) s += wss[i];
+    *out = s;
+  }
 }
 
 __global__ void k_scale(const float* __restrict__ u, float* __restrict__ x, int64_t n,
@@ -282,8 +499,34 @@ __global__ void k_scale(const float* __restrict__ u, float* __restrict__ x, int6
     x[i] = __fmul_rn(u[i], a);
 }
 
-constexpr size_t stream_smem_bytes() {
-  return sizeof(int32_t) * TILE_BUF + sizeof(float) * TILE_BUF + sizeof(float) * PROD_LEN;
+int g_num_sms = 0;
+
+int num_sms(int dev) {
+  if (!g_num_sms) cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+  return g_num_sms > 0 ? g_num_sms : 148;
+}
+
+template <typename OT, bool SS>
+void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
+  constexpr size_t smem = sizeof(PanelSmem);
+  static bool attr = false;
+  if (!attr) {
+    SPMV_CUDA(cudaFuncSetAttribute(k_panel<OT, SS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)smem));
+    attr = true;
+  }
+  static int per_sm = 0;
+  if (!per_sm) {
+    SPMV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_panel<OT, SS>, PT_THREADS,
+                                                            smem));
+    if (per_sm < 1) per_sm = 1;
+  }
+  const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(p->K, cap));
+  const int use_win = p->opts.smem_window ? 1 : 0;
+  k_panel<OT, SS><<<grid, PT_THREADS, smem, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
+                                                 p->d_desc, p->K, p->y_offset, p->x_len, use_win,
+                                                 ss_in, p->d_tile_ss, p->opts.evict_first);
 }
 
 template <typename OT>
@@ -291,28 +534,18 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
                 cudaStream_t s) {
   const OT* rp = (const OT*)p->d_rp;
   const bool SS = ss_out != nullptr;
-  const int ef = p->opts.evict_first;
   if (p->K) {
-    const size_t smem = stream_smem_bytes();
-    if (SS) {
-      static bool attr = false;
-      if (!attr) {
-        SPMV_CUDA(cudaFuncSetAttribute(k_stream<OT, true>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        attr = true;
-      }
-      k_stream<OT, true><<<(unsigned)p->K, ST_THREADS, smem, s>>>(
-          rp, p->d_col, p->d_val, x, y, p->d_tiles, ss_in, p->d_tile_ss, ef);
-    } else {
-      static bool attr = false;
-      if (!attr) {
-        SPMV_CUDA(cudaFuncSetAttribute(k_stream<OT, false>,
-                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        attr = true;
-      }
-      k_stream<OT, false><<<(unsigned)p->K, ST_THREADS, smem, s>>>(
-          rp, p->d_col, p->d_val, x, y, p->d_tiles, ss_in, p->d_tile_ss, ef);
-    }
+    if (SS) launch_panel<OT, true>(p, x, y, ss_in, s);
+    else launch_panel<OT, false>(p, x, y, ss_in, s);
+  }
+  if (p->n_warp) {
+    const unsigned g = (unsigned)std::min<int64_t>((p->n_warp + 7) / 8, (int64_t)num_sms(p->device) * 8);
+    if (SS)
+      k_warp_rows<OT, true><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, p->d_warp_rows,
+                                             p->n_warp, ss_in, p->d_warp_ss);
+    else
+      k_warp_rows<OT, false><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, p->d_warp_rows,
+                                              p->n_warp, ss_in, p->d_warp_ss);
   }
   if (p->n_cta) {
     if (SS)
@@ -335,8 +568,8 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
                                          p->d_chunk_part, ss_in, y, p->d_hub_ss);
   }
   if (SS)
-    k_ss_final<<<1, 1024, 0, s>>>(p->d_tile_ss, p->K, p->d_cta_ss, p->n_cta, p->d_hub_ss, p->n_hub,
-                                  ss_out);
+    k_ss_final<<<1, 1024, 0, s>>>(p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss,
+                                  p->n_cta, p->d_hub_ss, p->n_hub, ss_out);
   SPMV_LAUNCH_CHECK();
 }
 
@@ -369,6 +602,11 @@ void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
 
 }  // namespace
 
+int exec_launches(const spmv_plan_s* p, bool ss) {
+  return (p->K ? 1 : 0) + (p->n_warp ? 1 : 0) + (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0) +
+         (ss ? 1 : 0);
+}
+
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
           cudaStream_t s) {
   if (!p->permuted) SPMV_FAIL(SPMV_ESTATE, "spmv_exec before spmv_permute");
@@ -380,7 +618,9 @@ void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double*
 
 void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s) {
   if (iters < 1) SPMV_FAIL(SPMV_EINVAL, "iters must be >= 1");
-  if (p->world != 1) SPMV_FAIL(SPMV_EUNSUPPORTED, "spmv_iterate drives world == 1; use spmv_exec_scaled + collectives for world > 1");
+  if (p->world != 1)
+    SPMV_FAIL(SPMV_EUNSUPPORTED,
+              "spmv_iterate drives world == 1; use spmv_exec_scaled + collectives for world > 1");
   if (!p->permuted) SPMV_FAIL(SPMV_ESTATE, "spmv_iterate before spmv_permute");
   if (!p->d_u) {
     void* q = nullptr;

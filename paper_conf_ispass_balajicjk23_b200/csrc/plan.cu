@@ -207,12 +207,38 @@ __global__ void k_tiles(const OT* rp, int64_t nrows, int64_t K, int32_t* tiles) 
   }
 }
 
+template <typename OT>
+__global__ void k_tile_desc(const OT* rp, const int32_t* tiles, int64_t K, TileDesc* d) {
+  GRID_STRIDE(t, K) {
+    const int r0 = tiles[t], r1 = tiles[t + 1];
+    const int64_t e0 = (int64_t)rp[r0];
+    uint32_t cnt = 0, nr = 0, extra = 0;
+    if (r1 > r0) {
+      const int64_t lb = (int64_t)rp[r1 - 1], ee = (int64_t)rp[r1];
+      const bool last_long = (ee - lb) > STREAM_MAX;
+      cnt = (uint32_t)((last_long ? lb : ee) - e0);
+      nr = (uint32_t)((last_long ? r1 - 1 : r1) - r0);
+      extra = last_long ? 1u : 0u;
+    }
+    d[t].e0 = e0;
+    d[t].r0 = r0;
+    d[t].packed = cnt | (nr << 14) | (extra << 28);
+  }
+}
+
 // flags for a row-length predicate lo < L <= hi
 template <typename OT>
-__global__ void k_len_flag(const OT* rp, int64_t nrows, int64_t lo, int64_t hi, int32_t* f) {
+__global__ void k_len_flag(const OT* rp, int64_t nrows, int64_t lo, int64_t hi, int last_only,
+                           int32_t* f) {
   GRID_STRIDE(r, nrows) {
     int64_t L = (int64_t)rp[r + 1] - (int64_t)rp[r];
-    f[r] = (L > lo && L <= hi) ? 1 : 0;
+    bool ok = L > lo && L <= hi;
+    if (ok && last_only && r + 1 < nrows) {  // only the last row of a stream tile leaves it
+      const int64_t t0 = ((int64_t)rp[r] + r) / TILE_D;
+      const int64_t t1 = ((int64_t)rp[r + 1] + r + 1) / TILE_D;
+      ok = t1 != t0;
+    }
+    f[r] = ok ? 1 : 0;
   }
 }
 
@@ -270,7 +296,7 @@ __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* 
   int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t r = w; r < nrows; r += nw) {
     int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d;
-    if (L > STREAM_MAX) continue;
+    if (L > WARP_MAX) continue;  // longer rows: k_relabel_cta
     int64_t i = inv[rb + r];
     int64_t a = (int64_t)rpA[i];
     for (int64_t k = lane; k < L; k += 32) {
@@ -540,8 +566,8 @@ T d2h_one(const T* d, cudaStream_t s) {
 // flags -> ascending list of rows; returns count
 template <typename OT>
 int64_t class_list(const OT* rp, int64_t nrows, int64_t lo, int64_t hi, int32_t** out,
-                   int32_t* f, int64_t* pos, int64_t* tmp, cudaStream_t s) {
-  k_len_flag<OT><<<grid_for(nrows), TPB, 0, s>>>(rp, nrows, lo, hi, f);
+                   int32_t* f, int64_t* pos, int64_t* tmp, cudaStream_t s, int last_only = 0) {
+  k_len_flag<OT><<<grid_for(nrows), TPB, 0, s>>>(rp, nrows, lo, hi, last_only, f);
   exclusive_scan<int32_t>(f, nrows, pos, tmp, s);
   int64_t cnt = d2h_one(pos + nrows, s);
   *out = dalloc<int32_t>(cnt);
@@ -640,6 +666,8 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   p->K = nr ? (p->nnz_local + nr + TILE_D - 1) / TILE_D : 0;
   p->d_tiles = dalloc<int32_t>(p->K + 1);
   k_tiles<OT><<<grid_for(p->K + 1), TPB, 0, s>>>(rp, nr, p->K, p->d_tiles);
+  p->d_desc = dalloc<TileDesc>(p->K);
+  if (p->K) k_tile_desc<OT><<<grid_for(p->K), TPB, 0, s>>>(rp, p->d_tiles, p->K, p->d_desc);
   SPMV_LAUNCH_CHECK();
 
   // row classes + sort buckets
@@ -647,14 +675,15 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   int64_t* pos = dalloc<int64_t>(nr + 1);
   dfree(tmp);
   tmp = dalloc<int64_t>(scan_temp_len(std::max<int64_t>(nr, 1)));
-  p->n_cta = class_list<OT>(rp, nr, STREAM_MAX, CTA_MAX, &p->d_cta_rows, f, pos, tmp, s);
+  p->n_warp = class_list<OT>(rp, nr, STREAM_MAX, WARP_MAX, &p->d_warp_rows, f, pos, tmp, s, 1);
+  p->n_cta = class_list<OT>(rp, nr, WARP_MAX, CTA_MAX, &p->d_cta_rows, f, pos, tmp, s);
   p->n_hub = class_list<OT>(rp, nr, CTA_MAX, INT64_MAX, &p->d_hub_rows, f, pos, tmp, s);
   spmv_plan_s* ps = p;
   ps->n1 = class_list<OT>(rp, nr, 32, 128, &ps->s1, f, pos, tmp, s);
   ps->n2 = class_list<OT>(rp, nr, 128, 1024, &ps->s2, f, pos, tmp, s);
   ps->n3 = class_list<OT>(rp, nr, 1024, BIG_CHUNK, &ps->s3, f, pos, tmp, s);
   ps->nbig = class_list<OT>(rp, nr, BIG_CHUNK, INT64_MAX, &ps->big, f, pos, tmp, s);
-  ps->nlong = class_list<OT>(rp, nr, STREAM_MAX, INT64_MAX, &ps->longrows, f, pos, tmp, s);
+  ps->nlong = class_list<OT>(rp, nr, WARP_MAX, INT64_MAX, &ps->longrows, f, pos, tmp, s);
   // big row offsets in the key scratch
   ps->boff = dalloc<int64_t>(ps->nbig + 1);
   if (ps->nbig) {
@@ -703,6 +732,7 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   // exec scratch
   p->d_chunk_part = dalloc<double>(p->n_chunks);
   p->d_tile_ss = dalloc<double>(p->K);
+  p->d_warp_ss = dalloc<double>(p->n_warp);
   p->d_cta_ss = dalloc<double>(p->n_cta);
   p->d_hub_ss = dalloc<double>(p->n_hub);
   p->d_ss = dalloc<double>(4);
@@ -821,7 +851,8 @@ void plan_free(spmv_plan_s* p) {
   dfree(p->longrows);
   dfree(p->d_perm); dfree(p->d_inv);
   if (p->d_rp) { cudaFree(p->d_rp); p->d_rp = nullptr; }
-  dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows);
+  dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows); dfree(p->d_desc);
+  dfree(p->d_warp_rows); dfree(p->d_warp_ss);
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
   dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
   dfree(p->d_ss); dfree(p->d_u);

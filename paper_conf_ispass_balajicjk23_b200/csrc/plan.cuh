@@ -4,6 +4,14 @@
 
 #include "common.cuh"
 
+// 16-byte stream-tile descriptor (built by the plan, read by k_panel):
+// packed = cnt (entries streamed, 14 bits) | (rend - r0) << 14 | last_long << 28
+struct TileDesc {
+  int64_t e0;
+  int32_t r0;
+  uint32_t packed;
+};
+
 struct spmv_plan_s {
   int device = 0;
   spmv_opts_t opts{};
@@ -37,6 +45,9 @@ struct spmv_plan_s {
   // bins
   int64_t K = 0, n_cta = 0, n_hub = 0, n_chunks = 0, H = 0, max_hub_len = 0;
   int32_t* d_tiles = nullptr;      // [K+1]
+  TileDesc* d_desc = nullptr;      // [K]
+  int64_t n_warp = 0;
+  int32_t* d_warp_rows = nullptr;  // [n_warp]
   int32_t* d_cta_rows = nullptr;   // [n_cta]
   int32_t* d_hub_rows = nullptr;   // [n_hub]
   int32_t* d_hub_choff = nullptr;  // [n_hub+1] first chunk of each hub row
@@ -46,6 +57,7 @@ struct spmv_plan_s {
   // exec scratch
   double* d_chunk_part = nullptr;  // [n_chunks]
   double* d_tile_ss = nullptr;     // [K]
+  double* d_warp_ss = nullptr;     // [n_warp]
   double* d_cta_ss = nullptr;      // [n_cta]
   double* d_hub_ss = nullptr;      // [n_hub]
   double* d_ss = nullptr;          // [4] iterate scalars
@@ -75,5 +87,6 @@ void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStr
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
           cudaStream_t s);
 void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s);
+int exec_launches(const spmv_plan_s* p, bool ss);
 void scale_vec(const float* u, float* x, int64_t n, const double* ss, cudaStream_t s);
 }  // namespace spmv

@@ -39,14 +39,14 @@ class _Csr(ctypes.Structure):
 class _Opts(ctypes.Structure):
     _fields_ = [("l2_window", ctypes.c_int32), ("evict_first", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
-                ("device", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+                ("device", ctypes.c_int32), ("smem_window", ctypes.c_int32),
                 ("l2_hit_ratio", ctypes.c_double), ("reserved", ctypes.c_int64 * 8)]
 
 
 class _Info(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in (
         "n", "nnz", "row_begin", "row_end", "nnz_local", "x_len", "x_stride", "y_offset",
-        "n_tiles", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "hot_prefix", "ideal_bytes")] + \
+        "n_tiles", "n_warp_rows", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "hot_prefix", "ideal_bytes")] + \
         [(n, ctypes.c_int32) for n in ("offset_bytes", "world", "rank", "permuted",
                                        "l2_window_bytes", "r0", "r1", "r2")]
 
@@ -84,7 +84,7 @@ def lib() -> ctypes.CDLL:
             "spmv_scale_vec": (i32, [vp, vp, i64, dp, vp]),
             "spmv_plan_info": (i32, [vp, ctypes.POINTER(_Info)]),
             "spmv_export_csr": (i32, [vp, vp, vp, vp, vp]),
-            "spmv_export_bins": (i32, [vp, vp, vp, vp, vp, vp, vp]),
+            "spmv_export_bins": (i32, [vp, vp, vp, vp, vp, vp, vp, vp]),
             "spmv_export_partition": (i32, [vp, vp]),
             "spmv_export_inverse": (i32, [vp, vp, vp]),
             "spmv_destroy": (None, [vp]),
@@ -134,7 +134,8 @@ class Plan:
     """
 
     def __init__(self, row_ptr, col, val, perm=None, *, world=1, rank=0, l2_window=True,
-                 evict_first=True, l2_hit_ratio=1.0, permute=True, stream=None):
+                 evict_first=True, l2_hit_ratio=1.0, smem_window=True, permute=True,
+                 stream=None):
         import torch
         assert row_ptr.is_cuda and col.is_cuda and val.is_cuda
         assert col.dtype == torch.int32 and val.dtype == torch.float32
@@ -154,6 +155,7 @@ class Plan:
         o.world, o.rank = world, rank
         o.l2_window, o.evict_first = int(l2_window), int(evict_first)
         o.l2_hit_ratio = l2_hit_ratio
+        o.smem_window = int(smem_window)
         o.device = row_ptr.device.index if row_ptr.device.index is not None else -1
         h = ctypes.c_void_p()
         _check(lib().spmv_plan(ctypes.byref(A), _ptr(perm), ctypes.byref(o), ctypes.byref(h)))
@@ -219,10 +221,12 @@ class Plan:
         import torch
         i = self.info()
         mk = lambda m: torch.empty(max(m, 0), dtype=torch.int32, device=self.device)  # noqa: E731
-        d = {"tiles": mk(i["n_tiles"] + 1), "cta_rows": mk(i["n_cta_rows"]),
+        d = {"tiles": mk(i["n_tiles"] + 1), "warp_rows": mk(i["n_warp_rows"]),
+             "cta_rows": mk(i["n_cta_rows"]),
              "hub_rows": mk(i["n_hub_rows"]), "chunk_row": mk(i["n_hub_chunks"]),
              "chunk_idx": mk(i["n_hub_chunks"])}
-        _check(lib().spmv_export_bins(self._h, _ptr(d["tiles"]), _ptr(d["cta_rows"]),
+        _check(lib().spmv_export_bins(self._h, _ptr(d["tiles"]), _ptr(d["warp_rows"]),
+                                      _ptr(d["cta_rows"]),
                                       _ptr(d["hub_rows"]), _ptr(d["chunk_row"]),
                                       _ptr(d["chunk_idx"]), _stream_ptr(stream)))
         return d

@@ -62,7 +62,8 @@ def long_rows_matrix(seed=0):
     L = rng.integers(0, 20, n)
     L[rng.random(n) < 0.3] = 0
     special = {5: 40000, 17: 16385, 99: 16384, 1000: 9000, 1001: 2049, 1002: 2048, 2500: 700,
-               2501: 33, 2502: 32, 29999: 70000}
+               2501: 33, 2502: 32, 3000: 3000, 3001: 5, 3002: 7, 3500: 1500, 3501: 3,
+               29999: 70000}
     for r, l in special.items():
         L[r] = l
     rp = np.concatenate([[0], np.cumsum(L)])
@@ -110,7 +111,8 @@ def test_permute_and_bins_bitexact(dev, name, make, which):
     assert np.array_equal(v.view(np.int32), Bv.view(np.int32))
     bins = {k: t.cpu().numpy() for k, t in P.export_bins().items()}
     assert np.array_equal(bins["tiles"], oplan.tile_bounds(Bp))
-    cta, hub, cr, ci = oplan.row_classes(Bp)
+    warp, cta, hub, cr, ci = oplan.row_classes(Bp)
+    assert np.array_equal(bins["warp_rows"], warp)
     assert np.array_equal(bins["cta_rows"], cta)
     assert np.array_equal(bins["hub_rows"], hub)
     assert np.array_equal(bins["chunk_row"], cr) and np.array_equal(bins["chunk_idx"], ci)
@@ -288,3 +290,24 @@ def test_bench_config_full_size(dev):
     yA, absA = cref.spmv_neumaier(A.row_ptr, A.col, A.val, w.x)
     _check_y(y, permute.permute_vec(yA, perm), permute.permute_vec(absA, perm), "all rows")
     P.close()
+
+
+@pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("sbm16x1024", "longrows", "stencil24")])
+def test_smem_window_and_l2_options_bitwise(dev, name, make):
+    """The x window, L2 policies and an unaligned x (window disabled) change
+    where x is read from, never y."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = make()
+    perm, _ = spmv.reorder(A.row_ptr, A.col, "rabbit")
+    x = torch.from_numpy(synth.vector(A.n, 8)).to(dev)
+    ys = []
+    for kw in ({}, {"smem_window": False}, {"evict_first": False, "l2_window": False}):
+        P = mk_plan(A, perm, dev, **kw)
+        xB = P.permute_vec(x)
+        ys.append(P.exec(xB).cpu().numpy())
+        buf = torch.zeros(A.n + 1, device=dev)
+        buf[1:] = xB                      # 4-byte offset: not 16-byte aligned
+        ys.append(P.exec(buf[1:]).cpu().numpy())
+        P.close()
+    for y in ys[1:]:
+        assert np.array_equal(y.view(np.int32), ys[0].view(np.int32))

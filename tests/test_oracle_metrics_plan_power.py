@@ -59,7 +59,8 @@ def test_tile_bounds(case):
     elif case == "empty_tail":
         rp = np.concatenate([np.arange(0, 3000, 3), np.full(5000, 2997)]).astype(np.int64)
     elif case == "long_rows":
-        L = np.array([1, 5000, 2, 2048, 2049, 0, 0, 40000, 3] + [7] * 500)
+        L = np.array([1, 5000, 2, 2048, 2049, 0, 0, 40000, 3, 128, 129, 127, 0, 5, 1024, 1023,
+                      1025, 0, 1, 512, 513, 511] + [7] * 500)
         rp = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
     else:
         rp = np.zeros(1, np.int64)
@@ -71,19 +72,32 @@ def test_tile_bounds(case):
         for r in range(b[k], b[k + 1]):
             assert tid[r] == k
     L = np.diff(rp)
+    inside = plan.stream_rows(rp)
+    warp, cta, hub, _, _ = plan.row_classes(rp)
+    assert sorted(np.nonzero(~inside)[0].tolist()) == sorted(warp.tolist() + cta.tolist() + hub.tolist())
     for k in range(len(b) - 1):
         rows = range(b[k], b[k + 1])
-        long_ = [r for r in rows if L[r] > plan.STREAM_MAX]
-        assert not long_ or long_ == [b[k + 1] - 1]          # only the last row can be long
-        s = sum(L[r] for r in rows if L[r] <= plan.STREAM_MAX)
-        assert s < 2 * plan.TILE_D
+        huge = [r for r in rows if L[r] >= plan.TILE_D]
+        assert not huge or huge == [b[k + 1] - 1]            # rows >= TILE_D are always last
+        out = [r for r in rows if not inside[r] and L[r] <= plan.WARP_MAX]
+        assert not out or out == [b[k + 1] - 1]              # short-enough rows leave only if last
+        s = sum(L[r] for r in rows if inside[r])
+        assert s < plan.TILE_D + plan.STREAM_MAX             # fits the tile buffer
         assert b[k + 1] - b[k] <= plan.TILE_D
 
 
 def test_row_classes_and_partition():
-    L = np.array([1, 5000, 2, 2048, 2049, 0, 16384, 16385, 40000, 3])
+    # a 1500-entry row followed by short rows of the same tile stays inside it
+    rp2 = np.array([0, 1500, 1502, 1507])
+    assert plan.stream_rows(rp2).all() and len(plan.row_classes(rp2)[0]) == 0
+    L = np.array([1, 5000, 2, 2048, 2049, 0, 16384, 16385, 40000, 3, 1024, 1025])
     rp = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
-    cta, hub, cr, ci = plan.row_classes(rp)
+    warp, cta, hub, cr, ci = plan.row_classes(rp)
+    # c_r = row_ptr[r] + r = 0, 2, 5003, 5006, 7055, 9105, 9106, 25491, 41877, 81878,
+    # 81882, 82907 -> tiles (// 8192) 0,0,0,0,0,1,1,3,5,9,9,10: row 3 (L 2048) is
+    # not last in its tile and stays inside it; rows with L > 2048 never do
+    assert plan.TILE_D == 8192
+    assert warp.tolist() == [11]
     assert cta.tolist() == [1, 4, 6]
     assert hub.tolist() == [7, 8]
     assert cr.tolist() == [7, 7] + [8, 8, 8]
