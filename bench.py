@@ -149,7 +149,10 @@ def run_gpu(args):
     if A.nnz < 2**31:
         rp_d = rp_d.to(torch.int32)
     flush = torch.empty(512 * 2**20 // 4, dtype=torch.float32, device=dev)
-    stream = torch.cuda.current_stream()
+    # a dedicated (non-legacy) stream: the L2 access-policy window of spmv_exec
+    # is a stream attribute and cannot be set on the legacy default stream
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
     line = None
     for ordering in orderings:
         perm, st = reorder_cached(args, w.name, A, ordering)

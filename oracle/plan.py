@@ -5,7 +5,7 @@ The paper runs cuSPARSE and never describes scheduling (Alg. 1
 is a plain "parfor row"); these are build constants (reading c23), RE-DECLARED
 here from DESIGN.md §Plan, not imported from the library:
 
-  TILE_D      = 8192   stream tile "diagonal": row r (r < N) belongs to tile
+  TILE_D      = 3072   stream tile "diagonal": row r (r < N) belongs to tile
                         k = floor((row_ptr[r] + r) / TILE_D); tiles
                         k = 0 .. K-1, K = ceil((NZ + N) / TILE_D);
                         bounds b_k = lower_bound_{r in [0,N]}(row_ptr[r] + r >= k*TILE_D)
@@ -31,7 +31,7 @@ from __future__ import annotations
 
 import numpy as np
 
-TILE_D = 8192
+TILE_D = 3072
 STREAM_MAX = 1024
 WARP_MAX = 2048
 CTA_MAX = 16384

@@ -11,7 +11,7 @@ namespace spmv {
 
 // Build constants (reading c23; declared in include/spmv.h and DESIGN.md §Plan;
 // re-declared independently in oracle/plan.py).
-constexpr int TILE_D = 8192;        // stream tile: rows + entries
+constexpr int TILE_D = 3072;        // stream tile: rows + entries
 constexpr int STREAM_MAX = 1024;    // longest row computed inside a stream tile
 constexpr int SHORT_MAX = 32;       // canonical order: sequential up to here
 constexpr int WARP_MAX = 2048;      // warp-per-row class upper bound (canonical W = 32)

@@ -3,7 +3,7 @@
 // Alg. 1 of the paper:  Y[row] += values[i] * X[coords[i]].
 // B200 design:
 //   k_panel      persistent CTAs over contiguous row panels of stream tiles
-//                (TILE_D = 8192 rows+entries, row aligned); a 2-stage ring of
+//                (TILE_D = 3072 rows+entries, row aligned); a 2-stage ring of
 //                cp.async.bulk (TMA bulk engine) + mbarrier copies of tile
 //                col/val (L2 evict_first); a sliding
 //                shared-memory x window follows the diagonal, so
@@ -100,13 +100,13 @@ __device__ __forceinline__ double warp_sum_d(double s) {
 
 // ------------------------------------------------------------ stream tiles
 // k_panel: persistent CTAs, each over a contiguous range of stream tiles (a
-// panel of consecutive rows), one CTA of 16 warps per SM.  Thread 0 keeps the
+// panel of consecutive rows), two CTAs of 16 warps per SM.  Thread 0 keeps the
 // next tile in flight while the current one is computed (2-stage ring) with
 // cp.async.bulk copies (TMA bulk engine) of the tile's col / val (L2
 // evict_first), completing on per-stage mbarriers; tile descriptors are
 // precomputed by the plan and prefetched, so the producer has no dependent
-// loads on its path.  Tiles are large (TILE_D = 8192 rows+entries, ~64 KB of
-// matrix) so per-tile bookkeeping is amortised over ~16 entries per thread.
+// loads on its path.  Tiles are large (TILE_D = 3072 rows+entries, ~24 KB of
+// matrix) so per-tile bookkeeping is amortised over ~6 entries per thread.
 // x is read through a SLIDING WINDOW: a shared-memory ring of XWIN floats that
 // holds x[c] at slot c % XWIN for c in [whi(t) - XWIN, whi(t)), whi(t) =
 // (last row of tile t) + XLEAD.  Community-ordered matrices put most columns
@@ -170,14 +170,14 @@ __device__ __forceinline__ void issue_panel_tile(const TileView& v,
 }
 
 template <typename OT, bool SS>
-__global__ void __launch_bounds__(PT_THREADS, 1)
+__global__ void __launch_bounds__(PT_THREADS, 2)
     k_panel(const OT* __restrict__ rp, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
             const TileDesc* __restrict__ desc, int64_t K, int64_t diag, int64_t xlen,
             int use_win_i, const double* __restrict__ ss_in, double* __restrict__ tile_ss,
             int evict_first) {
-  constexpr int SEGW = 2;  // window advance prefetched per thread (2 x 512 floats)
-  constexpr int RPF = 2;   // row pointers prefetched per thread
+  constexpr int SEGW = 1;  // window advance prefetched per thread (512 floats)
+  constexpr int RPF = 1;   // row pointers prefetched per thread
   extern __shared__ __align__(16) unsigned char smraw[];
   PanelSmem& S = *reinterpret_cast<PanelSmem*>(smraw);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;

@@ -94,10 +94,11 @@ def test_row_classes_and_partition():
     rp = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
     warp, cta, hub, cr, ci = plan.row_classes(rp)
     # c_r = row_ptr[r] + r = 0, 2, 5003, 5006, 7055, 9105, 9106, 25491, 41877, 81878,
-    # 81882, 82907 -> tiles (// 8192) 0,0,0,0,0,1,1,3,5,9,9,10: row 3 (L 2048) is
-    # not last in its tile and stays inside it; rows with L > 2048 never do
-    assert plan.TILE_D == 8192
-    assert warp.tolist() == [11]
+    # 81882, 82907 -> tiles (// 3072) 0,0,1,1,2,2,2,8,13,26,26,26: rows 3 and 11
+    # (1024 < L <= 2048) are last in their tile; row 10 is not; rows with
+    # L > 2048 (1, 4, 6) never stay inside a tile
+    assert plan.TILE_D == 3072
+    assert warp.tolist() == [3, 11]
     assert cta.tolist() == [1, 4, 6]
     assert hub.tolist() == [7, 8]
     assert cr.tolist() == [7, 7] + [8, 8, 8]
