@@ -280,9 +280,20 @@ __global__ void k_colcnt(const int32_t* colA, const int32_t* perm, int64_t nnz, 
 
 __global__ void k_first_cold(const uint32_t* cnt, int64_t n, int64_t nnz,
                              unsigned long long* H) {
+  // smallest j with !(colcnt_B[j] * N > NZ): warp-level min first, one atomic per warp
+  unsigned long long best = ~0ull;
   GRID_STRIDE(j, n) {
-    if (!((int64_t)cnt[j] * n > nnz)) atomicMin(H, (unsigned long long)j);
+    if (!((int64_t)cnt[j] * n > nnz)) {
+      best = (unsigned long long)j;
+      break;  // grid-stride order is ascending per thread
+    }
   }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    unsigned long long other = __shfl_xor_sync(0xffffffffu, best, o);
+    best = other < best ? other : best;
+  }
+  if ((threadIdx.x & 31) == 0 && best != ~0ull) atomicMin(H, best);
 }
 
 // ------------------------------------------------------------- P A P^T data
