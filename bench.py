@@ -7,7 +7,7 @@ N = 1: workload = BASELINE.json configs[1] (planted-community SBM, 4M rows,
 64M nnz).  Input prep (host RABBIT / RABBIT++ reorder, GPU plan + P A P^T)
 happens once and is reported separately (PAPER.md:221 amortisation).  A
 step is one spmv_exec y_B = B x_B over the whole matrix with x_B, B resident
-in HBM; L2 is flushed (512 MiB write) before every step, outside the CUDA
+in HBM; L2 is flushed (512 MiB read) before every step, outside the CUDA
 events that time it, so each step pays compulsory traffic like the paper's
 ideal model (PAPER.md:96-98).  value = ideal bytes / step time (GB/s);
 runtime / ideal = peak / value.
@@ -148,7 +148,14 @@ def run_gpu(args):
     val_d = torch.from_numpy(A.val).to(dev)
     if A.nnz < 2**31:
         rp_d = rp_d.to(torch.int32)
-    flush = torch.empty(512 * 2**20 // 4, dtype=torch.float32, device=dev)
+    # L2 flush by READING 512 MiB (4x L2): leaves L2 full of clean lines, so the
+    # timed step pays compulsory DRAM reads without write-backs of the flush
+    flush = torch.zeros(512 * 2**20 // 4, dtype=torch.float32, device=dev)
+    sink = torch.zeros((), dtype=torch.float32, device=dev)
+
+    def flush_l2():
+        torch.sum(flush, dim=0, out=sink)
+
     # a dedicated (non-legacy) stream: the L2 access-policy window of spmv_exec
     # is a stream attribute and cannot be set on the legacy default stream
     stream = torch.cuda.Stream()
@@ -161,7 +168,7 @@ def run_gpu(args):
         perm_d = torch.from_numpy(perm).to(dev)
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        P = spmv.Plan(rp_d, col_d, val_d, perm_d, world=world, rank=rank)
+        P = spmv.Plan(rp_d, col_d, val_d, perm_d, world=world, rank=rank, variant=args.variant)
         torch.cuda.synchronize()
         plan_s = time.perf_counter() - t0
         info = P.info()
@@ -198,7 +205,7 @@ def run_gpu(args):
                 state["t"] = t + 1
             launches += 1  # exec_scaled's fixed-order norm reduction
         for _ in range(args.warmup):
-            flush.zero_()
+            flush_l2()
             step()
         torch.cuda.synchronize()
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
@@ -212,7 +219,7 @@ def run_gpu(args):
             time.sleep(0.3)
         wall0 = time.perf_counter()
         for i in range(K):
-            flush.zero_()
+            flush_l2()
             ev[i][0].record(stream)
             step()
             ev[i][1].record(stream)
@@ -262,8 +269,9 @@ def run_gpu(args):
                               "parallelism": f"row-block x{world}" if world > 1 else "1 GPU",
                               "step": "spmv_exec" if world == 1 else
                               "exec_scaled + all_reduce + all_gather (power iteration)",
-                              "l2": "flushed before every step (512 MiB write, outside the events)",
+                              "l2": "flushed before every step (512 MiB read, outside the events)",
                               "ideal_bytes": ideal, "ideal_bytes_paper_4B_offsets": ideal_p96,
+                              "kernel_variant": ["lane", "panel"][args.variant],
                               "wall_s_timed_region": round(wall, 4)}
             line["runtime_over_ideal"] = round(hbm / gbs, 4)
             line["gflops"] = round(2 * A.nnz / (ms * 1e-3) / 1e9, 2)
@@ -401,6 +409,7 @@ def main():
     ap.add_argument("--seed", type=int, default=20230423)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--perm-cache", default=None, help="dev only: memoise reorder results here")
+    ap.add_argument("--variant", type=int, default=0, help="short-row kernel: 0 lane, 1 panel")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

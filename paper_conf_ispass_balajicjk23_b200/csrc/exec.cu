@@ -19,6 +19,7 @@
 //                (power-iteration norm; deterministic).
 // No tensor cores: SpMV is not a dense contraction (AI <= 0.25 flop/B).
 #include <cmath>
+#include <cstdlib>
 
 #include "plan.cuh"
 
@@ -529,16 +530,229 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
                                                  ss_in, p->d_tile_ss, p->opts.evict_first);
 }
 
+// --------------------------------------------------------- lane-per-row
+// k_lane (variant 1): persistent CTAs over contiguous panels of 256-row
+// blocks, lane per row.  A lane streams its row's col/val straight from
+// global memory with 128-bit loads of aligned 4-entry chunks (L2 evict_first
+// hint, L1 allocating, so the 32 rows of a warp share their lines across the
+// chunk steps) and sums the row sequentially (canonical W = 1, L <= 32);
+// rows with 32 < L <= 2048 are taken by the whole warp (canonical W = 32,
+// coalesced 128-byte loads); longer rows belong to k_cta_rows / k_hub_*.
+// x comes from the same sliding shared-memory window as k_panel (one CTA
+// barrier per 256-row block).  No staging of the matrix in shared memory.
+constexpr int LN_THREADS = 256;
+constexpr int LN_WARPS = LN_THREADS / 32;
+constexpr int LN_CTAS_PER_SM = 8;
+
+__device__ __forceinline__ float lds_f32(uint32_t saddr) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(saddr));
+  return v;
+}
+
+// 256-bit (one full 32-byte sector) streaming loads, sm_100: LDG.E.NA.256,
+// not allocated in L1, with an L2 eviction-priority hint
+__device__ __forceinline__ void ld_v8_stream(const int32_t* p, uint64_t pol, int (&r)[8]) {
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7])
+      : "l"(p), "l"(pol));
+}
+
+__device__ __forceinline__ void ld_v8_stream(const float* p, uint64_t pol, float (&r)[8]) {
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+      : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
+        "=f"(r[7])
+      : "l"(p), "l"(pol));
+}
+
+__device__ __forceinline__ int4 ld_v4_hint(const int32_t* p, uint64_t pol) {
+  int4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
+
+__device__ __forceinline__ float4 ld_v4_hint(const float* p, uint64_t pol) {
+  float4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+      : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
+
+template <typename OT, bool SS>
+__global__ void __launch_bounds__(LN_THREADS)
+    k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
+           const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
+           int64_t nrows, int64_t diag, int64_t xlen, int use_win_i,
+           const double* __restrict__ ss_in, double* __restrict__ blk_ss, int evict_first) {
+  __shared__ float win[XWIN];
+  __shared__ double wss[2][LN_WARPS];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
+  const int64_t b0 = (NB * (int64_t)blockIdx.x) / gridDim.x;
+  const int64_t b1 = (NB * (int64_t)(blockIdx.x + 1)) / gridDim.x;
+  if (b0 >= b1) return;
+  const bool use_win = use_win_i != 0;
+  const int xl = (int)xlen, dg = (int)diag;
+  const float alpha = alpha_of(ss_in);
+  const uint64_t pol = l2_policy(evict_first);
+  const uint32_t wbase = smem_u32(win);
+  auto blk_end = [&](int64_t b) {
+    const int64_t e = (b + 1) * LN_THREADS;
+    return (int)(e < nrows ? e : nrows);
+  };
+  int whi = 0;
+  if (use_win) {
+    const int h = blk_end(b0) + dg + XLEAD;
+    whi = h < xl ? h : xl;
+    for (int u = tid; u < XWIN; u += LN_THREADS) {
+      const int c = whi - XWIN + u;
+      if (c >= 0) win[c & (XWIN - 1)] = __ldg(x + c);
+    }
+  }
+  __syncthreads();
+  int sb = 0;
+  // row pointers of the first block (later blocks are prefetched one ahead)
+  int64_t a_n = 0, e_n = 0;
+  {
+    const int r = (int)(b0 * LN_THREADS) + tid;
+    if (r < blk_end(b0)) {
+      a_n = (int64_t)rp[r];
+      e_n = (int64_t)rp[r + 1];
+    }
+  }
+  for (int64_t blk = b0; blk < b1; ++blk) {
+    const int R0 = (int)(blk * LN_THREADS), R1 = blk_end(blk);
+    const int r = R0 + tid;
+    const int64_t a = a_n, e = e_n;
+    if (blk + 1 < b1) {
+      const int rn = R1 + tid;
+      a_n = e_n = 0;
+      if (rn < blk_end(blk + 1)) {
+        a_n = (int64_t)rp[rn];
+        e_n = (int64_t)rp[rn + 1];
+      }
+    }
+    // window advance for the next block: loads issued now, stored after this
+    // block's rows (into slots this block does not read)
+    int whi_next = whi, seg_lo = whi;
+    float segv = 0.f;
+    if (use_win && blk + 1 < b1) {
+      const int h = blk_end(blk + 1) + dg + XLEAD;
+      whi_next = h < xl ? h : xl;
+      seg_lo = whi_next - whi > XWIN ? whi_next - XWIN : whi;
+      if (seg_lo + tid < whi_next) segv = __ldg(x + seg_lo + tid);
+    }
+    const int vlo = whi_next - XWIN > 0 ? whi_next - XWIN : 0;
+    const uint32_t span = (use_win && whi > vlo) ? (uint32_t)(whi - vlo) : 0u;
+    const int L = (int)(e - a);
+    float res = 0.f;
+    if (L <= SHORT_MAX) {  // canonical W = 1: sequential, 4-entry aligned chunks
+      // Branch-free slots: every slot of a chunk holds a valid column of some
+      // row (or the zero tail padding), so its x read is always safe; slots
+      // outside [a, e) contribute an exact +0 (res starts at +0 and is never -0).
+      const int32_t* cp = col + (a & ~7ll);
+      const float* vp = val + (a & ~7ll);
+      const int lo = (int)(a & 7), hi = lo + L;
+      for (int k = 0; k < hi; k += 8) {
+        int cc[8];
+        float vv[8], xv[8];
+        ld_v8_stream(cp + k, pol, cc);
+        ld_v8_stream(vp + k, pol, vv);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const bool inw = (uint32_t)(cc[i] - vlo) < span;
+          const float xs = lds_f32(wbase + (((uint32_t)cc[i] & (XWIN - 1)) << 2));
+          float xg = 0.f;
+          if (!inw) xg = __ldg(x + cc[i]);
+          xv[i] = inw ? xs : xg;
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const float p = __fmul_rn(vv[i], xv[i]);
+          res = __fadd_rn(res, (k + i >= lo && k + i < hi) ? p : 0.f);
+        }
+      }
+    }
+    unsigned m = __ballot_sync(0xffffffffu, L > SHORT_MAX && L <= WARP_MAX);
+    while (m) {  // canonical W = 32: strided partials + xor tree
+      const int src = __ffs(m) - 1;
+      m &= m - 1;
+      const int64_t aa = __shfl_sync(0xffffffffu, a, src);
+      const int LL = __shfl_sync(0xffffffffu, L, src);
+      float acc = 0.f;
+      for (int u = lane; u < LL; u += 32) {
+        const int c = __ldcs(col + aa + u);
+        const float xv = (uint32_t)(c - vlo) < span ? win[c & (XWIN - 1)] : __ldg(x + c);
+        acc = __fadd_rn(acc, __fmul_rn(__ldcs(val + aa + u), xv));
+      }
+      acc = warp_tree(acc);
+      if (lane == src) res = acc;
+    }
+    double ssacc = 0.0;
+    if (r < R1 && L <= WARP_MAX) {
+      const float o = __fmul_rn(res, alpha);
+      y[r] = o;
+      if (SS) ssacc = (double)o * (double)o;
+    }
+    if (use_win && blk + 1 < b1) {
+      if (seg_lo + tid < whi_next) win[(seg_lo + tid) & (XWIN - 1)] = segv;
+      for (int c = seg_lo + LN_THREADS + tid; c < whi_next; c += LN_THREADS)
+        win[c & (XWIN - 1)] = __ldg(x + c);
+    }
+    if (SS) {
+      ssacc = warp_sum_d(ssacc);
+      if (lane == 0) wss[sb][warp] = ssacc;
+    }
+    __syncthreads();  // window advance visible; wss[sb] complete
+    if (SS && tid == 0) {
+      double t = 0.0;
+      for (int w = 0; w < LN_WARPS; ++w) t += wss[sb][w];
+      blk_ss[blk] = t;
+    }
+    sb ^= 1;
+    whi = whi_next;
+  }
+}
+
+template <typename OT, bool SS>
+void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
+  static int occ = 0;
+  if (!occ) {
+    SPMV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_lane<OT, SS>, LN_THREADS, 0));
+    occ = std::max(occ, 1);
+  }
+  int lim = LN_CTAS_PER_SM;
+  if (const char* e = getenv("SPMV_LANE_CTAS")) lim = atoi(e);  // dev knob
+  const int per_sm = std::max(1, std::min(occ, lim));
+  const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
+  const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
+  const int use_win = p->opts.smem_window ? 1 : 0;
+  k_lane<OT, SS><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
+                                             p->nrows, p->y_offset, p->x_len, use_win, ss_in,
+                                             p->d_blk_ss, p->opts.evict_first);
+}
+
 template <typename OT>
 void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
                 cudaStream_t s) {
   const OT* rp = (const OT*)p->d_rp;
   const bool SS = ss_out != nullptr;
-  if (p->K) {
+  const bool lane_mode = p->opts.variant != 1;
+  if (lane_mode) {
+    if (p->nrows) {
+      if (SS) launch_lane<OT, true>(p, x, y, ss_in, s);
+      else launch_lane<OT, false>(p, x, y, ss_in, s);
+    }
+  } else if (p->K) {
     if (SS) launch_panel<OT, true>(p, x, y, ss_in, s);
     else launch_panel<OT, false>(p, x, y, ss_in, s);
   }
-  if (p->n_warp) {
+  if (p->n_warp && !lane_mode) {
     const unsigned g = (unsigned)std::min<int64_t>((p->n_warp + 7) / 8, (int64_t)num_sms(p->device) * 8);
     if (SS)
       k_warp_rows<OT, true><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, p->d_warp_rows,
@@ -567,9 +781,15 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
       k_hub_fix<false><<<g, 128, 0, s>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub,
                                          p->d_chunk_part, ss_in, y, p->d_hub_ss);
   }
-  if (SS)
-    k_ss_final<<<1, 1024, 0, s>>>(p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss,
-                                  p->n_cta, p->d_hub_ss, p->n_hub, ss_out);
+  if (SS) {
+    if (lane_mode)
+      k_ss_final<<<1, 1024, 0, s>>>(p->d_blk_ss, (p->nrows + LN_THREADS - 1) / LN_THREADS,
+                                    nullptr, 0, p->d_cta_ss, p->n_cta, p->d_hub_ss, p->n_hub,
+                                    ss_out);
+    else
+      k_ss_final<<<1, 1024, 0, s>>>(p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss,
+                                    p->n_cta, p->d_hub_ss, p->n_hub, ss_out);
+  }
   SPMV_LAUNCH_CHECK();
 }
 
@@ -603,8 +823,9 @@ void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
 }  // namespace
 
 int exec_launches(const spmv_plan_s* p, bool ss) {
-  return (p->K ? 1 : 0) + (p->n_warp ? 1 : 0) + (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0) +
-         (ss ? 1 : 0);
+  const bool lane_mode = p->opts.variant != 1;
+  return (lane_mode ? (p->nrows ? 1 : 0) : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
+         (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0) + (ss ? 1 : 0);
 }
 
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,

@@ -743,6 +743,7 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   // exec scratch
   p->d_chunk_part = dalloc<double>(p->n_chunks);
   p->d_tile_ss = dalloc<double>(p->K);
+  p->d_blk_ss = dalloc<double>((nr + 255) / 256);
   p->d_warp_ss = dalloc<double>(p->n_warp);
   p->d_cta_ss = dalloc<double>(p->n_cta);
   p->d_hub_ss = dalloc<double>(p->n_hub);
@@ -865,7 +866,7 @@ void plan_free(spmv_plan_s* p) {
   dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows); dfree(p->d_desc);
   dfree(p->d_warp_rows); dfree(p->d_warp_ss);
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
-  dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
+  dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_blk_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
   dfree(p->d_ss); dfree(p->d_u);
 }
 

@@ -40,7 +40,8 @@ class _Opts(ctypes.Structure):
     _fields_ = [("l2_window", ctypes.c_int32), ("evict_first", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("smem_window", ctypes.c_int32),
-                ("l2_hit_ratio", ctypes.c_double), ("reserved", ctypes.c_int64 * 8)]
+                ("l2_hit_ratio", ctypes.c_double), ("variant", ctypes.c_int64),
+                ("reserved", ctypes.c_int64 * 7)]
 
 
 class _Info(ctypes.Structure):
@@ -134,8 +135,8 @@ class Plan:
     """
 
     def __init__(self, row_ptr, col, val, perm=None, *, world=1, rank=0, l2_window=True,
-                 evict_first=True, l2_hit_ratio=1.0, smem_window=True, permute=True,
-                 stream=None):
+                 evict_first=True, l2_hit_ratio=1.0, smem_window=True, variant=0,
+                 permute=True, stream=None):
         import torch
         assert row_ptr.is_cuda and col.is_cuda and val.is_cuda
         assert col.dtype == torch.int32 and val.dtype == torch.float32
@@ -156,6 +157,7 @@ class Plan:
         o.l2_window, o.evict_first = int(l2_window), int(evict_first)
         o.l2_hit_ratio = l2_hit_ratio
         o.smem_window = int(smem_window)
+        o.variant = int(variant)
         o.device = row_ptr.device.index if row_ptr.device.index is not None else -1
         h = ctypes.c_void_p()
         _check(lib().spmv_plan(ctypes.byref(A), _ptr(perm), ctypes.byref(o), ctypes.byref(h)))

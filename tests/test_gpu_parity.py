@@ -292,7 +292,7 @@ def test_bench_config_full_size(dev):
     P.close()
 
 
-@pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("sbm16x1024", "longrows", "stencil24")])
+@pytest.mark.parametrize("name,make", CASES)
 def test_smem_window_and_l2_options_bitwise(dev, name, make):
     """The x window, L2 policies and an unaligned x (window disabled) change
     where x is read from, never y."""
@@ -301,7 +301,8 @@ def test_smem_window_and_l2_options_bitwise(dev, name, make):
     perm, _ = spmv.reorder(A.row_ptr, A.col, "rabbit")
     x = torch.from_numpy(synth.vector(A.n, 8)).to(dev)
     ys = []
-    for kw in ({}, {"smem_window": False}, {"evict_first": False, "l2_window": False}):
+    for kw in ({}, {"smem_window": False}, {"evict_first": False, "l2_window": False},
+               {"variant": 1}, {"variant": 1, "smem_window": False}):
         P = mk_plan(A, perm, dev, **kw)
         xB = P.permute_vec(x)
         ys.append(P.exec(xB).cpu().numpy())
