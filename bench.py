@@ -280,7 +280,7 @@ def run_gpu(args):
                                 "peak": hbm, "unit": "GB/s",
                                 "frac": round(kern_bytes / (ms * 1e-3) / 1e9 / hbm, 4),
                                 "traffic": tr.get("dram_bytes") if tr else None,
-                                "kernel": "k_stream (+k_cta_rows/k_hub_* if present)",
+                                "kernel": ["k_lane", "k_panel"][args.variant] + " (+k_cta_rows/k_hub_* if present)",
                                 "peak_source": peak_src,
                                 "algorithmic_bytes_per_launch": kern_bytes}
             line["e2e"] = e2e
