@@ -657,6 +657,7 @@ __global__ void __launch_bounds__(LN_THREADS)
       const int32_t* cp = col + (a & ~7ll);
       const float* vp = val + (a & ~7ll);
       const int lo = (int)(a & 7), hi = lo + L;
+#pragma unroll 2
       for (int k = 0; k < hi; k += 8) {
         int cc[8];
         float vv[8], xv[8];

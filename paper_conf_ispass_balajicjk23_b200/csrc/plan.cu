@@ -743,7 +743,7 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   // exec scratch
   p->d_chunk_part = dalloc<double>(p->n_chunks);
   p->d_tile_ss = dalloc<double>(p->K);
-  p->d_blk_ss = dalloc<double>((nr + 255) / 256);
+  p->d_blk_ss = dalloc<double>((nr + 63) / 64);  // >= blocks of k_lane (>= 64 rows each)
   p->d_warp_ss = dalloc<double>(p->n_warp);
   p->d_cta_ss = dalloc<double>(p->n_cta);
   p->d_hub_ss = dalloc<double>(p->n_hub);

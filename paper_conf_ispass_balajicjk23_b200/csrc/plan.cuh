@@ -57,7 +57,7 @@ struct spmv_plan_s {
   // exec scratch
   double* d_chunk_part = nullptr;  // [n_chunks]
   double* d_tile_ss = nullptr;     // [K]
-  double* d_blk_ss = nullptr;      // [ceil(nrows/256)] (lane variant)
+  double* d_blk_ss = nullptr;      // [ceil(nrows/64)] per-block sumsq (lane variant)
   double* d_warp_ss = nullptr;     // [n_warp]
   double* d_cta_ss = nullptr;      // [n_cta]
   double* d_hub_ss = nullptr;      // [n_hub]
