@@ -133,10 +133,15 @@ def run_gpu(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.single_device:  # test mode: every rank on cuda:0 (gloo only)
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(args.backend)
     w, gen_s = load_workload(args.config)
     A = w.A
     hbm, peak_src = peaks()
@@ -198,8 +203,16 @@ def run_gpu(args):
                 t = state["t"]
                 ss_out = ss[t & 1:(t & 1) + 1]
                 P.exec_scaled(state["xa"], state["xb"][off:off + nr], state["ss_in"], ss_out)
-                dist.all_reduce(ss_out)
-                dist.all_gather_into_tensor(state["xb"], state["xb"][off:off + M])
+                if args.backend == "nccl":
+                    dist.all_reduce(ss_out)
+                    dist.all_gather_into_tensor(state["xb"], state["xb"][off:off + M])
+                else:  # gloo test path: host staging
+                    h = ss_out.cpu()
+                    dist.all_reduce(h)
+                    ss_out.copy_(h)
+                    hx = state["xb"].cpu()
+                    dist.all_gather_into_tensor(hx, hx[off:off + M].clone())
+                    state["xb"].copy_(hx)
                 state["ss_in"] = ss_out
                 state["xa"], state["xb"] = state["xb"], state["xa"]
                 state["t"] = t + 1
@@ -232,7 +245,12 @@ def run_gpu(args):
         ms = sum(times) / K
         if world > 1:
             t = torch.tensor([ms], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            if args.backend == "nccl":
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            else:
+                h = t.cpu()
+                dist.all_reduce(h, op=dist.ReduceOp.MAX)
+                t.copy_(h)
             ms = float(t.item())
         # warm (no flush) back-to-back
         torch.cuda.synchronize()
@@ -257,9 +275,11 @@ def run_gpu(args):
             res["dram_over_ideal_ncu"] = tr.get("dram_bytes", 0) / ideal
         results[ordering] = res
         if is_main:
-            e2e = None
             if world == 1:
                 e2e = e2e_measure(P, A, w.x, args, dev, ideal)
+            else:
+                e2e = e2e_dist_measure(P, loc, w.x, perm, step_state=state, step=step, args=args,
+                                       dev=dev, ideal=ideal, world=world)
             line = dict(metric=METRIC, value=round(gbs, 2), unit="GB/s", n_gpus=world, steps=K,
                         warmup=args.warmup, ms_per_step=round(ms, 5), higher_is_better=True,
                         scaling="strong", vs_baseline=None, dtype="f32",
@@ -344,6 +364,47 @@ def e2e_measure(P, A, x_host, args, dev, ideal):
             "path": "pinned H2D x -> spmv_permute_vec -> spmv_exec -> spmv_permute_vec^T -> D2H y"}
 
 
+def e2e_dist_measure(P, loc, x_host, perm, step_state, step, args, dev, ideal, world):
+    """N > 1: per step, pinned H2D of this rank's slice of x_B into its segment of
+    the padded x, the distributed step (exec_scaled + all-reduce + all-gather),
+    D2H of the 8-byte norm; max over ranks of the per-step time."""
+    import torch
+    import torch.distributed as dist
+    b0, b1 = P.export_partition()[loc.rank], P.export_partition()[loc.rank + 1]
+    xB = P.permute_vec(torch.from_numpy(x_host).to(dev))  # setup, outside the timed region
+    xs = xB[b0:b1].cpu().pin_memory()
+    ssh = torch.empty(1, dtype=torch.float64).pin_memory()
+    off = loc.y_offset
+
+    def e2e_step():
+        step_state["xa"][off:off + (b1 - b0)].copy_(xs, non_blocking=True)
+        step()
+        ssh.copy_(step_state["ss_in"], non_blocking=True)
+
+    for _ in range(args.warmup):
+        e2e_step()
+    torch.cuda.synchronize()
+    dist.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(args.steps):
+        e2e_step()
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / args.steps
+    t = torch.tensor([ms], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX) if args.backend == "gloo" else None
+    if args.backend == "nccl":
+        td = t.to(dev)
+        dist.all_reduce(td, op=dist.ReduceOp.MAX)
+        t = td.cpu()
+    ms = float(t.item())
+    return {"value": round(ideal / (ms * 1e-3) / 1e9, 2), "unit": "GB/s", "ms_per_step": round(ms, 5),
+            "h2d_bytes_per_step": 4 * int(P.info()["n"]), "d2h_bytes_per_step": 8 * world,
+            "path": "pinned H2D of each rank's x slice -> spmv_exec_scaled -> NCCL all-reduce "
+                    "+ all-gather -> D2H of the norm (summed over ranks)"}
+
+
 # ------------------------------------------------------------------- oracle
 def cpu_baseline(A, x, ideal_bytes, budget_s=10.0, steps=None, warmup=0):
     """The oracle as it stands (plain C fp64 CSR loop, OpenMP over all host
@@ -410,6 +471,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--perm-cache", default=None, help="dev only: memoise reorder results here")
     ap.add_argument("--variant", type=int, default=0, help="short-row kernel: 0 lane, 1 panel")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="collectives for N > 1 (gloo: host-staged, test only)")
+    ap.add_argument("--single-device", action="store_true",
+                    help="test only: put every rank on cuda:0 (with --backend gloo)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -16,6 +16,8 @@ here from DESIGN.md §Plan, not imported from the library:
   WARP_MAX    = 2048   last-in-tile rows with STREAM_MAX < L <= WARP_MAX: one
                         warp per row
   CTA_MAX     = 16384  WARP_MAX < L <= CTA_MAX (any position): one CTA per row
+  SHORT_MAX   = 32     lane variant: L <= SHORT_MAX lane per row; the MID list
+                        (SHORT_MAX < L <= WARP_MAX, any position) one warp per row
   HUB_CHUNK   = 16384  L > CTA_MAX: hub row cut into ceil(L / HUB_CHUNK)
                         chunks of HUB_CHUNK entries (merge-path split)
 
@@ -31,6 +33,7 @@ from __future__ import annotations
 
 import numpy as np
 
+SHORT_MAX = 32
 TILE_D = 3072
 STREAM_MAX = 1024
 WARP_MAX = 2048
@@ -81,6 +84,13 @@ def row_classes(row_ptr):
             ch_i.append(c)
     return (np.array(warp, np.int64), np.array(cta, np.int64), np.array(hub, np.int64),
             np.array(ch_r, np.int64), np.array(ch_i, np.int64))
+
+
+def mid_rows(row_ptr) -> np.ndarray:
+    """Rows computed warp-per-row by the lane variant: SHORT_MAX < L <= WARP_MAX
+    (SHORT_MAX = 32), ascending, any position."""
+    L = np.diff(np.asarray(row_ptr, np.int64))
+    return np.nonzero((L > SHORT_MAX) & (L <= WARP_MAX))[0].astype(np.int64)
 
 
 def stream_rows(row_ptr) -> np.ndarray:

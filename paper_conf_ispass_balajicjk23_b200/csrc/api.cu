@@ -175,6 +175,7 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->y_offset = p->y_offset;
   info->n_tiles = p->K;
   info->n_warp_rows = p->n_warp;
+  info->n_mid_rows = p->n_mid;
   info->n_cta_rows = p->n_cta;
   info->n_hub_rows = p->n_hub;
   info->n_hub_chunks = p->n_chunks;
@@ -221,14 +222,16 @@ spmv_status spmv_export_csr(spmv_plan_t p, int64_t* row_ptr, int32_t* col, float
   API_END
 }
 
-spmv_status spmv_export_bins(spmv_plan_t p, int32_t* tiles, int32_t* warp_rows, int32_t* cta_rows,
-                             int32_t* hub_rows, int32_t* chunk_row, int32_t* chunk_idx,
-                             void* stream) {
+spmv_status spmv_export_bins(spmv_plan_t p, int32_t* tiles, int32_t* mid_rows, int32_t* warp_rows,
+                             int32_t* cta_rows, int32_t* hub_rows, int32_t* chunk_row,
+                             int32_t* chunk_idx, void* stream) {
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_export_bins: NULL plan");
   use_device(p);
   cudaStream_t s = S(stream);
   if (tiles) SPMV_CUDA(cudaMemcpyAsync(tiles, p->d_tiles, 4 * (p->K + 1), cudaMemcpyDeviceToDevice, s));
+  if (mid_rows && p->n_mid)
+    SPMV_CUDA(cudaMemcpyAsync(mid_rows, p->d_mid_rows, 4 * p->n_mid, cudaMemcpyDeviceToDevice, s));
   if (warp_rows && p->n_warp)
     SPMV_CUDA(cudaMemcpyAsync(warp_rows, p->d_warp_rows, 4 * p->n_warp, cudaMemcpyDeviceToDevice, s));
   if (cta_rows && p->n_cta)

@@ -536,8 +536,9 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 // global memory with 128-bit loads of aligned 4-entry chunks (L2 evict_first
 // hint, L1 allocating, so the 32 rows of a warp share their lines across the
 // chunk steps) and sums the row sequentially (canonical W = 1, L <= 32);
-// rows with 32 < L <= 2048 are taken by the whole warp (canonical W = 32,
-// coalesced 128-byte loads); longer rows belong to k_cta_rows / k_hub_*.
+// rows with L > 32 are load-balanced over their own kernels (k_warp_rows over
+// the plan's mid list, k_cta_rows, k_hub_*), so a power-law row never stalls a
+// block of short rows.
 // x comes from the same sliding shared-memory window as k_panel (one CTA
 // barrier per 256-row block).  No staging of the matrix in shared memory.
 constexpr int LN_THREADS = 256;
@@ -678,23 +679,8 @@ __global__ void __launch_bounds__(LN_THREADS)
         }
       }
     }
-    unsigned m = __ballot_sync(0xffffffffu, L > SHORT_MAX && L <= WARP_MAX);
-    while (m) {  // canonical W = 32: strided partials + xor tree
-      const int src = __ffs(m) - 1;
-      m &= m - 1;
-      const int64_t aa = __shfl_sync(0xffffffffu, a, src);
-      const int LL = __shfl_sync(0xffffffffu, L, src);
-      float acc = 0.f;
-      for (int u = lane; u < LL; u += 32) {
-        const int c = __ldcs(col + aa + u);
-        const float xv = (uint32_t)(c - vlo) < span ? win[c & (XWIN - 1)] : __ldg(x + c);
-        acc = __fadd_rn(acc, __fmul_rn(__ldcs(val + aa + u), xv));
-      }
-      acc = warp_tree(acc);
-      if (lane == src) res = acc;
-    }
     double ssacc = 0.0;
-    if (r < R1 && L <= WARP_MAX) {
+    if (r < R1 && L <= SHORT_MAX) {  // longer rows: k_warp_rows / k_cta_rows / k_hub_*
       const float o = __fmul_rn(res, alpha);
       y[r] = o;
       if (SS) ssacc = (double)o * (double)o;
@@ -753,14 +739,17 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
     if (SS) launch_panel<OT, true>(p, x, y, ss_in, s);
     else launch_panel<OT, false>(p, x, y, ss_in, s);
   }
-  if (p->n_warp && !lane_mode) {
-    const unsigned g = (unsigned)std::min<int64_t>((p->n_warp + 7) / 8, (int64_t)num_sms(p->device) * 8);
-    if (SS)
-      k_warp_rows<OT, true><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, p->d_warp_rows,
-                                             p->n_warp, ss_in, p->d_warp_ss);
-    else
-      k_warp_rows<OT, false><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, p->d_warp_rows,
-                                              p->n_warp, ss_in, p->d_warp_ss);
+  {
+    const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
+    const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
+    double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
+    if (nw) {
+      const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
+      if (SS)
+        k_warp_rows<OT, true><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
+      else
+        k_warp_rows<OT, false><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
+    }
   }
   if (p->n_cta) {
     if (SS)
@@ -785,8 +774,8 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   if (SS) {
     if (lane_mode)
       k_ss_final<<<1, 1024, 0, s>>>(p->d_blk_ss, (p->nrows + LN_THREADS - 1) / LN_THREADS,
-                                    nullptr, 0, p->d_cta_ss, p->n_cta, p->d_hub_ss, p->n_hub,
-                                    ss_out);
+                                    p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta, p->d_hub_ss,
+                                    p->n_hub, ss_out);
     else
       k_ss_final<<<1, 1024, 0, s>>>(p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss,
                                     p->n_cta, p->d_hub_ss, p->n_hub, ss_out);
@@ -825,7 +814,7 @@ void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
 
 int exec_launches(const spmv_plan_s* p, bool ss) {
   const bool lane_mode = p->opts.variant != 1;
-  return (lane_mode ? (p->nrows ? 1 : 0) : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
+  return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0) : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
          (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0) + (ss ? 1 : 0);
 }
 

@@ -687,6 +687,7 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   dfree(tmp);
   tmp = dalloc<int64_t>(scan_temp_len(std::max<int64_t>(nr, 1)));
   p->n_warp = class_list<OT>(rp, nr, STREAM_MAX, WARP_MAX, &p->d_warp_rows, f, pos, tmp, s, 1);
+  p->n_mid = class_list<OT>(rp, nr, SHORT_MAX, WARP_MAX, &p->d_mid_rows, f, pos, tmp, s);
   p->n_cta = class_list<OT>(rp, nr, WARP_MAX, CTA_MAX, &p->d_cta_rows, f, pos, tmp, s);
   p->n_hub = class_list<OT>(rp, nr, CTA_MAX, INT64_MAX, &p->d_hub_rows, f, pos, tmp, s);
   spmv_plan_s* ps = p;
@@ -745,6 +746,7 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   p->d_tile_ss = dalloc<double>(p->K);
   p->d_blk_ss = dalloc<double>((nr + 63) / 64);  // >= blocks of k_lane (>= 64 rows each)
   p->d_warp_ss = dalloc<double>(p->n_warp);
+  p->d_mid_ss = dalloc<double>(p->n_mid);
   p->d_cta_ss = dalloc<double>(p->n_cta);
   p->d_hub_ss = dalloc<double>(p->n_hub);
   p->d_ss = dalloc<double>(4);
@@ -864,7 +866,7 @@ void plan_free(spmv_plan_s* p) {
   dfree(p->d_perm); dfree(p->d_inv);
   if (p->d_rp) { cudaFree(p->d_rp); p->d_rp = nullptr; }
   dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows); dfree(p->d_desc);
-  dfree(p->d_warp_rows); dfree(p->d_warp_ss);
+  dfree(p->d_warp_rows); dfree(p->d_warp_ss); dfree(p->d_mid_rows); dfree(p->d_mid_ss);
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
   dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_blk_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
   dfree(p->d_ss); dfree(p->d_u);

@@ -47,7 +47,9 @@ struct spmv_plan_s {
   int32_t* d_tiles = nullptr;      // [K+1]
   TileDesc* d_desc = nullptr;      // [K]
   int64_t n_warp = 0;
-  int32_t* d_warp_rows = nullptr;  // [n_warp]
+  int32_t* d_warp_rows = nullptr;  // [n_warp] k_panel: last-in-tile rows, 1024 < L <= 2048
+  int64_t n_mid = 0;
+  int32_t* d_mid_rows = nullptr;   // [n_mid] k_lane: all rows with 32 < L <= 2048
   int32_t* d_cta_rows = nullptr;   // [n_cta]
   int32_t* d_hub_rows = nullptr;   // [n_hub]
   int32_t* d_hub_choff = nullptr;  // [n_hub+1] first chunk of each hub row
@@ -59,6 +61,7 @@ struct spmv_plan_s {
   double* d_tile_ss = nullptr;     // [K]
   double* d_blk_ss = nullptr;      // [ceil(nrows/64)] per-block sumsq (lane variant)
   double* d_warp_ss = nullptr;     // [n_warp]
+  double* d_mid_ss = nullptr;      // [n_mid]
   double* d_cta_ss = nullptr;      // [n_cta]
   double* d_hub_ss = nullptr;      // [n_hub]
   double* d_ss = nullptr;          // [4] iterate scalars

@@ -47,7 +47,8 @@ class _Opts(ctypes.Structure):
 class _Info(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in (
         "n", "nnz", "row_begin", "row_end", "nnz_local", "x_len", "x_stride", "y_offset",
-        "n_tiles", "n_warp_rows", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "hot_prefix", "ideal_bytes")] + \
+        "n_tiles", "n_warp_rows", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "n_mid_rows",
+        "hot_prefix", "ideal_bytes")] + \
         [(n, ctypes.c_int32) for n in ("offset_bytes", "world", "rank", "permuted",
                                        "l2_window_bytes", "r0", "r1", "r2")]
 
@@ -85,7 +86,7 @@ def lib() -> ctypes.CDLL:
             "spmv_scale_vec": (i32, [vp, vp, i64, dp, vp]),
             "spmv_plan_info": (i32, [vp, ctypes.POINTER(_Info)]),
             "spmv_export_csr": (i32, [vp, vp, vp, vp, vp]),
-            "spmv_export_bins": (i32, [vp, vp, vp, vp, vp, vp, vp, vp]),
+            "spmv_export_bins": (i32, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
             "spmv_export_partition": (i32, [vp, vp]),
             "spmv_export_inverse": (i32, [vp, vp, vp]),
             "spmv_destroy": (None, [vp]),
@@ -223,11 +224,13 @@ class Plan:
         import torch
         i = self.info()
         mk = lambda m: torch.empty(max(m, 0), dtype=torch.int32, device=self.device)  # noqa: E731
-        d = {"tiles": mk(i["n_tiles"] + 1), "warp_rows": mk(i["n_warp_rows"]),
+        d = {"tiles": mk(i["n_tiles"] + 1), "mid_rows": mk(i["n_mid_rows"]),
+             "warp_rows": mk(i["n_warp_rows"]),
              "cta_rows": mk(i["n_cta_rows"]),
              "hub_rows": mk(i["n_hub_rows"]), "chunk_row": mk(i["n_hub_chunks"]),
              "chunk_idx": mk(i["n_hub_chunks"])}
-        _check(lib().spmv_export_bins(self._h, _ptr(d["tiles"]), _ptr(d["warp_rows"]),
+        _check(lib().spmv_export_bins(self._h, _ptr(d["tiles"]), _ptr(d["mid_rows"]),
+                                      _ptr(d["warp_rows"]),
                                       _ptr(d["cta_rows"]),
                                       _ptr(d["hub_rows"]), _ptr(d["chunk_row"]),
                                       _ptr(d["chunk_idx"]), _stream_ptr(stream)))

@@ -112,6 +112,7 @@ def test_permute_and_bins_bitexact(dev, name, make, which):
     bins = {k: t.cpu().numpy() for k, t in P.export_bins().items()}
     assert np.array_equal(bins["tiles"], oplan.tile_bounds(Bp))
     warp, cta, hub, cr, ci = oplan.row_classes(Bp)
+    assert np.array_equal(bins["mid_rows"], oplan.mid_rows(Bp))
     assert np.array_equal(bins["warp_rows"], warp)
     assert np.array_equal(bins["cta_rows"], cta)
     assert np.array_equal(bins["hub_rows"], hub)

@@ -99,6 +99,7 @@ def test_row_classes_and_partition():
     # L > 2048 (1, 4, 6) never stay inside a tile
     assert plan.TILE_D == 3072
     assert warp.tolist() == [3, 11]
+    assert plan.mid_rows(rp).tolist() == [3, 10, 11]
     assert cta.tolist() == [1, 4, 6]
     assert hub.tolist() == [7, 8]
     assert cr.tolist() == [7, 7] + [8, 8, 8]
