@@ -269,7 +269,7 @@ def run_gpu(args):
                "n_communities": st.n_communities, "largest_comm_frac": st.largest_comm_frac,
                "modularity": st.modularity, "skew": st.skew, "hubs": st.n_hubs,
                "H": info["hot_prefix"], "tiles": info["n_tiles"], "cta_rows": info["n_cta_rows"],
-               "hub_rows": info["n_hub_rows"], "l2_window_bytes": info["l2_window_bytes"]}
+               "hub_rows": info["n_hub_rows"], "l2_window_bytes": P.info()["l2_window_bytes"]}
         tr = ncu_traffic(w.name, ordering)
         if tr:
             res["dram_over_ideal_ncu"] = tr.get("dram_bytes", 0) / ideal

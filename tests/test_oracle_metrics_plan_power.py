@@ -140,3 +140,13 @@ def test_power_iteration_perron_root():
     val = np.concatenate([D[r, c] for r, c in enumerate(rows)]).astype(np.float32)
     x, lam = power.power_iteration(rp, col, val, np.ones(A.n, np.float32), 400)
     assert abs(lam - ev) / ev < 1e-3
+
+
+def test_mid_rows():
+    rng = np.random.default_rng(4)
+    L = rng.integers(0, 40, 700)
+    L[[3, 300, 650]] = [100, 2048, 5000]
+    rp = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
+    mid = plan.mid_rows(rp)
+    assert set(mid.tolist()) == {r for r in range(len(L)) if 32 < L[r] <= 2048}
+    assert np.all(np.diff(mid) > 0)
