@@ -531,197 +531,102 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 }
 
 // --------------------------------------------------------- lane-per-row
-// k_lane (variant 1): persistent CTAs over contiguous panels of 256-row
-// blocks, lane per row.  A lane streams its row's col/val straight from
-// global memory with 128-bit loads of aligned 4-entry chunks (L2 evict_first
-// hint, L1 allocating, so the 32 rows of a warp share their lines across the
-// chunk steps) and sums the row sequentially (canonical W = 1, L <= 32);
-// rows with L > 32 are load-balanced over their own kernels (k_warp_rows over
-// the plan's mid list, k_cta_rows, k_hub_*), so a power-law row never stalls a
-// block of short rows.
-// x comes from the same sliding shared-memory window as k_panel (one CTA
-// barrier per 256-row block).  No staging of the matrix in shared memory.
+// k_lane (variant 0, default): lane per row for rows with L <= 32, canonical
+// W = 1 (sequential), grid-stride over 256-row blocks (CTA i takes blocks i,
+// i + G, ...).  A lane streams its row in 8-entry, 32-byte-aligned chunks with
+// sm_100 256-bit loads (LDG.E.NA.256: one full sector per lane, not allocated
+// in L1), and gathers x with L1-allocating loads: community order
+// puts a block's columns on few lines, which L1 and L2 keep on chip.  Rows
+// with L > 32 are skipped here and load-balanced over their own kernels
+// (k_warp_rows over the plan's mid list, k_cta_rows, k_hub_*).
+// Design note (profiles/r01_summary.md, r26): a persistent variant with a
+// sliding shared-memory x window, one barrier per block and evict_first
+// stream hints ran 1.25x slower than this plain form on SBM 4M/64M.
 constexpr int LN_THREADS = 256;
 constexpr int LN_WARPS = LN_THREADS / 32;
-constexpr int LN_CTAS_PER_SM = 8;
+constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 
-__device__ __forceinline__ float lds_f32(uint32_t saddr) {
-  float v;
-  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(saddr));
-  return v;
-}
-
-// 256-bit (one full 32-byte sector) streaming loads, sm_100: LDG.E.NA.256,
-// not allocated in L1, with an L2 eviction-priority hint
-__device__ __forceinline__ void ld_v8_stream(const int32_t* p, uint64_t pol, int (&r)[8]) {
-  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+__device__ __forceinline__ void ld_v8_stream(const int32_t* p, int (&r)[8]) {
+  asm("ld.global.nc.L1::no_allocate.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
         "=r"(r[7])
-      : "l"(p), "l"(pol));
+      : "l"(p));
 }
 
-__device__ __forceinline__ void ld_v8_stream(const float* p, uint64_t pol, float (&r)[8]) {
-  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+__device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
+  asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
       : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
         "=f"(r[7])
-      : "l"(p), "l"(pol));
-}
-
-__device__ __forceinline__ int4 ld_v4_hint(const int32_t* p, uint64_t pol) {
-  int4 r;
-  asm("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
-      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
-      : "l"(p), "l"(pol));
-  return r;
-}
-
-__device__ __forceinline__ float4 ld_v4_hint(const float* p, uint64_t pol) {
-  float4 r;
-  asm("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
-      : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
-      : "l"(p), "l"(pol));
-  return r;
+      : "l"(p));
 }
 
 template <typename OT, bool SS>
 __global__ void __launch_bounds__(LN_THREADS)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
-           int64_t nrows, int64_t diag, int64_t xlen, int use_win_i,
-           const double* __restrict__ ss_in, double* __restrict__ blk_ss, int evict_first) {
-  __shared__ float win[XWIN];
-  __shared__ double wss[2][LN_WARPS];
+           int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss) {
+  __shared__ double wss[LN_WARPS];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
-  const int64_t b0 = (NB * (int64_t)blockIdx.x) / gridDim.x;
-  const int64_t b1 = (NB * (int64_t)(blockIdx.x + 1)) / gridDim.x;
-  if (b0 >= b1) return;
-  const bool use_win = use_win_i != 0;
-  const int xl = (int)xlen, dg = (int)diag;
   const float alpha = alpha_of(ss_in);
-  const uint64_t pol = l2_policy(evict_first);
-  const uint32_t wbase = smem_u32(win);
-  auto blk_end = [&](int64_t b) {
-    const int64_t e = (b + 1) * LN_THREADS;
-    return (int)(e < nrows ? e : nrows);
-  };
-  int whi = 0;
-  if (use_win) {
-    const int h = blk_end(b0) + dg + XLEAD;
-    whi = h < xl ? h : xl;
-    for (int u = tid; u < XWIN; u += LN_THREADS) {
-      const int c = whi - XWIN + u;
-      if (c >= 0) win[c & (XWIN - 1)] = __ldg(x + c);
-    }
-  }
-  __syncthreads();
-  int sb = 0;
-  // row pointers of the first block (later blocks are prefetched one ahead)
-  int64_t a_n = 0, e_n = 0;
-  {
-    const int r = (int)(b0 * LN_THREADS) + tid;
-    if (r < blk_end(b0)) {
-      a_n = (int64_t)rp[r];
-      e_n = (int64_t)rp[r + 1];
-    }
-  }
-  for (int64_t blk = b0; blk < b1; ++blk) {
-    const int R0 = (int)(blk * LN_THREADS), R1 = blk_end(blk);
-    const int r = R0 + tid;
-    const int64_t a = a_n, e = e_n;
-    if (blk + 1 < b1) {
-      const int rn = R1 + tid;
-      a_n = e_n = 0;
-      if (rn < blk_end(blk + 1)) {
-        a_n = (int64_t)rp[rn];
-        e_n = (int64_t)rp[rn + 1];
-      }
-    }
-    // window advance for the next block: loads issued now, stored after this
-    // block's rows (into slots this block does not read)
-    int whi_next = whi, seg_lo = whi;
-    float segv = 0.f;
-    if (use_win && blk + 1 < b1) {
-      const int h = blk_end(blk + 1) + dg + XLEAD;
-      whi_next = h < xl ? h : xl;
-      seg_lo = whi_next - whi > XWIN ? whi_next - XWIN : whi;
-      if (seg_lo + tid < whi_next) segv = __ldg(x + seg_lo + tid);
-    }
-    const int vlo = whi_next - XWIN > 0 ? whi_next - XWIN : 0;
-    const uint32_t span = (use_win && whi > vlo) ? (uint32_t)(whi - vlo) : 0u;
-    const int L = (int)(e - a);
+  for (int64_t blk = blockIdx.x; blk < NB; blk += gridDim.x) {
+    const int64_t r = blk * LN_THREADS + tid;
     float res = 0.f;
-    if (L <= SHORT_MAX) {  // canonical W = 1: sequential, 4-entry aligned chunks
-      // Branch-free slots: every slot of a chunk holds a valid column of some
-      // row (or the zero tail padding), so its x read is always safe; slots
-      // outside [a, e) contribute an exact +0 (res starts at +0 and is never -0).
-      const int32_t* cp = col + (a & ~7ll);
-      const float* vp = val + (a & ~7ll);
-      const int lo = (int)(a & 7), hi = lo + L;
+    bool mine = false;
+    if (r < nrows) {
+      const int64_t a = (int64_t)rp[r], e = (int64_t)rp[r + 1];
+      const int L = (int)(e - a);
+      if (L <= SHORT_MAX) {  // longer rows: k_warp_rows / k_cta_rows / k_hub_*
+        mine = true;
+        // Every slot of a chunk holds a valid column of some row (or the zero
+        // tail padding), so its x read is always safe; slots outside [a, e)
+        // get x = 0, an exact +-0 product (res starts at +0, never -0).
+        const int32_t* cp = col + (a & ~7ll);
+        const float* vp = val + (a & ~7ll);
+        const int lo = (int)(a & 7), hi = lo + L;
 #pragma unroll 2
-      for (int k = 0; k < hi; k += 8) {
-        int cc[8];
-        float vv[8], xv[8];
-        ld_v8_stream(cp + k, pol, cc);
-        ld_v8_stream(vp + k, pol, vv);
+        for (int k = 0; k < hi; k += 8) {
+          int cc[8];
+          float vv[8];
+          ld_v8_stream(cp + k, cc);
+          ld_v8_stream(vp + k, vv);
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const bool inw = (uint32_t)(cc[i] - vlo) < span;
-          const float xs = lds_f32(wbase + (((uint32_t)cc[i] & (XWIN - 1)) << 2));
-          float xg = 0.f;
-          if (!inw) xg = __ldg(x + cc[i]);
-          xv[i] = inw ? xs : xg;
-        }
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const float p = __fmul_rn(vv[i], xv[i]);
-          res = __fadd_rn(res, (k + i >= lo && k + i < hi) ? p : 0.f);
+          for (int i = 0; i < 8; ++i) {
+            const float xv = __ldg(x + cc[i]);
+            res = __fadd_rn(res, __fmul_rn(vv[i], (k + i >= lo && k + i < hi) ? xv : 0.f));
+          }
         }
       }
     }
     double ssacc = 0.0;
-    if (r < R1 && L <= SHORT_MAX) {  // longer rows: k_warp_rows / k_cta_rows / k_hub_*
+    if (mine) {
       const float o = __fmul_rn(res, alpha);
       y[r] = o;
       if (SS) ssacc = (double)o * (double)o;
     }
-    if (use_win && blk + 1 < b1) {
-      if (seg_lo + tid < whi_next) win[(seg_lo + tid) & (XWIN - 1)] = segv;
-      for (int c = seg_lo + LN_THREADS + tid; c < whi_next; c += LN_THREADS)
-        win[c & (XWIN - 1)] = __ldg(x + c);
-    }
-    if (SS) {
+    if (SS) {  // fixed-order per-block sum of y^2 (independent of the grid)
       ssacc = warp_sum_d(ssacc);
-      if (lane == 0) wss[sb][warp] = ssacc;
+      if (lane == 0) wss[warp] = ssacc;
+      __syncthreads();
+      if (tid == 0) {
+        double t = 0.0;
+        for (int w = 0; w < LN_WARPS; ++w) t += wss[w];
+        blk_ss[blk] = t;
+      }
+      __syncthreads();
     }
-    __syncthreads();  // window advance visible; wss[sb] complete
-    if (SS && tid == 0) {
-      double t = 0.0;
-      for (int w = 0; w < LN_WARPS; ++w) t += wss[sb][w];
-      blk_ss[blk] = t;
-    }
-    sb ^= 1;
-    whi = whi_next;
   }
 }
 
 template <typename OT, bool SS>
 void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
-  static int occ = 0;
-  if (!occ) {
-    SPMV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_lane<OT, SS>, LN_THREADS, 0));
-    occ = std::max(occ, 1);
-  }
-  int lim = LN_CTAS_PER_SM;
-  if (const char* e = getenv("SPMV_LANE_CTAS")) lim = atoi(e);  // dev knob
-  const int per_sm = std::max(1, std::min(occ, lim));
+  int per_sm = LN_CTAS_PER_SM;
+  if (const char* e = getenv("SPMV_LANE_CTAS")) per_sm = std::max(1, atoi(e));  // dev knob
   const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
   const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
-  const int use_win = p->opts.smem_window ? 1 : 0;
   k_lane<OT, SS><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
-                                             p->nrows, p->y_offset, p->x_len, use_win, ss_in,
-                                             p->d_blk_ss, p->opts.evict_first);
+                                             p->nrows, ss_in, p->d_blk_ss);
 }
 
 template <typename OT>
