@@ -546,22 +546,36 @@ constexpr int LN_THREADS = 256;
 constexpr int LN_WARPS = LN_THREADS / 32;
 constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 
+template <int EF>
 __device__ __forceinline__ void ld_v8_stream(const int32_t* p, int (&r)[8]) {
-  asm("ld.global.nc.L1::no_allocate.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
-        "=r"(r[7])
-      : "l"(p));
+  if constexpr (EF)
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+          "=r"(r[7])
+        : "l"(p));
+  else
+    asm("ld.global.nc.L1::no_allocate.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+          "=r"(r[7])
+        : "l"(p));
 }
 
+template <int EF>
 __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
-  asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-      : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
-        "=f"(r[7])
-      : "l"(p));
+  if constexpr (EF)
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
+          "=f"(r[7])
+        : "l"(p));
+  else
+    asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
+          "=f"(r[7])
+        : "l"(p));
 }
 
-template <typename OT, bool SS>
-__global__ void __launch_bounds__(LN_THREADS)
+template <typename OT, bool SS, int EF, int MINB>
+__global__ void __launch_bounds__(LN_THREADS, MINB)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
            int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss) {
@@ -569,27 +583,43 @@ __global__ void __launch_bounds__(LN_THREADS)
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
   const float alpha = alpha_of(ss_in);
+  // row pointers are loaded one block iteration ahead
+  OT a_n = 0, e_n = 0;
+  {
+    const int64_t r = (int64_t)blockIdx.x * LN_THREADS + tid;
+    if (r < nrows) {
+      a_n = rp[r];
+      e_n = rp[r + 1];
+    }
+  }
   for (int64_t blk = blockIdx.x; blk < NB; blk += gridDim.x) {
     const int64_t r = blk * LN_THREADS + tid;
+    const OT a = a_n, e = e_n;
+    {
+      const int64_t rn = r + (int64_t)gridDim.x * LN_THREADS;
+      if (rn < nrows) {
+        a_n = rp[rn];
+        e_n = rp[rn + 1];
+      }
+    }
     float res = 0.f;
     bool mine = false;
     if (r < nrows) {
-      const int64_t a = (int64_t)rp[r], e = (int64_t)rp[r + 1];
       const int L = (int)(e - a);
       if (L <= SHORT_MAX) {  // longer rows: k_warp_rows / k_cta_rows / k_hub_*
         mine = true;
         // Every slot of a chunk holds a valid column of some row (or the zero
         // tail padding), so its x read is always safe; slots outside [a, e)
         // get x = 0, an exact +-0 product (res starts at +0, never -0).
-        const int32_t* cp = col + (a & ~7ll);
-        const float* vp = val + (a & ~7ll);
+        const int32_t* cp = col + (a & ~(OT)7);
+        const float* vp = val + (a & ~(OT)7);
         const int lo = (int)(a & 7), hi = lo + L;
 #pragma unroll 2
         for (int k = 0; k < hi; k += 8) {
           int cc[8];
           float vv[8];
-          ld_v8_stream(cp + k, cc);
-          ld_v8_stream(vp + k, vv);
+          ld_v8_stream<EF>(cp + k, cc);
+          ld_v8_stream<EF>(vp + k, vv);
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
             const float xv = __ldg(x + cc[i]);
@@ -618,15 +648,31 @@ __global__ void __launch_bounds__(LN_THREADS)
   }
 }
 
-template <typename OT, bool SS>
-void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
+template <typename OT, bool SS, int EF, int MINB>
+void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
   int per_sm = LN_CTAS_PER_SM;
   if (const char* e = getenv("SPMV_LANE_CTAS")) per_sm = std::max(1, atoi(e));  // dev knob
   const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
   const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
-  k_lane<OT, SS><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
-                                             p->nrows, ss_in, p->d_blk_ss);
+  k_lane<OT, SS, EF, MINB><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val,
+                                                       x, y, p->nrows, ss_in, p->d_blk_ss);
+}
+
+template <typename OT, bool SS>
+void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
+  int ef = p->opts.evict_first ? 1 : 0, minb = 1;
+  if (const char* e = getenv("SPMV_LANE_EF")) ef = atoi(e);      // dev knob
+  if (const char* e = getenv("SPMV_LANE_MINB")) minb = atoi(e);  // dev knob
+  if (ef) {
+    if (minb >= 8) launch_lane_t<OT, SS, 1, 8>(p, x, y, ss_in, s);
+    else if (minb >= 6) launch_lane_t<OT, SS, 1, 6>(p, x, y, ss_in, s);
+    else launch_lane_t<OT, SS, 1, 1>(p, x, y, ss_in, s);
+  } else {
+    if (minb >= 8) launch_lane_t<OT, SS, 0, 8>(p, x, y, ss_in, s);
+    else if (minb >= 6) launch_lane_t<OT, SS, 0, 6>(p, x, y, ss_in, s);
+    else launch_lane_t<OT, SS, 0, 1>(p, x, y, ss_in, s);
+  }
 }
 
 template <typename OT>
@@ -694,7 +740,9 @@ void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
   int maxwin = 0, maxpers = 0;
   cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, p->device);
   cudaDeviceGetAttribute(&maxpers, cudaDevAttrMaxPersistingL2CacheSize, p->device);
-  int64_t bytes = std::min<int64_t>(p->H * 4, (int64_t)maxwin);
+  int64_t want = p->H;
+  if (const char* e = getenv("SPMV_WIN_ALL")) if (atoi(e)) want = p->x_len;  // dev knob
+  int64_t bytes = std::min<int64_t>(want * 4, (int64_t)maxwin);
   bytes = std::min<int64_t>(bytes, (int64_t)maxpers);
   if (bytes <= 0) return;
   size_t cur = 0;
