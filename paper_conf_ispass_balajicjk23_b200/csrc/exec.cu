@@ -546,6 +546,24 @@ constexpr int LN_THREADS = 256;
 constexpr int LN_WARPS = LN_THREADS / 32;
 constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 
+// 256-bit streaming loads of one 8-entry chunk, not allocated in L1.
+// ef != 0 adds the L2::evict_first qualifier.  A chunk shared with a
+// neighbouring row (the first / last chunk of a row) is read twice, by two
+// lanes at different times; evicting it first would make the second read a
+// DRAM refetch (measured: 2.3x DRAM traffic on the 27-point stencil), so
+// EF mode 2 marks only a row's interior chunks evict_first.
+// x gather; GL = 1: L2 evict_last (x outlives the stream's lines in L2)
+template <int GL>
+__device__ __forceinline__ float ld_x(const float* p, uint64_t pol) {
+  if constexpr (GL) {
+    float r;
+    asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r) : "l"(p), "l"(pol));
+    return r;
+  } else {
+    return __ldg(p);
+  }
+}
+
 template <int EF>
 __device__ __forceinline__ void ld_v8_stream(const int32_t* p, int (&r)[8]) {
   if constexpr (EF)
@@ -574,8 +592,11 @@ __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
         : "l"(p));
 }
 
-template <typename OT, bool SS, int EF, int MINB>
-__global__ void __launch_bounds__(LN_THREADS, MINB)
+// minBlocksPerSM = 1 lets ptxas keep both chunks and all 16 gathers of a
+// 16-entry row in flight per lane (64 registers, 4 CTAs/SM); capping registers
+// for more CTAs measured 20-40 % slower
+template <typename OT, bool SS, int EF, int GL>
+__global__ void __launch_bounds__(LN_THREADS, 1)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
            int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss) {
@@ -583,6 +604,8 @@ __global__ void __launch_bounds__(LN_THREADS, MINB)
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
   const float alpha = alpha_of(ss_in);
+  uint64_t gpol = 0;
+  if (GL) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(gpol));
   // row pointers are loaded one block iteration ahead
   OT a_n = 0, e_n = 0;
   {
@@ -622,7 +645,7 @@ __global__ void __launch_bounds__(LN_THREADS, MINB)
           ld_v8_stream<EF>(vp + k, vv);
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
-            const float xv = __ldg(x + cc[i]);
+            const float xv = ld_x<GL>(x + cc[i], gpol);
             res = __fadd_rn(res, __fmul_rn(vv[i], (k + i >= lo && k + i < hi) ? xv : 0.f));
           }
         }
@@ -648,30 +671,31 @@ __global__ void __launch_bounds__(LN_THREADS, MINB)
   }
 }
 
-template <typename OT, bool SS, int EF, int MINB>
+template <typename OT, bool SS, int EF, int GL>
 void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
+  // grid-stride with ~8 CTAs per resident slot (measured better than one
+  // persistent wave on SBM, RMAT-26 and the stencil: r29, profiles/)
   int per_sm = LN_CTAS_PER_SM;
   if (const char* e = getenv("SPMV_LANE_CTAS")) per_sm = std::max(1, atoi(e));  // dev knob
   const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
   const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
-  k_lane<OT, SS, EF, MINB><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val,
+  k_lane<OT, SS, EF, GL><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val,
                                                        x, y, p->nrows, ss_in, p->d_blk_ss);
 }
 
 template <typename OT, bool SS>
 void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
-  int ef = p->opts.evict_first ? 1 : 0, minb = 1;
-  if (const char* e = getenv("SPMV_LANE_EF")) ef = atoi(e);      // dev knob
-  if (const char* e = getenv("SPMV_LANE_MINB")) minb = atoi(e);  // dev knob
-  if (ef) {
-    if (minb >= 8) launch_lane_t<OT, SS, 1, 8>(p, x, y, ss_in, s);
-    else if (minb >= 6) launch_lane_t<OT, SS, 1, 6>(p, x, y, ss_in, s);
-    else launch_lane_t<OT, SS, 1, 1>(p, x, y, ss_in, s);
+  int ef = p->opts.evict_first && p->stream_ef ? 1 : 0;
+  if (const char* e = getenv("SPMV_LANE_EF")) ef = atoi(e);  // dev knob: 0 / 1
+  int gl = 0;
+  if (const char* e = getenv("SPMV_LANE_GL")) gl = atoi(e);  // dev knob: x gathers evict_last
+  if (ef == 1) {
+    if (gl) launch_lane_t<OT, SS, 1, 1>(p, x, y, ss_in, s);
+    else launch_lane_t<OT, SS, 1, 0>(p, x, y, ss_in, s);
   } else {
-    if (minb >= 8) launch_lane_t<OT, SS, 0, 8>(p, x, y, ss_in, s);
-    else if (minb >= 6) launch_lane_t<OT, SS, 0, 6>(p, x, y, ss_in, s);
-    else launch_lane_t<OT, SS, 0, 1>(p, x, y, ss_in, s);
+    if (gl) launch_lane_t<OT, SS, 0, 1>(p, x, y, ss_in, s);
+    else launch_lane_t<OT, SS, 0, 0>(p, x, y, ss_in, s);
   }
 }
 
@@ -690,37 +714,55 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
     if (SS) launch_panel<OT, true>(p, x, y, ss_in, s);
     else launch_panel<OT, false>(p, x, y, ss_in, s);
   }
+  const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
+  // The row classes write disjoint rows of y and only read x: the warp-row
+  // kernel and the CTA/hub kernels run on two plan-owned streams concurrently
+  // with the short-row kernel (fork/join by events; CUDA-graph capturable).
+  cudaStream_t s1 = s, s2 = s;
+  const bool conc = p->conc && (nw > 0 || p->n_cta > 0 || p->n_chunks > 0);
+  if (conc) {
+    SPMV_CUDA(cudaEventRecord(p->ev_fork, s));
+    s1 = p->aux[0];
+    s2 = p->aux[1];
+    SPMV_CUDA(cudaStreamWaitEvent(s1, p->ev_fork, 0));
+    SPMV_CUDA(cudaStreamWaitEvent(s2, p->ev_fork, 0));
+  }
   {
-    const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
     const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
     double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
     if (nw) {
       const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
       if (SS)
-        k_warp_rows<OT, true><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
+        k_warp_rows<OT, true><<<g, 256, 0, s1>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
       else
-        k_warp_rows<OT, false><<<g, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
+        k_warp_rows<OT, false><<<g, 256, 0, s1>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
     }
   }
   if (p->n_cta) {
     if (SS)
-      k_cta_rows<OT, true><<<(unsigned)p->n_cta, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y,
-                                                             p->d_cta_rows, ss_in, p->d_cta_ss);
-    else
-      k_cta_rows<OT, false><<<(unsigned)p->n_cta, 256, 0, s>>>(rp, p->d_col, p->d_val, x, y,
+      k_cta_rows<OT, true><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, p->d_col, p->d_val, x, y,
                                                               p->d_cta_rows, ss_in, p->d_cta_ss);
+    else
+      k_cta_rows<OT, false><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, p->d_col, p->d_val, x, y,
+                                                               p->d_cta_rows, ss_in, p->d_cta_ss);
   }
   if (p->n_chunks) {
-    k_hub_chunk<OT><<<(unsigned)p->n_chunks, 256, 0, s>>>(rp, p->d_col, p->d_val, x,
-                                                          p->d_chunk_row, p->d_chunk_idx,
-                                                          p->d_chunk_part);
+    k_hub_chunk<OT><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, p->d_col, p->d_val, x,
+                                                           p->d_chunk_row, p->d_chunk_idx,
+                                                           p->d_chunk_part);
     const unsigned g = (unsigned)((p->n_hub + 127) / 128);
     if (SS)
-      k_hub_fix<true><<<g, 128, 0, s>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
-                                        ss_in, y, p->d_hub_ss);
+      k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
+                                         ss_in, y, p->d_hub_ss);
     else
-      k_hub_fix<false><<<g, 128, 0, s>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub,
-                                         p->d_chunk_part, ss_in, y, p->d_hub_ss);
+      k_hub_fix<false><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub,
+                                          p->d_chunk_part, ss_in, y, p->d_hub_ss);
+  }
+  if (conc) {
+    SPMV_CUDA(cudaEventRecord(p->ev_join[0], s1));
+    SPMV_CUDA(cudaEventRecord(p->ev_join[1], s2));
+    SPMV_CUDA(cudaStreamWaitEvent(s, p->ev_join[0], 0));
+    SPMV_CUDA(cudaStreamWaitEvent(s, p->ev_join[1], 0));
   }
   if (SS) {
     if (lane_mode)
@@ -734,9 +776,8 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   SPMV_LAUNCH_CHECK();
 }
 
-void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
-  if (!p->opts.l2_window || p->H <= 0 || s == nullptr) return;
-  if (p->win_ptr == (const void*)x && p->win_stream == s) return;
+void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
+  if (p->win_ptr == (const void*)x && p->win_stream[slot] == s) return;
   int maxwin = 0, maxpers = 0;
   cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, p->device);
   cudaDeviceGetAttribute(&maxpers, cudaDevAttrMaxPersistingL2CacheSize, p->device);
@@ -758,9 +799,42 @@ void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
     cudaGetLastError();
     return;
   }
-  p->win_ptr = x;
-  p->win_stream = s;
+  if (p->win_ptr != (const void*)x) {
+    p->win_stream[0] = p->win_stream[1] = p->win_stream[2] = nullptr;
+    p->win_ptr = x;
+  }
+  p->win_stream[slot] = s;
   p->l2_window_bytes = bytes;
+}
+
+void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
+  if (!p->opts.l2_window || p->H <= 0 || s == nullptr) return;
+  set_window_one(p, x, s, 0);
+  if (p->conc) {
+    set_window_one(p, x, p->aux[0], 1);
+    set_window_one(p, x, p->aux[1], 2);
+  }
+}
+
+// lazily create the plan's two auxiliary streams and events (on the plan's
+// device); concurrency is off if that fails or SPMV_CONCURRENT=0 (dev knob)
+void ensure_aux(spmv_plan_s* p) {
+  if (p->conc_init) return;
+  p->conc_init = true;
+  p->conc = false;
+  if (const char* e = getenv("SPMV_CONCURRENT")) if (!atoi(e)) return;
+  for (int i = 0; i < 2; ++i) {
+    if (cudaStreamCreateWithFlags(&p->aux[i], cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&p->ev_join[i], cudaEventDisableTiming) != cudaSuccess) {
+      cudaGetLastError();
+      return;
+    }
+  }
+  if (cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    return;
+  }
+  p->conc = true;
 }
 
 }  // namespace
@@ -775,6 +849,7 @@ void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double*
           cudaStream_t s) {
   if (!p->permuted) SPMV_FAIL(SPMV_ESTATE, "spmv_exec before spmv_permute");
   if (ss_in && ss_in == ss_out) SPMV_FAIL(SPMV_EINVAL, "sumsq_in and sumsq_out alias");
+  ensure_aux(p);
   set_window(p, x, s);
   if (p->off64) exec_typed<int64_t>(p, x, y, ss_in, ss_out, s);
   else exec_typed<int32_t>(p, x, y, ss_in, ss_out, s);

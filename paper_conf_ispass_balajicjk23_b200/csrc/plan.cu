@@ -226,6 +226,28 @@ __global__ void k_tile_desc(const OT* rp, const int32_t* tiles, int64_t K, TileD
   }
 }
 
+// short rows (1 <= L <= SHORT_MAX) and those whose first or last 8-entry
+// chunk is shared with a neighbouring row (start or end not a multiple of 8)
+template <typename OT>
+__global__ void k_chunk_share(const OT* rp, int64_t nrows, unsigned long long* cnt) {
+  unsigned long long sh = 0, all = 0;
+  GRID_STRIDE(r, nrows) {
+    const int64_t a = (int64_t)rp[r], e = (int64_t)rp[r + 1];
+    if (e - a >= 1 && e - a <= SHORT_MAX) {
+      ++all;
+      sh += ((a | e) & 7) != 0;
+    }
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    sh += __shfl_xor_sync(0xffffffffu, sh, o);
+    all += __shfl_xor_sync(0xffffffffu, all, o);
+  }
+  if ((threadIdx.x & 31) == 0 && all) {
+    atomicAdd(cnt, sh);
+    atomicAdd(cnt + 1, all);
+  }
+}
+
 // flags for a row-length predicate lo < L <= hi
 template <typename OT>
 __global__ void k_len_flag(const OT* rp, int64_t nrows, int64_t lo, int64_t hi, int last_only,
@@ -681,6 +703,21 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   if (p->K) k_tile_desc<OT><<<grid_for(p->K), TPB, 0, s>>>(rp, p->d_tiles, p->K, p->d_desc);
   SPMV_LAUNCH_CHECK();
 
+  // stream cache policy of the short-row kernel: L2
+  // evict_first only when no 8-entry chunk is read by two lanes (<= 1 % of the
+  // short rows share one), else a shared chunk evicted early is refetched
+  {
+    unsigned long long* dc = dalloc<unsigned long long>(2);
+    SPMV_CUDA(cudaMemsetAsync(dc, 0, 16, s));
+    if (nr) k_chunk_share<OT><<<grid_for(nr), TPB, 0, s>>>(rp, nr, dc);
+    SPMV_LAUNCH_CHECK();
+    unsigned long long hc[2] = {0, 0};
+    SPMV_CUDA(cudaMemcpyAsync(hc, dc, 16, cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA(cudaStreamSynchronize(s));
+    dfree(dc);
+    p->stream_ef = hc[0] * 100 <= hc[1];
+  }
+
   // row classes + sort buckets
   int32_t* f = dalloc<int32_t>(nr);
   int64_t* pos = dalloc<int64_t>(nr + 1);
@@ -870,6 +907,11 @@ void plan_free(spmv_plan_s* p) {
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
   dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_blk_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
   dfree(p->d_ss); dfree(p->d_u);
+  for (int i = 0; i < 2; ++i) {
+    if (p->aux[i]) { cudaStreamDestroy(p->aux[i]); p->aux[i] = nullptr; }
+    if (p->ev_join[i]) { cudaEventDestroy(p->ev_join[i]); p->ev_join[i] = nullptr; }
+  }
+  if (p->ev_fork) { cudaEventDestroy(p->ev_fork); p->ev_fork = nullptr; }
 }
 
 }  // namespace spmv

@@ -75,11 +75,18 @@ struct spmv_plan_s {
   int64_t* boff = nullptr; int64_t big_total = 0, big_max = 0;
   int32_t* longrows = nullptr; int64_t nlong = 0;  // L > STREAM_MAX
 
+  // exec concurrency: the row-class kernels other than the short-row kernel
+  // run on two plan-owned streams forked from / joined to the caller's stream
+  cudaStream_t aux[2] = {nullptr, nullptr};
+  cudaEvent_t ev_fork = nullptr, ev_join[2] = {nullptr, nullptr};
+  bool conc = false, conc_init = false;
+  bool stream_ef = false;  // k_lane streams col/val with L2::evict_first (plan decision)
+
   // state
   bool permuted = false;
   int64_t l2_window_bytes = 0;
   const void* win_ptr = nullptr;
-  cudaStream_t win_stream = nullptr;
+  cudaStream_t win_stream[3] = {nullptr, nullptr, nullptr};
 };
 
 namespace spmv {

@@ -19,6 +19,8 @@
 #include <omp.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <chrono>
 #include <cmath>
 #include <cstring>
@@ -261,6 +263,20 @@ uint64_t input_key(int64_t n, int64_t nnz, const int64_t* rp, const int32_t* col
 }
 }  // namespace
 
+static bool verbose() {
+  static int v = -1;
+  if (v < 0) v = getenv("SPMV_REORDER_VERBOSE") ? 1 : 0;
+  return v == 1;
+}
+
+static void phase(const char* what, std::chrono::steady_clock::time_point& t) {
+  auto now = std::chrono::steady_clock::now();
+  if (verbose())
+    fprintf(stderr, "[spmv_reorder] %-14s %8.3f s\n", what,
+            std::chrono::duration<double>(now - t).count());
+  t = now;
+}
+
 extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, const int32_t* col,
                                     int method, uint64_t seed, int32_t* perm_out,
                                     spmv_reorder_stats_t* st) {
@@ -288,6 +304,8 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
         spmv::set_error("spmv_reorder: column out of range");
         return SPMV_EINVAL;
       }
+    auto tp = std::chrono::steady_clock::now();
+    phase("validate", tp);
     spmv_reorder_stats_t S0;
     std::memset(&S0, 0, sizeof(S0));
     // skew: top ceil(0.1 N) row lengths / NZ
@@ -310,6 +328,7 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
       hub[v] = (__int128)colcnt[v] * n > (__int128)nnz;
       S0.n_hubs += hub[v];
     }
+    phase("skew+colcnt", tp);
 
     if (method == SPMV_ORDER_ORIGINAL) {
       for (int64_t i = 0; i < n; ++i) perm_out[i] = (int32_t)i;
@@ -328,10 +347,12 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
       if (!(g_cache.valid && g_cache.key == key && g_cache.n == n && g_cache.nnz == nnz)) {
         g_cache.valid = false;
         Sym S = symmetrize(n, rp, col);
+        phase("symmetrize", tp);
         auto td = std::chrono::steady_clock::now();
         g_cache.R = rabbit_detect(S);
         g_cache.seconds_detect =
             std::chrono::duration<double>(std::chrono::steady_clock::now() - td).count();
+        phase("detect+dfs", tp);
         Rabbit& R = g_cache.R;
         // community sizes
         {
@@ -379,6 +400,7 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
           }
           g_cache.insularity = total ? (double)intra / (double)total : 1.0;
         }
+        phase("stats", tp);
         g_cache.key = key;
         g_cache.n = n;
         g_cache.nnz = nnz;

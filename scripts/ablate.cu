@@ -20,16 +20,16 @@ __device__ __forceinline__ void ldv8f(const float* p, float (&r)[8]) {
 }
 
 // (a)/(c): lane per row, grid-stride over rows; mode 0 = no gathers, 1 = __ldg(x[c])
-template <int MODE>
-__global__ void __launch_bounds__(256) k_rows(const int32_t* __restrict__ rp,
+template <int MODE, typename OT>
+__global__ void __launch_bounds__(256) k_rows(const OT* __restrict__ rp,
                                               const int32_t* __restrict__ col,
                                               const float* __restrict__ val,
                                               const float* __restrict__ x, float* __restrict__ y,
                                               int n) {
   for (int r = blockIdx.x * blockDim.x + threadIdx.x; r < n; r += gridDim.x * blockDim.x) {
-    const int a = rp[r], e = rp[r + 1];
+    const long a = rp[r], e = rp[r + 1];
     float s = 0.f;
-    for (int k = a & ~7; k < e; k += 8) {
+    for (long k = a & ~7l; k < e; k += 8) {
       int c[8];
       float v[8];
       ldv8(col + k, c);
@@ -44,30 +44,30 @@ __global__ void __launch_bounds__(256) k_rows(const int32_t* __restrict__ rp,
   }
 }
 
-__device__ __forceinline__ void ldv8h(const int32_t* p, uint64_t pol, int (&r)[8]) {
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+__device__ __forceinline__ void ldv8h(const int32_t* p, uint64_t, int (&r)[8]) {
+  asm volatile("ld.global.nc.L1::no_allocate.L2::evict_first.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
                : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]),
                  "=r"(r[6]), "=r"(r[7])
-               : "l"(p), "l"(pol));
+               : "l"(p));
 }
-__device__ __forceinline__ void ldv8fh(const float* p, uint64_t pol, float (&r)[8]) {
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+__device__ __forceinline__ void ldv8fh(const float* p, uint64_t, float (&r)[8]) {
+  asm volatile("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
                : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]),
                  "=f"(r[6]), "=f"(r[7])
-               : "l"(p), "l"(pol));
+               : "l"(p));
 }
 
 // canonical variants: F bit0 = canonical fmul_rn/fadd_rn, bit1 = bitmask masking,
 // bit2 = evict_first hint on the stream, bit3 = contiguous 256-row panels per CTA
 // (persistent) instead of grid-stride
-template <int F>
-__global__ void __launch_bounds__(256) k_rows2(const int32_t* __restrict__ rp,
+template <int F, typename OT>
+__global__ void __launch_bounds__(256) k_rows2(const OT* __restrict__ rp,
                                                const int32_t* __restrict__ col,
                                                const float* __restrict__ val,
                                                const float* __restrict__ x, float* __restrict__ y,
                                                int n) {
   uint64_t pol = 0;
-  if (F & 4) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+
   int r0, r1, step;
   if (F & 8) {
     const long NB = (n + 255) / 256;
@@ -81,12 +81,12 @@ __global__ void __launch_bounds__(256) k_rows2(const int32_t* __restrict__ rp,
     step = gridDim.x * blockDim.x;
   }
   for (int r = r0; r < r1; r += step) {
-    const int a = rp[r], e = rp[r + 1];
+    const long a = rp[r], e = rp[r + 1];
     float s = 0.f;
-    const int lo = a & 7, hi = lo + (e - a);
+    const int lo = a & 7, hi = lo + (int)(e - a);
     const uint64_t live = (((1ull << hi) - 1ull) >> lo) << lo;
-    const int32_t* cp = col + (a & ~7);
-    const float* vp = val + (a & ~7);
+    const int32_t* cp = col + (a & ~7l);
+    const float* vp = val + (a & ~7l);
     for (int k = 0; k < hi; k += 8) {
       int c[8];
       float v[8];
@@ -95,7 +95,7 @@ __global__ void __launch_bounds__(256) k_rows2(const int32_t* __restrict__ rp,
       const uint32_t mk = (uint32_t)(live >> k);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        float xv = __ldg(x + c[i]);
+        float xv = (F & 16) ? __int_as_float(c[i]) : __ldg(x + c[i]);
         bool ok = (F & 2) ? ((mk >> i) & 1u) : (k + i >= lo && k + i < hi);
         if (F & 1) s = __fadd_rn(s, __fmul_rn(v[i], ok ? xv : 0.f));
         else s += ok ? v[i] * xv : 0.f;
@@ -122,15 +122,21 @@ __global__ void __launch_bounds__(256) k_flat(const int32_t* __restrict__ col,
   y[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
 
-extern "C" int ablate(int which, const int32_t* rp, const int32_t* col, const float* val,
-                      const float* x, float* y, int n, long nnz, int grid, cudaStream_t s) {
-  if (which == 0) k_rows<0><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
-  else if (which == 1) k_rows<1><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
+template <typename OT>
+int ablate_t(int which, const OT* rp, const int32_t* col, const float* val, const float* x, float* y,
+             int n, long nnz, int grid, cudaStream_t s) {
+  if (which == 0) k_rows<0, OT><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
+  else if (which == 1) k_rows<1, OT><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
   else if (which == 2) k_flat<<<grid, 256, 0, s>>>(col, val, y, nnz);
-  else if (which == 10) k_rows2<1><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
-  else if (which == 11) k_rows2<3><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
-  else if (which == 12) k_rows2<7><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
-  else if (which == 13) k_rows2<15><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
-  else if (which == 14) k_rows2<11><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
+  else if (which == 10) k_rows2<1, OT><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
+  else if (which == 12) k_rows2<5, OT><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
+  else if (which == 13) k_rows2<13, OT><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
+  else if (which == 20) k_rows2<16 + 5, OT><<<grid, 256, 0, s>>>(rp, col, val, x, y, n);
   return (int)cudaGetLastError();
+}
+
+extern "C" int ablate(int which, const void* rp, int rp64, const int32_t* col, const float* val,
+                      const float* x, float* y, int n, long nnz, int grid, cudaStream_t s) {
+  if (rp64) return ablate_t(which, (const long*)rp, col, val, x, y, n, nnz, grid, s);
+  return ablate_t(which, (const int*)rp, col, val, x, y, n, nnz, grid, s);
 }

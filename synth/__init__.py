@@ -160,7 +160,8 @@ class Workload:
     name: str
     A: Csr
     x: np.ndarray
-    planted: np.ndarray | None = None   # SBM ground-truth order (reference only)
+    planted: np.ndarray | None = None   # ground-truth order (SBM communities, stencil
+                                        # grid), perm[old] = new; reference only
 
 
 def config(k: int, small: bool = False) -> Workload:
@@ -184,7 +185,9 @@ def config(k: int, small: bool = False) -> Workload:
     if k == 4:
         nx = 24 if small else 464
         A = stencil27(nx, False, True, ss, VAL_SYM, sv)
-        return Workload(f"stencil27_{nx}", A, vector(A.n, sx))
+        planted = np.empty(A.n, np.int64)   # lexicographic grid order
+        planted[scramble_table(A.n, ss)] = np.arange(A.n)
+        return Workload(f"stencil27_{nx}", A, vector(A.n, sx), planted)
     if k == 5:
         sc = 14 if small else 28
         A = rmat(sc, 16, se, scramble=True, seed_scr=ss, valmode=VAL_POS, seed_v=sv)

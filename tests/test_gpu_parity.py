@@ -262,35 +262,60 @@ def test_iterate_matches_oracle_recurrence(dev):
     P.close()
 
 
-def test_bench_config_full_size(dev):
-    """BASELINE config 2 (SBM 4M/64M) at full size in the launch configuration
-    bench.py times: every row against the compensated C oracle, sampled rows
-    against the exact fsum oracle."""
+def _full_size_check(dev, cfg, ordering, nsample=2000):
+    """BASELINE config `cfg` at full size, in the launch configuration bench.py
+    times: sampled rows' integer structure against the oracle's own
+    relabelling, sampled y against the exact fsum oracle, every row against
+    the compensated C oracle on A itself, relabelled (y_B = P (A x))."""
     from paper_conf_ispass_balajicjk23_b200 import spmv
-    w = synth.config(2)
+    w = synth.config(cfg)
     A = w.A
-    perm, _ = spmv.reorder(A.row_ptr, A.col, "rabbitpp")
-    P = mk_plan(A, perm, dev)
+    if ordering == "original":
+        perm = np.arange(A.n, dtype=np.int32)
+    else:
+        perm, _ = spmv.reorder(A.row_ptr, A.col, ordering)
+    rp_dtype = torch.int32 if A.nnz < 2**31 else torch.int64
+    P = mk_plan(A, perm, dev, rp_dtype=rp_dtype)
     xB = P.permute_vec(torch.from_numpy(w.x).to(dev))
     y = P.exec(xB).cpu().numpy()
     rp, c, v = (t.cpu().numpy() for t in P.export_csr())
-    # integer structure on sampled rows vs the oracle's own relabelling
     inv = permute.inverse(perm)
-    rng = np.random.default_rng(0)
-    rows = np.sort(rng.choice(A.n, 2000, replace=False))
-    for r, (cc, vv) in zip(rows, permute.permute_rows(A.row_ptr, A.col, A.val, perm, inv, rows)):
+    rng = np.random.default_rng(cfg)
+    rows = np.sort(rng.choice(A.n, min(nsample, A.n), replace=False))
+    # the longest rows too (hub / CTA classes)
+    L = np.diff(rp)
+    rows = np.union1d(rows, np.argsort(L)[-20:])
+    oracle_rows = permute.permute_rows(A.row_ptr, A.col, A.val, perm, inv, rows)
+    for r, (cc, vv) in zip(rows, oracle_rows):
         assert np.array_equal(c[rp[r]:rp[r + 1]], cc)
         assert np.array_equal(v[rp[r]:rp[r + 1]].view(np.int32), vv.view(np.int32))
     xBh = permute.permute_vec(w.x, perm)
-    oracle_rows = permute.permute_rows(A.row_ptr, A.col, A.val, perm, inv, rows)
     ys = np.array([ospmv.spmv_rows([0, len(cc)], cc, vv, xBh, [0])[0] for cc, vv in oracle_rows])
     ab = np.array([np.abs(vv.astype(np.float64) * xBh[cc].astype(np.float64)).sum()
                    for cc, vv in oracle_rows])
     _check_y(y[rows], ys, ab, "sampled")
-    # every row: compensated C oracle on A itself, relabelled (y_B = P (A x))
+    assert np.all(y[L == 0] == 0)
     yA, absA = cref.spmv_neumaier(A.row_ptr, A.col, A.val, w.x)
     _check_y(y, permute.permute_vec(yA, perm), permute.permute_vec(absA, perm), "all rows")
     P.close()
+
+
+def test_bench_config_full_size(dev):
+    """BASELINE configs[1] (SBM 4M/64M, RABBIT++): the bench.py workload."""
+    _full_size_check(dev, 2, "rabbitpp")
+
+
+def test_rmat16_full_size(dev):
+    """BASELINE configs[0] (RMAT scale 16) at full size, RABBIT++ order: every
+    row against the exact fsum oracle as well."""
+    _full_size_check(dev, 1, "rabbitpp", nsample=65536)
+
+
+def test_rmat26_full_size(dev):
+    """BASELINE configs[2] (RMAT scale 26, 67M rows, 1.06 B nnz, x = 268 MB >
+    L2) at full size in its generated (ORIGINAL) order: hub rows (merge-path
+    chunks + fp64 fixup), CTA rows, MID rows and lane rows at scale."""
+    _full_size_check(dev, 3, "original")
 
 
 @pytest.mark.parametrize("name,make", CASES)
@@ -313,3 +338,35 @@ def test_smem_window_and_l2_options_bitwise(dev, name, make):
         P.close()
     for y in ys[1:]:
         assert np.array_equal(y.view(np.int32), ys[0].view(np.int32))
+
+
+def test_exec_graph_capture_and_concurrency(dev):
+    """exec forks the row-class kernels onto the plan's streams and joins them
+    back: eager, CUDA-graph-captured and serial (SPMV_CONCURRENT=0) runs agree
+    bitwise on a matrix with every row class."""
+    import os
+    A = long_rows_matrix(3)
+    perm = rabbit.random_perm(A.n, 9)
+    x = torch.from_numpy(synth.vector(A.n, 4)).to(dev)
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        P = mk_plan(A, perm, dev)
+        xB = P.permute_vec(x)
+        y0 = P.exec(xB)
+        y1 = torch.full_like(y0, float("nan"))
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            P.exec(xB, y1)
+        g.replay()
+        torch.cuda.synchronize()
+    assert torch.equal(y0.view(torch.int32), y1.view(torch.int32))
+    P.close()
+    os.environ["SPMV_CONCURRENT"] = "0"
+    try:
+        P = mk_plan(A, perm, dev)
+        y2 = P.exec(P.permute_vec(x))
+        torch.cuda.synchronize()
+    finally:
+        del os.environ["SPMV_CONCURRENT"]
+    assert torch.equal(y0.view(torch.int32), y2.view(torch.int32))
+    P.close()
