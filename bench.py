@@ -190,8 +190,7 @@ def run_gpu(args):
             xB = P.pad_vec(xB, to_padded=True)
         ideal = 2 * A.n * 4 + (A.n + 1) * info["offset_bytes"] + 2 * A.nnz * 4
         ideal_p96 = 2 * A.n * 4 + (A.n + 1 + 2 * A.nnz) * 4
-        launches = (1 if info["n_tiles"] else 0) + (1 if info["n_cta_rows"] else 0) + \
-            (2 if info["n_hub_chunks"] else 0)
+        launches = info["exec_launches"]
         is_main = ordering == main
         K = args.steps if is_main else max(10, args.steps // 4)
         if world == 1:

@@ -190,6 +190,7 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->permuted = p->permuted ? 1 : 0;
   info->l2_window_bytes = (int32_t)p->l2_window_bytes;
   info->stream_evict_first = (p->opts.evict_first && p->stream_ef) ? 1 : 0;
+  info->exec_launches = spmv::exec_launches(p, false);
   API_END
 }
 
