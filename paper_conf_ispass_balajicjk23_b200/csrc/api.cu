@@ -135,6 +135,14 @@ spmv_status spmv_exec(spmv_plan_t p, const float* x_B, float* y_B, void* stream)
   API_END
 }
 
+spmv_status spmv_exec_spmm4(spmv_plan_t p, const float* X_B, float* Y_B, void* stream) {
+  API_BEGIN
+  if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_spmm4: NULL plan");
+  if (p->nrows && (!X_B || !Y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_spmm4: NULL matrix");
+  spmv::exec_spmm4(p, X_B, Y_B, S(stream));
+  API_END
+}
+
 spmv_status spmv_exec_scaled(spmv_plan_t p, const float* x_B, float* y_B,
                              const double* sumsq_in, double* sumsq_out, void* stream) {
   API_BEGIN
@@ -191,6 +199,7 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->l2_window_bytes = (int32_t)p->l2_window_bytes;
   info->stream_evict_first = (p->opts.evict_first && p->stream_ef) ? 1 : 0;
   info->exec_launches = spmv::exec_launches(p, false);
+  info->spmm4_launches = spmv::spmm4_launches(p);
   API_END
 }
 

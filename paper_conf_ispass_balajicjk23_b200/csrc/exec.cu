@@ -783,6 +783,7 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   cudaDeviceGetAttribute(&maxpers, cudaDevAttrMaxPersistingL2CacheSize, p->device);
   int64_t want = p->H;
   if (const char* e = getenv("SPMV_WIN_ALL")) if (atoi(e)) want = p->x_len;  // dev knob
+  if (const char* e = getenv("SPMV_WIN_COLS")) want = std::min<int64_t>(p->x_len, atoll(e));  // dev knob
   int64_t bytes = std::min<int64_t>(want * 4, (int64_t)maxwin);
   bytes = std::min<int64_t>(bytes, (int64_t)maxpers);
   if (bytes <= 0) return;
@@ -822,6 +823,10 @@ void ensure_aux(spmv_plan_s* p) {
   if (p->conc_init) return;
   p->conc_init = true;
   p->conc = false;
+  if (const char* e = getenv("SPMV_L2_FETCH")) {  // dev knob: L2 miss fetch granularity (B)
+    cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)atoi(e));
+    cudaGetLastError();
+  }
   if (const char* e = getenv("SPMV_CONCURRENT")) if (!atoi(e)) return;
   for (int i = 0; i < 2; ++i) {
     if (cudaStreamCreateWithFlags(&p->aux[i], cudaStreamNonBlocking) != cudaSuccess ||
@@ -838,6 +843,8 @@ void ensure_aux(spmv_plan_s* p) {
 }
 
 }  // namespace
+
+void exec_streams(spmv_plan_s* p) { ensure_aux(p); }
 
 int exec_launches(const spmv_plan_s* p, bool ss) {
   const bool lane_mode = p->opts.variant != 1;

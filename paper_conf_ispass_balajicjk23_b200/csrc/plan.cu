@@ -904,6 +904,7 @@ void plan_free(spmv_plan_s* p) {
   if (p->d_rp) { cudaFree(p->d_rp); p->d_rp = nullptr; }
   dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows); dfree(p->d_desc);
   dfree(p->d_warp_rows); dfree(p->d_warp_ss); dfree(p->d_mid_rows); dfree(p->d_mid_ss);
+  dfree(p->d_chunk_part4);
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
   dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_blk_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
   dfree(p->d_ss); dfree(p->d_u);

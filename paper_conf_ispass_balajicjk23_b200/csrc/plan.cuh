@@ -58,6 +58,7 @@ struct spmv_plan_s {
 
   // exec scratch
   double* d_chunk_part = nullptr;  // [n_chunks]
+  double* d_chunk_part4 = nullptr; // [4 n_chunks] spmv_exec_spmm4 (allocated on first use)
   double* d_tile_ss = nullptr;     // [K]
   double* d_blk_ss = nullptr;      // [ceil(nrows/64)] per-block sumsq (lane variant)
   double* d_warp_ss = nullptr;     // [n_warp]
@@ -99,5 +100,7 @@ void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double*
           cudaStream_t s);
 void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s);
 int exec_launches(const spmv_plan_s* p, bool ss);
+void exec_spmm4(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s);
+int spmm4_launches(const spmv_plan_s* p);
 void scale_vec(const float* u, float* x, int64_t n, const double* ss, cudaStream_t s);
 }  // namespace spmv

@@ -50,7 +50,7 @@ class _Info(ctypes.Structure):
         "n_tiles", "n_warp_rows", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "n_mid_rows",
         "hot_prefix", "ideal_bytes")] + \
         [(n, ctypes.c_int32) for n in ("offset_bytes", "world", "rank", "permuted",
-                                       "l2_window_bytes", "stream_evict_first", "exec_launches", "r1")]
+                                       "l2_window_bytes", "stream_evict_first", "exec_launches", "spmm4_launches")]
 
 
 class _Stats(ctypes.Structure):
@@ -82,6 +82,7 @@ def lib() -> ctypes.CDLL:
             "spmv_pad_vec": (i32, [vp, vp, vp, i32, vp]),
             "spmv_exec": (i32, [vp, vp, vp, vp]),
             "spmv_exec_scaled": (i32, [vp, vp, vp, dp, dp, vp]),
+            "spmv_exec_spmm4": (i32, [vp, vp, vp, vp]),
             "spmv_iterate": (i32, [vp, vp, i32, ctypes.POINTER(ctypes.c_double), vp]),
             "spmv_scale_vec": (i32, [vp, vp, i64, dp, vp]),
             "spmv_plan_info": (i32, [vp, ctypes.POINTER(_Info)]),
@@ -199,6 +200,16 @@ class Plan:
             y = torch.empty(info["row_end"] - info["row_begin"], dtype=torch.float32, device=x.device)
         _check(lib().spmv_exec(self._h, _ptr(x), _ptr(y), _stream_ptr(stream)))
         return y
+
+    def exec_spmm4(self, X, Y=None, stream=None):
+        """Y_B = B X_B for X_B of shape (x_len, 4), row-major fp32 (SpMM-CSR-4)."""
+        import torch
+        if Y is None:
+            info = self.info()
+            Y = torch.empty((info["row_end"] - info["row_begin"], 4), dtype=torch.float32,
+                            device=X.device)
+        _check(lib().spmv_exec_spmm4(self._h, _ptr(X), _ptr(Y), _stream_ptr(stream)))
+        return Y
 
     def exec_scaled(self, x, y, sumsq_in=None, sumsq_out=None, stream=None):
         _check(lib().spmv_exec_scaled(self._h, _ptr(x), _ptr(y), _ptr(sumsq_in), _ptr(sumsq_out),

@@ -102,3 +102,36 @@ def test_compulsory_traffic_pins():
         assert metrics.ideal_bytes(c["n"], c["nnz"], c["w_off"]) == c["bytes"]
     ai = GOLD["arithmetic_intensity_upper_bound"]
     assert ai["flops_per_nz"] / ai["bytes_per_nz"] == ai["ai"]
+
+
+# ---- SpMM-CSR-4 (Table IV) -------------------------------
+@pytest.mark.parametrize("seed", range(4))
+def test_spmm_vs_dense_bruteforce_and_scipy(seed):
+    n = 41
+    rp, col, val, _ = rand_csr(n, 5, seed)
+    X = np.random.default_rng(100 + seed).uniform(-1, 1, (n, 4)).astype(np.float32)
+    Y = spmv.spmm(rp, col, val, X).astype(np.float64)
+    D = spmv.dense(n, rp, col, val)
+    scale = spmv.abs_rowsum_mat(rp, col, val, X)
+    # dense brute force in fp64, then the one fp32 rounding: within 1 ulp-ish of fp32
+    assert np.all(np.abs(Y - D @ X.astype(np.float64)) <= 2 ** -23 * scale + 1e-300)
+    S = sp.csr_matrix((val.astype(np.float64), col, rp), shape=(n, n))
+    assert np.all(np.abs(Y - S @ X.astype(np.float64)) <= 2 ** -23 * scale + 1e-300)
+
+
+def test_spmm_exact_cancellation_and_empty_rows():
+    # row 0: 1e8*1 + 1*1 - 1e8*1 = 1 exactly in column 0; column 1 uses x = 0
+    rp = np.array([0, 3, 3, 4], np.int64)
+    col = np.array([0, 1, 2, 0], np.int32)
+    val = np.array([1e8, 1.0, -1e8, 2.0], np.float32)
+    X = np.array([[1, 0, 0.5, -1], [1, 0, 0.5, -1], [1, 0, 0.5, -1]], np.float32)
+    Y = spmv.spmm(rp, col, val, X)
+    assert Y[0, 0] == 1.0 and Y[0, 1] == 0.0 and Y[0, 2] == 0.5 and Y[0, 3] == -1.0
+    assert np.all(Y[1] == 0) and np.array_equal(Y[2], 2 * X[0])
+
+
+def test_spmm_rows_sample_agrees():
+    rp, col, val, _ = rand_csr(60, 6, 9)
+    X = np.random.default_rng(3).uniform(-1, 1, (60, 4)).astype(np.float32)
+    rows = [0, 7, 59, 31]
+    assert np.array_equal(spmv.spmm_rows(rp, col, val, X, rows), spmv.spmm(rp, col, val, X)[rows])
