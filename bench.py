@@ -277,8 +277,10 @@ def run_gpu(args):
                "H": info["hot_prefix"], "tiles": info["n_tiles"], "cta_rows": info["n_cta_rows"],
                "hub_rows": info["n_hub_rows"], "l2_window_bytes": P.info()["l2_window_bytes"],
                "stream_evict_first": info["stream_evict_first"]}
-        if world == 1 and not args.no_spmm4:
-            res["spmm4"] = spmm4_measure(P, A, info, K, flush_l2, stream, dev, hbm)
+        if world == 1 and not args.no_side:
+            # the paper's Table IV kernels on the same reordered matrix
+            res["spmm4"] = side_measure("spmm4", P, A, info, K, flush_l2, stream, dev, hbm)
+            res["coo"] = side_measure("coo", P, A, info, K, flush_l2, stream, dev, hbm)
         tr = ncu_traffic(w.name, ordering)
         if tr:
             res["dram_over_ideal_ncu"] = tr.get("dram_bytes", 0) / ideal
@@ -339,29 +341,44 @@ def run_gpu(args):
         dist.destroy_process_group()
 
 
-def spmm4_measure(P, A, info, K, flush_l2, stream, dev, hbm):
-    """SpMM-CSR-4 (Table IV) on the same plan, cold L2 like
-    the SpMV steps; ideal = 8 NZ + (N+1) w_off + 16 N (X) + 16 N (Y)."""
+def side_measure(kind, P, A, info, K, flush_l2, stream, dev, hbm):
+    """Table IV kernels on the same plan, cold L2 like the
+    SpMV steps, ideal traffic "updated according to the kernel":
+      spmm4: 8 NZ + (N+1) w_off + 16 N (X) + 16 N (Y)
+      coo:   12 NZ + 4 N (x) + 4 N (y)"""
     import torch
-    X = torch.empty((A.n, 4), dtype=torch.float32, device=dev).uniform_(-1, 1)
-    Y = torch.empty_like(X)
+    if kind == "spmm4":
+        X = torch.empty((A.n, 4), dtype=torch.float32, device=dev).uniform_(-1, 1)
+        Y = torch.empty_like(X)
+        ideal = 32 * A.n + (A.n + 1) * info["offset_bytes"] + 8 * A.nnz
+        flops = 8 * A.nnz
+
+        def run():
+            P.exec_spmm4(X, Y)
+    else:
+        X = torch.empty(A.n, dtype=torch.float32, device=dev).uniform_(-1, 1)
+        Y = torch.empty_like(X)
+        ideal = 8 * A.n + 12 * A.nnz
+        flops = 2 * A.nnz
+
+        def run():
+            P.exec_coo(X, Y)
     for _ in range(3):
         flush_l2()
-        P.exec_spmm4(X, Y)
+        run()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(K)]
     torch.cuda.synchronize()
     for i in range(K):
         flush_l2()
         ev[i][0].record(stream)
-        P.exec_spmm4(X, Y)
+        run()
         ev[i][1].record(stream)
     torch.cuda.synchronize()
     ms = sum(a.elapsed_time(b) for a, b in ev) / K
-    ideal = 32 * A.n + (A.n + 1) * info["offset_bytes"] + 8 * A.nnz
     gbs = ideal / (ms * 1e-3) / 1e9
-    return {"ms": ms, "ideal_bytes": ideal, "gbs_ideal_over_t": gbs, "runtime_over_ideal": hbm / gbs,
-            "gflops": 8 * A.nnz / (ms * 1e-3) / 1e9, "launches": info["spmm4_launches"]}
+    return {"ms": round(ms, 5), "ideal_bytes": ideal, "gbs_ideal_over_t": round(gbs, 2),
+            "runtime_over_ideal": round(hbm / gbs, 4), "gflops": round(flops / (ms * 1e-3) / 1e9, 2)}
 
 
 def e2e_measure(P, A, x_host, args, dev, ideal):
@@ -503,7 +520,8 @@ def main():
                     help="comma list; the last one is the headline line")
     ap.add_argument("--seed", type=int, default=20230423)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-spmm4", action="store_true", help="skip the SpMM-CSR-4 side measurement")
+    ap.add_argument("--no-side", action="store_true",
+                    help="skip the Table IV side measurements (SpMM-CSR-4, SpMV-COO)")
     ap.add_argument("--perm-cache", default=None, help="dev only: memoise reorder results here")
     ap.add_argument("--variant", type=int, default=0, help="short-row kernel: 0 lane, 1 panel")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],

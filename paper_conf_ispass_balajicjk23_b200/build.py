@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libspmv.so")
-SOURCES = ["api.cu", "plan.cu", "exec.cu", "spmm.cu", "reorder.cpp"]
+SOURCES = ["api.cu", "plan.cu", "exec.cu", "spmm.cu", "coo.cu", "reorder.cpp"]
 HEADERS = ["common.cuh", "plan.cuh"]
 
 

@@ -143,6 +143,15 @@ spmv_status spmv_exec_spmm4(spmv_plan_t p, const float* X_B, float* Y_B, void* s
   API_END
 }
 
+spmv_status spmv_exec_coo(spmv_plan_t p, const float* x_B, float* y_B, void* stream) {
+  API_BEGIN
+  if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_coo: NULL plan");
+  if (p->nrows && (!x_B || !y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_coo: NULL vector");
+  use_device(p);
+  spmv::exec_coo(p, x_B, y_B, S(stream));
+  API_END
+}
+
 spmv_status spmv_exec_scaled(spmv_plan_t p, const float* x_B, float* y_B,
                              const double* sumsq_in, double* sumsq_out, void* stream) {
   API_BEGIN
@@ -269,6 +278,15 @@ spmv_status spmv_export_inverse(spmv_plan_t p, int32_t* inv, void* stream) {
   use_device(p);
   if (p->n)
     SPMV_CUDA(cudaMemcpyAsync(inv, p->d_inv, 4 * p->n, cudaMemcpyDeviceToDevice, S(stream)));
+  API_END
+}
+
+spmv_status spmv_export_coo_rows(spmv_plan_t p, int32_t* rows, void* stream) {
+  API_BEGIN
+  if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_export_coo_rows: NULL plan");
+  if (!p->permuted) SPMV_FAIL(SPMV_ESTATE, "spmv_export_coo_rows before spmv_permute");
+  use_device(p);
+  spmv::export_coo_rows(p, rows, S(stream));
   API_END
 }
 

@@ -898,6 +898,7 @@ void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStr
 }
 
 void plan_free(spmv_plan_s* p) {
+  coo_free(p);
   dfree(p->s1); dfree(p->s2); dfree(p->s3); dfree(p->big); dfree(p->boff);
   dfree(p->longrows);
   dfree(p->d_perm); dfree(p->d_inv);

@@ -59,6 +59,14 @@ struct spmv_plan_s {
   // exec scratch
   double* d_chunk_part = nullptr;  // [n_chunks]
   double* d_chunk_part4 = nullptr; // [4 n_chunks] spmv_exec_spmm4 (allocated on first use)
+
+  // COO form of B (spmv_exec_coo; built on first use): row index per entry and
+  // per-tile pieces of rows that cross a 2048-entry tile boundary
+  int64_t coo_tiles = 0;
+  int32_t* d_coo_row = nullptr;    // [nnz_local + 8]
+  int32_t* d_coo_trow = nullptr;   // [2 coo_tiles] first / last row of each tile
+  double* d_coo_tpart = nullptr;   // [2 coo_tiles] fp64 pieces (first / last row)
+  uint8_t* d_coo_tflag = nullptr;  // [coo_tiles]
   double* d_tile_ss = nullptr;     // [K]
   double* d_blk_ss = nullptr;      // [ceil(nrows/64)] per-block sumsq (lane variant)
   double* d_warp_ss = nullptr;     // [n_warp]
@@ -102,5 +110,8 @@ void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s
 int exec_launches(const spmv_plan_s* p, bool ss);
 void exec_spmm4(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s);
 int spmm4_launches(const spmv_plan_s* p);
+void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s);
+void export_coo_rows(spmv_plan_s* p, int32_t* rows, cudaStream_t s);
+void coo_free(spmv_plan_s* p);
 void scale_vec(const float* u, float* x, int64_t n, const double* ss, cudaStream_t s);
 }  // namespace spmv

@@ -83,6 +83,8 @@ def lib() -> ctypes.CDLL:
             "spmv_exec": (i32, [vp, vp, vp, vp]),
             "spmv_exec_scaled": (i32, [vp, vp, vp, dp, dp, vp]),
             "spmv_exec_spmm4": (i32, [vp, vp, vp, vp]),
+            "spmv_exec_coo": (i32, [vp, vp, vp, vp]),
+            "spmv_export_coo_rows": (i32, [vp, vp, vp]),
             "spmv_iterate": (i32, [vp, vp, i32, ctypes.POINTER(ctypes.c_double), vp]),
             "spmv_scale_vec": (i32, [vp, vp, i64, dp, vp]),
             "spmv_plan_info": (i32, [vp, ctypes.POINTER(_Info)]),
@@ -200,6 +202,22 @@ class Plan:
             y = torch.empty(info["row_end"] - info["row_begin"], dtype=torch.float32, device=x.device)
         _check(lib().spmv_exec(self._h, _ptr(x), _ptr(y), _stream_ptr(stream)))
         return y
+
+    def exec_coo(self, x, y=None, stream=None):
+        """y_B = B x_B reading B as COO triplets (SpMV-COO)."""
+        import torch
+        if y is None:
+            info = self.info()
+            y = torch.empty(info["row_end"] - info["row_begin"], dtype=torch.float32, device=x.device)
+        _check(lib().spmv_exec_coo(self._h, _ptr(x), _ptr(y), _stream_ptr(stream)))
+        return y
+
+    def export_coo_rows(self):
+        import torch
+        info = self.info()
+        rows = torch.empty(info["nnz_local"], dtype=torch.int32, device=self.device)
+        _check(lib().spmv_export_coo_rows(self._h, _ptr(rows), _stream_ptr(None)))
+        return rows
 
     def exec_spmm4(self, X, Y=None, stream=None):
         """Y_B = B X_B for X_B of shape (x_len, 4), row-major fp32 (SpMM-CSR-4)."""

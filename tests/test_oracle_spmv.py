@@ -135,3 +135,29 @@ def test_spmm_rows_sample_agrees():
     X = np.random.default_rng(3).uniform(-1, 1, (60, 4)).astype(np.float32)
     rows = [0, 7, 59, 31]
     assert np.array_equal(spmv.spmm_rows(rp, col, val, X, rows), spmv.spmm(rp, col, val, X)[rows])
+
+
+# ---- SpMV-COO (Table IV) ---------------------------------
+@pytest.mark.parametrize("seed", range(4))
+def test_coo_rows_equal_scipy_and_spmv_coo_vs_dense(seed):
+    n = 53
+    rp, col, val, x = rand_csr(n, 4, seed)
+    rows = spmv.coo_rows(rp)
+    S = sp.csr_matrix((val, col, rp), shape=(n, n))
+    assert np.array_equal(rows, S.tocoo().row)  # library routine, duplicates kept
+    y = spmv.spmv_coo(n, rows, col, val, x).astype(np.float64)
+    D = spmv.dense(n, rp, col, val)
+    scale = spmv.abs_rowsum(rp, col, val, x)
+    assert np.all(np.abs(y - D @ x.astype(np.float64)) <= 2 ** -23 * scale + 1e-300)
+    # triplet order does not matter (exact sums)
+    sh = np.random.default_rng(seed).permutation(len(rows))
+    y2 = spmv.spmv_coo(n, rows[sh], col[sh], val[sh], x)
+    assert np.array_equal(y2.view(np.int32), y.astype(np.float32).view(np.int32))
+
+
+def test_coo_empty_rows_and_cancellation():
+    rows = np.array([2, 2, 2], np.int64)
+    col = np.array([0, 1, 2], np.int32)
+    val = np.array([1e8, 1.0, -1e8], np.float32)
+    y = spmv.spmv_coo(5, rows, col, val, np.ones(5, np.float32))
+    assert list(y) == [0, 0, 1.0, 0, 0]
