@@ -209,6 +209,8 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->stream_evict_first = (p->opts.evict_first && p->stream_ef) ? 1 : 0;
   info->exec_launches = spmv::exec_launches(p, false);
   info->spmm4_launches = spmv::spmm4_launches(p);
+  info->hot_cols = p->hot_S;
+  info->hot_nnz = p->hot_nnz;
   API_END
 }
 

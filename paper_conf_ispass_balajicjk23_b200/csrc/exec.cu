@@ -99,6 +99,37 @@ __device__ __forceinline__ double warp_sum_d(double s) {
   return s;
 }
 
+// x gather of the lane-mode kernels.  HOT == 0: plain L1-allocating __ldg.
+// HOT != 0 (hot-column set): a column coded c < 0 is hot and
+// read from the 192 KB contiguous copy xh[~c] with L1::evict_last, so the hot
+// lines stay L1-resident for the whole launch and cost no L2 request after
+// their first touch per SM; other columns are read with __ldg (HOT == 1) or
+// without allocating in L1 (HOT == 2), which keeps L1 for the hot copy.
+template <int HOT>
+__device__ __forceinline__ float gx(const float* __restrict__ x, const float* __restrict__ xh,
+                                    int c) {
+  if constexpr (HOT == 0) {
+    return __ldg(x + c);
+  } else {
+    float r;
+    if (c < 0) {
+      asm("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(r) : "l"(xh + ~c));
+    } else if constexpr (HOT == 1) {
+      r = __ldg(x + c);
+    } else {
+      asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(x + c));
+    }
+    return r;
+  }
+}
+
+__global__ void k_hot_gather(const float* __restrict__ x, const int32_t* __restrict__ hot_cols,
+                             int64_t S, float* __restrict__ xh) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S;
+       i += (int64_t)gridDim.x * blockDim.x)
+    xh[i] = x[hot_cols[i]];
+}
+
 // ------------------------------------------------------------ stream tiles
 // k_panel: persistent CTAs, each over a contiguous range of stream tiles (a
 // panel of consecutive rows), two CTAs of 16 warps per SM.  Thread 0 keeps the
@@ -354,12 +385,13 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 }
 
 // ------------------------------------------------------------- long rows
-template <typename OT, bool SS>
+template <typename OT, bool SS, int HOT>
 __global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
                 float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
-                const double* __restrict__ ss_in, double* __restrict__ row_ss) {
+                const double* __restrict__ ss_in, double* __restrict__ row_ss,
+                const float* __restrict__ xh) {
   const int lane = threadIdx.x & 31;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float alpha = alpha_of(ss_in);
@@ -376,13 +408,14 @@ __global__ void __launch_bounds__(256)
                 c3 = __ldcs(cc + j + 96);
       const float v0 = __ldcs(vv + j), v1 = __ldcs(vv + j + 32), v2 = __ldcs(vv + j + 64),
                   v3 = __ldcs(vv + j + 96);
-      const float x0 = __ldg(x + c0), x1 = __ldg(x + c1), x2 = __ldg(x + c2), x3 = __ldg(x + c3);
+      const float x0 = gx<HOT>(x, xh, c0), x1 = gx<HOT>(x, xh, c1), x2 = gx<HOT>(x, xh, c2),
+                  x3 = gx<HOT>(x, xh, c3);
       s = __fadd_rn(s, __fmul_rn(v0, x0));
       s = __fadd_rn(s, __fmul_rn(v1, x1));
       s = __fadd_rn(s, __fmul_rn(v2, x2));
       s = __fadd_rn(s, __fmul_rn(v3, x3));
     }
-    for (; j < L; j += 32) s = __fadd_rn(s, __fmul_rn(__ldcs(vv + j), __ldg(x + __ldcs(cc + j))));
+    for (; j < L; j += 32) s = __fadd_rn(s, __fmul_rn(__ldcs(vv + j), gx<HOT>(x, xh, __ldcs(cc + j))));
     s = warp_tree(s);
     if (lane == 0) {
       const float v = __fmul_rn(s, alpha);
@@ -393,10 +426,11 @@ __global__ void __launch_bounds__(256)
 }
 
 // canonical W = 256 sum of entries [b, b + L) of a row
+template <int HOT>
 __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             const float* __restrict__ val,
                                             const float* __restrict__ x, int64_t b, int64_t L,
-                                            float* red) {
+                                            float* red, const float* __restrict__ xh) {
   const int tid = threadIdx.x;
   float s = 0.f;
   int64_t t = tid;
@@ -405,13 +439,15 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
               c2 = __ldcs(col + b + t + 512), c3 = __ldcs(col + b + t + 768);
     const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256),
                 v2 = __ldcs(val + b + t + 512), v3 = __ldcs(val + b + t + 768);
-    const float x0 = __ldg(x + c0), x1 = __ldg(x + c1), x2 = __ldg(x + c2), x3 = __ldg(x + c3);
+    const float x0 = gx<HOT>(x, xh, c0), x1 = gx<HOT>(x, xh, c1), x2 = gx<HOT>(x, xh, c2),
+                x3 = gx<HOT>(x, xh, c3);
     s = __fadd_rn(s, __fmul_rn(v0, x0));
     s = __fadd_rn(s, __fmul_rn(v1, x1));
     s = __fadd_rn(s, __fmul_rn(v2, x2));
     s = __fadd_rn(s, __fmul_rn(v3, x3));
   }
-  for (; t < L; t += 256) s = __fadd_rn(s, __fmul_rn(__ldcs(val + b + t), __ldg(x + __ldcs(col + b + t))));
+  for (; t < L; t += 256)
+    s = __fadd_rn(s, __fmul_rn(__ldcs(val + b + t), gx<HOT>(x, xh, __ldcs(col + b + t))));
   red[tid] = s;
   __syncthreads();
 #pragma unroll
@@ -424,16 +460,16 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
   return r;  // valid in thread 0
 }
 
-template <typename OT, bool SS>
+template <typename OT, bool SS, int HOT>
 __global__ void __launch_bounds__(256)
     k_cta_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
                const int32_t* __restrict__ rows, const double* __restrict__ ss_in,
-               double* __restrict__ row_ss) {
+               double* __restrict__ row_ss, const float* __restrict__ xh) {
   __shared__ float red[256];
   const int r = rows[blockIdx.x];
   const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
-  const float s = cta_sum256(col, val, x, b, L, red);
+  const float s = cta_sum256<HOT>(col, val, x, b, L, red, xh);
   if (threadIdx.x == 0) {
     const float v = __fmul_rn(s, alpha_of(ss_in));
     y[r] = v;
@@ -441,19 +477,19 @@ __global__ void __launch_bounds__(256)
   }
 }
 
-template <typename OT>
+template <typename OT, int HOT>
 __global__ void __launch_bounds__(256)
     k_hub_chunk(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
                 const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_idx,
-                double* __restrict__ part) {
+                double* __restrict__ part, const float* __restrict__ xh) {
   __shared__ float red[256];
   const int c = blockIdx.x;
   const int r = chunk_row[c];
   const int64_t rb = (int64_t)rp[r], L = (int64_t)rp[r + 1] - rb;
   const int64_t b = rb + (int64_t)chunk_idx[c] * HUB_CHUNK;
   const int64_t m = min((int64_t)HUB_CHUNK, rb + L - b);
-  const float s = cta_sum256(col, val, x, b, m, red);
+  const float s = cta_sum256<HOT>(col, val, x, b, m, red, xh);
   if (threadIdx.x == 0) part[c] = (double)s;
 }
 
@@ -507,6 +543,14 @@ int num_sms(int dev) {
   return g_num_sms > 0 ? g_num_sms : 148;
 }
 
+// 0: no hot-column set; 1 / 2: HOT variant of the gathers (SPMV_HOT_COLD dev knob)
+int hot_mode(const spmv_plan_s* p) {
+  if (!p->hot_S || !p->d_col_hot || p->opts.variant == 1) return 0;
+  int m = 2;
+  if (const char* e = getenv("SPMV_HOT_COLD")) m = atoi(e) ? 2 : 1;  // dev knob
+  return m;
+}
+
 template <typename OT, bool SS>
 void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
   constexpr size_t smem = sizeof(PanelSmem);
@@ -552,18 +596,6 @@ constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 // lanes at different times; evicting it first would make the second read a
 // DRAM refetch (measured: 2.3x DRAM traffic on the 27-point stencil), so
 // EF mode 2 marks only a row's interior chunks evict_first.
-// x gather; GL = 1: L2 evict_last (x outlives the stream's lines in L2)
-template <int GL>
-__device__ __forceinline__ float ld_x(const float* p, uint64_t pol) {
-  if constexpr (GL) {
-    float r;
-    asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r) : "l"(p), "l"(pol));
-    return r;
-  } else {
-    return __ldg(p);
-  }
-}
-
 template <int EF>
 __device__ __forceinline__ void ld_v8_stream(const int32_t* p, int (&r)[8]) {
   if constexpr (EF)
@@ -595,17 +627,16 @@ __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
 // minBlocksPerSM = 1 lets ptxas keep both chunks and all 16 gathers of a
 // 16-entry row in flight per lane (64 registers, 4 CTAs/SM); capping registers
 // for more CTAs measured 20-40 % slower
-template <typename OT, bool SS, int EF, int GL>
+template <typename OT, bool SS, int EF, int HOT>
 __global__ void __launch_bounds__(LN_THREADS, 1)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
-           int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss) {
+           int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss,
+           const float* __restrict__ xh) {
   __shared__ double wss[LN_WARPS];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
   const float alpha = alpha_of(ss_in);
-  uint64_t gpol = 0;
-  if (GL) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(gpol));
   // row pointers are loaded one block iteration ahead
   OT a_n = 0, e_n = 0;
   {
@@ -645,7 +676,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
           ld_v8_stream<EF>(vp + k, vv);
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
-            const float xv = ld_x<GL>(x + cc[i], gpol);
+            const float xv = gx<HOT>(x, xh, cc[i]);
             res = __fadd_rn(res, __fmul_rn(vv[i], (k + i >= lo && k + i < hi) ? xv : 0.f));
           }
         }
@@ -671,7 +702,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
   }
 }
 
-template <typename OT, bool SS, int EF, int GL>
+template <typename OT, bool SS, int EF, int HOT>
 void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
   // grid-stride with ~8 CTAs per resident slot (measured better than one
   // persistent wave on SBM, RMAT-26 and the stencil: r29, profiles/)
@@ -680,31 +711,84 @@ void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in
   const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
   const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
-  k_lane<OT, SS, EF, GL><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val,
-                                                       x, y, p->nrows, ss_in, p->d_blk_ss);
+  k_lane<OT, SS, EF, HOT><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, HOT ? p->d_col_hot : p->d_col,
+                                                        p->d_val, x, y, p->nrows, ss_in,
+                                                        p->d_blk_ss, p->d_xh);
 }
 
 template <typename OT, bool SS>
 void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
   int ef = p->opts.evict_first && p->stream_ef ? 1 : 0;
   if (const char* e = getenv("SPMV_LANE_EF")) ef = atoi(e);  // dev knob: 0 / 1
-  int gl = 0;
-  if (const char* e = getenv("SPMV_LANE_GL")) gl = atoi(e);  // dev knob: x gathers evict_last
+  const int hot = hot_mode(p);
   if (ef == 1) {
-    if (gl) launch_lane_t<OT, SS, 1, 1>(p, x, y, ss_in, s);
+    if (hot == 2) launch_lane_t<OT, SS, 1, 2>(p, x, y, ss_in, s);
+    else if (hot == 1) launch_lane_t<OT, SS, 1, 1>(p, x, y, ss_in, s);
     else launch_lane_t<OT, SS, 1, 0>(p, x, y, ss_in, s);
   } else {
-    if (gl) launch_lane_t<OT, SS, 0, 1>(p, x, y, ss_in, s);
+    if (hot == 2) launch_lane_t<OT, SS, 0, 2>(p, x, y, ss_in, s);
+    else if (hot == 1) launch_lane_t<OT, SS, 0, 1>(p, x, y, ss_in, s);
     else launch_lane_t<OT, SS, 0, 0>(p, x, y, ss_in, s);
+  }
+}
+
+template <typename OT, bool SS, int HOT>
+void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s1,
+                 cudaStream_t s2, bool lane_mode) {
+  const OT* rp = (const OT*)p->d_rp;
+  const int32_t* col = HOT ? p->d_col_hot : p->d_col;
+  const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
+  const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
+  double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
+  if (nw) {
+    const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
+    k_warp_rows<OT, SS, HOT><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh);
+  }
+  if (p->n_cta)
+    k_cta_rows<OT, SS, HOT><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
+                                                                p->d_cta_rows, ss_in, p->d_cta_ss,
+                                                                p->d_xh);
+  if (p->n_chunks) {
+    k_hub_chunk<OT, HOT><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, col, p->d_val, x,
+                                                                p->d_chunk_row, p->d_chunk_idx,
+                                                                p->d_chunk_part, p->d_xh);
+    const unsigned g = (unsigned)((p->n_hub + 127) / 128);
+    if (SS)
+      k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
+                                         ss_in, y, p->d_hub_ss);
+    else
+      k_hub_fix<false><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub,
+                                          p->d_chunk_part, ss_in, y, p->d_hub_ss);
   }
 }
 
 template <typename OT>
 void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
                 cudaStream_t s) {
-  const OT* rp = (const OT*)p->d_rp;
   const bool SS = ss_out != nullptr;
   const bool lane_mode = p->opts.variant != 1;
+  if (lane_mode && hot_mode(p)) {  // refresh the hot copy of x for this exec
+    const unsigned g = (unsigned)std::min<int64_t>((p->hot_S + 255) / 256, (int64_t)num_sms(p->device) * 4);
+    k_hot_gather<<<g, 256, 0, s>>>(x, p->d_hot_cols, p->hot_S, p->d_xh);
+  }
+  const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
+  // The row classes write disjoint rows of y and only read x: the warp-row
+  // kernel and the CTA/hub kernels run on two plan-owned streams concurrently
+  // with the short-row kernel (fork/join by events; CUDA-graph capturable).
+  // The fork is recorded before (early, default) or after the short-row
+  // launch (SPMV_FORK_EARLY=0: the other classes start when it has finished).
+  cudaStream_t s1 = s, s2 = s;
+  const bool conc = p->conc && (nw > 0 || p->n_cta > 0 || p->n_chunks > 0);
+  bool early = true;
+  if (const char* e = getenv("SPMV_FORK_EARLY")) early = atoi(e) != 0;  // dev knob
+  auto fork = [&]() {
+    SPMV_CUDA(cudaEventRecord(p->ev_fork, s));
+    s1 = p->aux[0];
+    s2 = p->aux[1];
+    SPMV_CUDA(cudaStreamWaitEvent(s1, p->ev_fork, 0));
+    SPMV_CUDA(cudaStreamWaitEvent(s2, p->ev_fork, 0));
+  };
+  if (conc && early) fork();
   if (lane_mode) {
     if (p->nrows) {
       if (SS) launch_lane<OT, true>(p, x, y, ss_in, s);
@@ -714,49 +798,18 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
     if (SS) launch_panel<OT, true>(p, x, y, ss_in, s);
     else launch_panel<OT, false>(p, x, y, ss_in, s);
   }
-  const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
-  // The row classes write disjoint rows of y and only read x: the warp-row
-  // kernel and the CTA/hub kernels run on two plan-owned streams concurrently
-  // with the short-row kernel (fork/join by events; CUDA-graph capturable).
-  cudaStream_t s1 = s, s2 = s;
-  const bool conc = p->conc && (nw > 0 || p->n_cta > 0 || p->n_chunks > 0);
-  if (conc) {
-    SPMV_CUDA(cudaEventRecord(p->ev_fork, s));
-    s1 = p->aux[0];
-    s2 = p->aux[1];
-    SPMV_CUDA(cudaStreamWaitEvent(s1, p->ev_fork, 0));
-    SPMV_CUDA(cudaStreamWaitEvent(s2, p->ev_fork, 0));
-  }
+  if (conc && !early) fork();
   {
-    const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
-    double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
-    if (nw) {
-      const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
-      if (SS)
-        k_warp_rows<OT, true><<<g, 256, 0, s1>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
-      else
-        k_warp_rows<OT, false><<<g, 256, 0, s1>>>(rp, p->d_col, p->d_val, x, y, wr, nw, ss_in, wss);
+    const int hot = lane_mode ? hot_mode(p) : 0;
+    if (SS) {
+      if (hot == 2) launch_rows<OT, true, 2>(p, x, y, ss_in, s1, s2, lane_mode);
+      else if (hot == 1) launch_rows<OT, true, 1>(p, x, y, ss_in, s1, s2, lane_mode);
+      else launch_rows<OT, true, 0>(p, x, y, ss_in, s1, s2, lane_mode);
+    } else {
+      if (hot == 2) launch_rows<OT, false, 2>(p, x, y, ss_in, s1, s2, lane_mode);
+      else if (hot == 1) launch_rows<OT, false, 1>(p, x, y, ss_in, s1, s2, lane_mode);
+      else launch_rows<OT, false, 0>(p, x, y, ss_in, s1, s2, lane_mode);
     }
-  }
-  if (p->n_cta) {
-    if (SS)
-      k_cta_rows<OT, true><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, p->d_col, p->d_val, x, y,
-                                                              p->d_cta_rows, ss_in, p->d_cta_ss);
-    else
-      k_cta_rows<OT, false><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, p->d_col, p->d_val, x, y,
-                                                               p->d_cta_rows, ss_in, p->d_cta_ss);
-  }
-  if (p->n_chunks) {
-    k_hub_chunk<OT><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, p->d_col, p->d_val, x,
-                                                           p->d_chunk_row, p->d_chunk_idx,
-                                                           p->d_chunk_part);
-    const unsigned g = (unsigned)((p->n_hub + 127) / 128);
-    if (SS)
-      k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
-                                         ss_in, y, p->d_hub_ss);
-    else
-      k_hub_fix<false><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub,
-                                          p->d_chunk_part, ss_in, y, p->d_hub_ss);
   }
   if (conc) {
     SPMV_CUDA(cudaEventRecord(p->ev_join[0], s1));
@@ -848,7 +901,8 @@ void exec_streams(spmv_plan_s* p) { ensure_aux(p); }
 
 int exec_launches(const spmv_plan_s* p, bool ss) {
   const bool lane_mode = p->opts.variant != 1;
-  return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0) : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
+  return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0) + (hot_mode(p) ? 1 : 0)
+                    : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
          (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0) + (ss ? 1 : 0);
 }
 

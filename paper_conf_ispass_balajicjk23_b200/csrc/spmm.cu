@@ -44,25 +44,42 @@ __device__ __forceinline__ float tree32(float s) {
   return s;
 }
 
+template <int EF>
 __device__ __forceinline__ void ld8_i(const int32_t* p, int (&r)[8]) {
-  asm("ld.global.nc.L1::no_allocate.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
-        "=r"(r[7])
-      : "l"(p));
+  if constexpr (EF)
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+          "=r"(r[7])
+        : "l"(p));
+  else
+    asm("ld.global.nc.L1::no_allocate.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+          "=r"(r[7])
+        : "l"(p));
 }
 
+template <int EF>
 __device__ __forceinline__ void ld8_f(const float* p, float (&r)[8]) {
-  asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-      : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
-        "=f"(r[7])
-      : "l"(p));
+  if constexpr (EF)
+    asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
+          "=f"(r[7])
+        : "l"(p));
+  else
+    asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+        : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
+          "=f"(r[7])
+        : "l"(p));
 }
 
-// lane per row, L <= SHORT_MAX, sequential: identical association to k_lane
-// (slots outside the row add an exact +-0 there; here they are skipped, which
-// gives the same bits because the running sum starts at +0 and is never -0)
-template <typename OT>
-__global__ void __launch_bounds__(L4_THREADS)
+// lane per row, L <= SHORT_MAX, sequential: the association of k_lane.  As
+// there, slots of a chunk outside the row read a valid X row (a neighbouring
+// row's column or the zero tail padding) whose value is replaced by 0, so they
+// contribute v * 0 = +-0 for the (finite) matrix value v, which
+// leaves the running sum unchanged (it starts at +0 and is never -0), so the
+// loop is branch-free and both chunks of a 16-entry row are in flight at once.
+template <typename OT, int EF>
+__global__ void __launch_bounds__(L4_THREADS, 2)
     k_lane4(const OT* __restrict__ rp, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ X, float* __restrict__ Y,
             int64_t nrows) {
@@ -75,14 +92,19 @@ __global__ void __launch_bounds__(L4_THREADS)
     const int32_t* cp = col + (a & ~(OT)7);
     const float* vp = val + (a & ~(OT)7);
     const int lo = (int)(a & 7), hi = lo + L;
+#pragma unroll 2
     for (int k = 0; k < hi; k += 8) {
       int cc[8];
       float vv[8];
-      ld8_i(cp + k, cc);
-      ld8_f(vp + k, vv);
+      ld8_i<EF>(cp + k, cc);
+      ld8_f<EF>(vp + k, vv);
 #pragma unroll
-      for (int i = 0; i < 8; ++i)
-        if (k + i >= lo && k + i < hi) fma4(s, vv[i], ldx4(X, cc[i]));
+      for (int i = 0; i < 8; ++i) {
+        const float4 xg = ldx4(X, cc[i]);
+        const bool in = k + i >= lo && k + i < hi;
+        const float4 xv = in ? xg : make_float4(0.f, 0.f, 0.f, 0.f);
+        fma4(s, vv[i], xv);
+      }
     }
     reinterpret_cast<float4*>(Y)[r] = s;
   }
@@ -220,7 +242,10 @@ void spmm4_typed(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s) {
   if (p->nrows) {
     const int64_t blocks = (p->nrows + L4_THREADS - 1) / L4_THREADS;
     const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)sms * 32));
-    k_lane4<OT><<<g, L4_THREADS, 0, s>>>(rp, p->d_col, p->d_val, X, Y, p->nrows);
+    if (p->opts.evict_first && p->stream_ef)
+      k_lane4<OT, 1><<<g, L4_THREADS, 0, s>>>(rp, p->d_col, p->d_val, X, Y, p->nrows);
+    else
+      k_lane4<OT, 0><<<g, L4_THREADS, 0, s>>>(rp, p->d_col, p->d_val, X, Y, p->nrows);
   }
   cudaStream_t s1 = s, s2 = s;
   const bool conc = p->conc && (p->n_mid > 0 || p->n_cta > 0 || p->n_chunks > 0);

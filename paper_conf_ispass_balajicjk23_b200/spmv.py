@@ -41,7 +41,7 @@ class _Opts(ctypes.Structure):
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("smem_window", ctypes.c_int32),
                 ("l2_hit_ratio", ctypes.c_double), ("variant", ctypes.c_int64),
-                ("reserved", ctypes.c_int64 * 7)]
+                ("hot_x", ctypes.c_int64), ("reserved", ctypes.c_int64 * 6)]
 
 
 class _Info(ctypes.Structure):
@@ -50,7 +50,8 @@ class _Info(ctypes.Structure):
         "n_tiles", "n_warp_rows", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "n_mid_rows",
         "hot_prefix", "ideal_bytes")] + \
         [(n, ctypes.c_int32) for n in ("offset_bytes", "world", "rank", "permuted",
-                                       "l2_window_bytes", "stream_evict_first", "exec_launches", "spmm4_launches")]
+                                       "l2_window_bytes", "stream_evict_first", "exec_launches", "spmm4_launches")] + \
+        [(n, ctypes.c_int64) for n in ("hot_cols", "hot_nnz")]
 
 
 class _Stats(ctypes.Structure):
@@ -140,7 +141,7 @@ class Plan:
 
     def __init__(self, row_ptr, col, val, perm=None, *, world=1, rank=0, l2_window=True,
                  evict_first=True, l2_hit_ratio=1.0, smem_window=True, variant=0,
-                 permute=True, stream=None):
+                 hot_x=0, permute=True, stream=None):
         import torch
         assert row_ptr.is_cuda and col.is_cuda and val.is_cuda
         assert col.dtype == torch.int32 and val.dtype == torch.float32
@@ -162,6 +163,7 @@ class Plan:
         o.l2_hit_ratio = l2_hit_ratio
         o.smem_window = int(smem_window)
         o.variant = int(variant)
+        o.hot_x = int(hot_x)
         o.device = row_ptr.device.index if row_ptr.device.index is not None else -1
         h = ctypes.c_void_p()
         _check(lib().spmv_plan(ctypes.byref(A), _ptr(perm), ctypes.byref(o), ctypes.byref(h)))

@@ -370,3 +370,39 @@ def test_exec_graph_capture_and_concurrency(dev):
         del os.environ["SPMV_CONCURRENT"]
     assert torch.equal(y0.view(torch.int32), y2.view(torch.int32))
     P.close()
+
+
+@pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("rmat12", "longrows", "kron14")])
+def test_hot_column_set_bitwise(dev, name, make, monkeypatch):
+    """The hot-column set (opts.hot_x) only changes where x is
+    read from: y (exec and exec_scaled, both gather variants) is bitwise equal
+    to the plan without it, and the exported CSR is unchanged."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = make()
+    perm = spmv.reorder(A.row_ptr, A.col, "rabbitpp")[0] if name != "longrows" else None
+    P0 = mk_plan(A, perm, dev, hot_x=-1)
+    P1 = mk_plan(A, perm, dev, hot_x=1)
+    i1 = P1.info()
+    assert P0.info()["hot_cols"] == 0 and 0 < i1["hot_cols"] <= 49152
+    # hot set = every column whose count reaches the threshold (recomputed here)
+    pm = np.arange(A.n) if perm is None else np.asarray(perm, np.int64)
+    Bp, Bc, Bv = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, pm)
+    cnt = np.bincount(Bc, minlength=A.n)
+    assert i1["hot_nnz"] == int(cnt[np.argsort(-cnt, kind="stable")[:i1["hot_cols"]]].sum())
+    for a, b in zip(P0.export_csr(), P1.export_csr()):
+        assert torch.equal(a, b)
+    xB = torch.from_numpy(permute.permute_vec(synth.vector(A.n, 4), pm)).to(dev)
+    y0 = P0.exec(xB)
+    for cold in ("0", "1"):
+        monkeypatch.setenv("SPMV_HOT_COLD", cold)
+        y1 = P1.exec(xB)
+        assert torch.equal(y0.view(torch.int32), y1.view(torch.int32)), cold
+    s0 = torch.zeros(1, dtype=torch.float64, device=dev)
+    s1 = torch.zeros(1, dtype=torch.float64, device=dev)
+    z0, z1 = torch.empty_like(y0), torch.empty_like(y0)
+    P0.exec_scaled(xB, z0, None, s0)
+    P1.exec_scaled(xB, z1, None, s1)
+    assert torch.equal(z0, z1) and torch.equal(s0, s1)
+    assert P1.info()["exec_launches"] == P0.info()["exec_launches"] + 1
+    P0.close()
+    P1.close()
