@@ -664,8 +664,9 @@ static void choose_hot(spmv_plan_s* p, const uint32_t* cnt, int64_t n, int64_t n
   p->hot_S = 0;
   int64_t mode = p->opts.hot_x;
   if (const char* e = getenv("SPMV_HOT")) mode = atoll(e);  // dev knob (A/B)
-  if (mode < 0 || p->world != 1 || p->opts.variant == 1 || n == 0 || nnz == 0) return;
-  if (mode == 0 && n < 4 * (int64_t)HOT_MAX) return;
+  // auto (0) is off: measured on C3 (profiles r33) the L1-resident copy does
+  // not shorten the L1-wavefront-bound gathers; kept for A/B (mode > 0)
+  if (mode <= 0 || p->world != 1 || p->opts.variant == 1 || n == 0 || nnz == 0) return;
   unsigned long long* nb = dalloc<unsigned long long>(2 * HOT_BINS);
   SPMV_CUDA(cudaMemsetAsync(nb, 0, sizeof(unsigned long long) * 2 * HOT_BINS, s));
   k_cnt_hist<<<grid_for(n), TPB, 0, s>>>(cnt, n, nb, nb + HOT_BINS);
