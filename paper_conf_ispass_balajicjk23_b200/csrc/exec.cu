@@ -425,6 +425,54 @@ __global__ void __launch_bounds__(256)
   }
 }
 
+// k_warp_rows with the hot-column set in shared memory (hot mode 3): one
+// persistent 1024-thread CTA per SM stages xh (<= 192 KB) once; a gather of a
+// hot column (coded c < 0) is a shared-memory read, so it costs bank cycles
+// instead of an L1 wavefront per distinct line (profiles r33: the gathers of
+// power-law rows are L1-wavefront bound).  Same association as k_warp_rows.
+template <typename OT, bool SS>
+__global__ void __launch_bounds__(1024, 1)
+    k_warp_rows_smem(const OT* __restrict__ rp, const int32_t* __restrict__ col,
+                     const float* __restrict__ val, const float* __restrict__ x,
+                     float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
+                     const double* __restrict__ ss_in, double* __restrict__ row_ss,
+                     const float* __restrict__ xh, int hot_S) {
+  extern __shared__ float sx[];
+  for (int i = threadIdx.x; i < hot_S; i += blockDim.x) sx[i] = xh[i];
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const float alpha = alpha_of(ss_in);
+  auto g = [&](int c) { return c < 0 ? sx[~c] : __ldg(x + c); };
+  for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < nrows; q += W) {
+    const int r = rows[q];
+    const int64_t b = (int64_t)rp[r];
+    const int L = (int)((int64_t)rp[r + 1] - b);
+    const int32_t* cc = col + b;
+    const float* vv = val + b;
+    float s = 0.f;
+    int j = lane;
+    for (; j + 96 < L; j += 128) {
+      const int c0 = __ldcs(cc + j), c1 = __ldcs(cc + j + 32), c2 = __ldcs(cc + j + 64),
+                c3 = __ldcs(cc + j + 96);
+      const float v0 = __ldcs(vv + j), v1 = __ldcs(vv + j + 32), v2 = __ldcs(vv + j + 64),
+                  v3 = __ldcs(vv + j + 96);
+      const float x0 = g(c0), x1 = g(c1), x2 = g(c2), x3 = g(c3);
+      s = __fadd_rn(s, __fmul_rn(v0, x0));
+      s = __fadd_rn(s, __fmul_rn(v1, x1));
+      s = __fadd_rn(s, __fmul_rn(v2, x2));
+      s = __fadd_rn(s, __fmul_rn(v3, x3));
+    }
+    for (; j < L; j += 32) s = __fadd_rn(s, __fmul_rn(__ldcs(vv + j), g(__ldcs(cc + j))));
+    s = warp_tree(s);
+    if (lane == 0) {
+      const float v = __fmul_rn(s, alpha);
+      y[r] = v;
+      if (SS) row_ss[q] = (double)v * (double)v;
+    }
+  }
+}
+
 // canonical W = 256 sum of entries [b, b + L) of a row
 template <int HOT>
 __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
@@ -543,11 +591,14 @@ int num_sms(int dev) {
   return g_num_sms > 0 ? g_num_sms : 148;
 }
 
-// 0: no hot-column set; 1 / 2: HOT variant of the gathers (SPMV_HOT_COLD dev knob)
+// 0: no hot-column set; 1 / 2: gathers of every lane-mode kernel read hot
+// columns from the L1-resident copy (cold: __ldg / no L1 allocation);
+// 3 (default): k_warp_rows_smem keeps the hot copy in shared memory, the other
+// kernels read the plain col array.  SPMV_HOT_MODE dev knob.
 int hot_mode(const spmv_plan_s* p) {
   if (!p->hot_S || !p->d_col_hot || p->opts.variant == 1) return 0;
-  int m = 2;
-  if (const char* e = getenv("SPMV_HOT_COLD")) m = atoi(e) ? 2 : 1;  // dev knob
+  int m = 3;
+  if (const char* e = getenv("SPMV_HOT_MODE")) m = std::min(3, std::max(1, atoi(e)));
   return m;
 }
 
@@ -720,7 +771,7 @@ template <typename OT, bool SS>
 void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
   int ef = p->opts.evict_first && p->stream_ef ? 1 : 0;
   if (const char* e = getenv("SPMV_LANE_EF")) ef = atoi(e);  // dev knob: 0 / 1
-  const int hot = hot_mode(p);
+  const int hot = hot_mode(p) == 3 ? 0 : hot_mode(p);
   if (ef == 1) {
     if (hot == 2) launch_lane_t<OT, SS, 1, 2>(p, x, y, ss_in, s);
     else if (hot == 1) launch_lane_t<OT, SS, 1, 1>(p, x, y, ss_in, s);
@@ -732,26 +783,41 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   }
 }
 
+// Row-class kernels other than the short-row one.  HOT 1/2: every gather
+// uses the coded columns; HOT 3: only the MID rows (k_warp_rows_smem, hot copy
+// in shared memory), the CTA / hub classes read the plain columns.
 template <typename OT, bool SS, int HOT>
 void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s1,
                  cudaStream_t s2, bool lane_mode) {
+  constexpr int HG = HOT == 3 ? 0 : HOT;  // gather variant of the CTA / hub (and MID) kernels
   const OT* rp = (const OT*)p->d_rp;
-  const int32_t* col = HOT ? p->d_col_hot : p->d_col;
+  const int32_t* col = HG ? p->d_col_hot : p->d_col;
   const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
   const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
   double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
-  if (nw) {
+  if (nw && HOT == 3) {
+    static bool attr = false;
+    if (!attr) {
+      SPMV_CUDA(cudaFuncSetAttribute(k_warp_rows_smem<OT, SS>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)(sizeof(float) * HOT_MAX)));
+      attr = true;
+    }
+    const size_t smem = sizeof(float) * (size_t)p->hot_S;
+    k_warp_rows_smem<OT, SS><<<(unsigned)num_sms(p->device), 1024, smem, s1>>>(
+        rp, p->d_col_hot, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh, (int)p->hot_S);
+  } else if (nw) {
     const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
-    k_warp_rows<OT, SS, HOT><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh);
+    k_warp_rows<OT, SS, HG><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh);
   }
   if (p->n_cta)
-    k_cta_rows<OT, SS, HOT><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
-                                                                p->d_cta_rows, ss_in, p->d_cta_ss,
-                                                                p->d_xh);
+    k_cta_rows<OT, SS, HG><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
+                                                               p->d_cta_rows, ss_in, p->d_cta_ss,
+                                                               p->d_xh);
   if (p->n_chunks) {
-    k_hub_chunk<OT, HOT><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, col, p->d_val, x,
-                                                                p->d_chunk_row, p->d_chunk_idx,
-                                                                p->d_chunk_part, p->d_xh);
+    k_hub_chunk<OT, HG><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, col, p->d_val, x,
+                                                               p->d_chunk_row, p->d_chunk_idx,
+                                                               p->d_chunk_part, p->d_xh);
     const unsigned g = (unsigned)((p->n_hub + 127) / 128);
     if (SS)
       k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
@@ -802,11 +868,13 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   {
     const int hot = lane_mode ? hot_mode(p) : 0;
     if (SS) {
-      if (hot == 2) launch_rows<OT, true, 2>(p, x, y, ss_in, s1, s2, lane_mode);
+      if (hot == 3) launch_rows<OT, true, 3>(p, x, y, ss_in, s1, s2, lane_mode);
+      else if (hot == 2) launch_rows<OT, true, 2>(p, x, y, ss_in, s1, s2, lane_mode);
       else if (hot == 1) launch_rows<OT, true, 1>(p, x, y, ss_in, s1, s2, lane_mode);
       else launch_rows<OT, true, 0>(p, x, y, ss_in, s1, s2, lane_mode);
     } else {
-      if (hot == 2) launch_rows<OT, false, 2>(p, x, y, ss_in, s1, s2, lane_mode);
+      if (hot == 3) launch_rows<OT, false, 3>(p, x, y, ss_in, s1, s2, lane_mode);
+      else if (hot == 2) launch_rows<OT, false, 2>(p, x, y, ss_in, s1, s2, lane_mode);
       else if (hot == 1) launch_rows<OT, false, 1>(p, x, y, ss_in, s1, s2, lane_mode);
       else launch_rows<OT, false, 0>(p, x, y, ss_in, s1, s2, lane_mode);
     }

@@ -375,7 +375,7 @@ def test_exec_graph_capture_and_concurrency(dev):
 @pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("rmat12", "longrows", "kron14")])
 def test_hot_column_set_bitwise(dev, name, make, monkeypatch):
     """The hot-column set (opts.hot_x) only changes where x is
-    read from: y (exec and exec_scaled, both gather variants) is bitwise equal
+    read from: y (exec and exec_scaled, all three gather modes) is bitwise equal
     to the plan without it, and the exported CSR is unchanged."""
     from paper_conf_ispass_balajicjk23_b200 import spmv
     A = make()
@@ -393,10 +393,11 @@ def test_hot_column_set_bitwise(dev, name, make, monkeypatch):
         assert torch.equal(a, b)
     xB = torch.from_numpy(permute.permute_vec(synth.vector(A.n, 4), pm)).to(dev)
     y0 = P0.exec(xB)
-    for cold in ("0", "1"):
-        monkeypatch.setenv("SPMV_HOT_COLD", cold)
+    for mode in ("1", "2", "3"):
+        monkeypatch.setenv("SPMV_HOT_MODE", mode)
         y1 = P1.exec(xB)
-        assert torch.equal(y0.view(torch.int32), y1.view(torch.int32)), cold
+        assert torch.equal(y0.view(torch.int32), y1.view(torch.int32)), mode
+    monkeypatch.delenv("SPMV_HOT_MODE")
     s0 = torch.zeros(1, dtype=torch.float64, device=dev)
     s1 = torch.zeros(1, dtype=torch.float64, device=dev)
     z0, z1 = torch.empty_like(y0), torch.empty_like(y0)
