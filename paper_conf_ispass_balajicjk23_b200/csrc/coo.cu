@@ -20,6 +20,7 @@
 // before the first / after the last entry) is zeroed by the thread holding
 // the entry after it, so y is written exactly once and needs no memset.
 #include <algorithm>
+#include <cstdlib>
 
 #include "plan.cuh"
 
@@ -212,6 +213,147 @@ __global__ void __launch_bounds__(CO_THREADS)
   }
 }
 
+// k_coo_w (variant 2): warp tiles of CW_TILE = 512 entries, 16 per lane (two
+// 256-bit chunks of row / col / val, 16 gathers in flight), no shared memory
+// and no CTA barrier.  Lane pieces of a row crossing lanes are combined with
+// a segmented suffix scan over the warp in fp64 (shuffles; the association is
+// fixed by the lane layout); pieces crossing warp tiles go through k_coo_fix
+// exactly like the CTA tiles of k_coo.
+constexpr int CW_E = 16;
+constexpr int CW_TILE = 32 * CW_E;
+
+template <int EF>
+__global__ void __launch_bounds__(256)
+    k_coo_w(const int32_t* __restrict__ row, const int32_t* __restrict__ col,
+            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
+            int64_t nnz, int64_t nrows, int64_t ntiles, int32_t* __restrict__ t_frow,
+            int32_t* __restrict__ t_lrow, double* __restrict__ t_fpart,
+            double* __restrict__ t_lpart, uint8_t* __restrict__ t_flags) {
+  const int lane = threadIdx.x & 31;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t tile = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < ntiles;
+       tile += W) {
+    const int64_t e0 = tile * CW_TILE;
+    const int64_t eb = e0 + (int64_t)lane * CW_E;
+    const int nh = (int)max((int64_t)0, min((int64_t)CW_E, nnz - eb));
+    int rr[16], cc[16];
+    float vv[16];
+    if (nh == CW_E) {
+      int r8[8], c8[8];
+      float v8[8];
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        ld8<EF>(row + eb + 8 * h, r8);
+        ld8<EF>(col + eb + 8 * h, c8);
+        ld8<EF>(val + eb + 8 * h, v8);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          rr[8 * h + i] = r8[i];
+          cc[8 * h + i] = c8[i];
+          vv[8 * h + i] = v8[i];
+        }
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        rr[i] = i < nh ? row[eb + i] : -1;
+        cc[i] = i < nh ? col[eb + i] : 0;
+        vv[i] = i < nh ? val[eb + i] : 0.f;
+      }
+    }
+    float xv[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) xv[i] = i < nh ? __ldg(x + cc[i]) : 0.f;
+    int mylast = -1;
+#pragma unroll
+    for (int i = 0; i < 16; ++i) mylast = i < nh ? rr[i] : mylast;
+    int prow = __shfl_up_sync(0xffffffffu, mylast, 1);
+    if (lane == 0) prow = e0 > 0 && nh > 0 ? row[e0 - 1] : -1;
+    int hrow = -1, cur = -1, last = prow;
+    float hsum = 0.f, run = 0.f;
+    bool single = true;
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      if (i < nh) {
+        const int r = rr[i];
+        if (r != cur) {
+          if (cur >= 0) {
+            if (hrow < 0) {
+              hrow = cur;
+              hsum = run;
+              if (cur != prow) y[cur] = run;  // started and ended in this lane
+            } else {
+              y[cur] = run;  // interior run
+            }
+            single = false;
+          }
+          zero_rows(y, (int64_t)last + 1, r);
+          cur = r;
+          run = 0.f;
+        }
+        run = __fadd_rn(run, __fmul_rn(vv[i], xv[i]));
+        last = r;
+      }
+    }
+    if (nh > 0 && eb + nh == nnz) zero_rows(y, (int64_t)cur + 1, nrows);
+    if (single) {
+      hrow = cur;
+      hsum = run;
+    }
+    const int64_t tile_end = min(nnz, e0 + CW_TILE);
+    // first row of the next warp tile (decides whether lane 31's chain is open)
+    int nxt = -1;
+    if (lane == 31 && tile_end < nnz) nxt = row[tile_end];
+    nxt = __shfl_sync(0xffffffffu, nxt, 31);
+    // cont: my head run continues the previous lane's last row
+    const bool cont = nh > 0 && hrow == prow;
+    const unsigned contm = __ballot_sync(0xffffffffu, cont);
+    // link: my (single) run is continued by the next lane (or next tile)
+    const bool link = nh > 0 && single &&
+                      (lane < 31 ? ((contm >> (lane + 1)) & 1u) != 0 : nxt == cur);
+    const unsigned linkm = __ballot_sync(0xffffffffu, link);
+    // segmented suffix sum S_l = v_l + (link_l ? S_{l+1} : 0), v_l = cont ? hsum : 0
+    double v = cont ? (double)hsum : 0.0;
+    bool f = link && lane < 31;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const double vo = __shfl_down_sync(0xffffffffu, v, d);
+      const bool fo = __shfl_down_sync(0xffffffffu, f ? 1 : 0, d) != 0;
+      if (f && lane + d < 32) {
+        v += vo;
+        f = fo;
+      }
+    }
+    const double vnext = __shfl_down_sync(0xffffffffu, v, 1);  // S_{l+1}
+    // chain from lane s runs through lane 31 into the next tile iff links s..31 are all set
+    auto open_from = [&](int st) { return st <= 31 && (linkm >> st) == (0xffffffffu >> st); };
+    // owner of my tail run (it starts in this lane)
+    if (nh > 0 && !(single && cur == prow)) {
+      const bool nc = lane < 31 && ((contm >> (lane + 1)) & 1u);
+      const double tot = (double)run + (nc ? vnext : 0.0);
+      const bool open = lane < 31 ? (nc && open_from(lane + 1)) : (nxt == cur);
+      if (open && nxt == cur && tile_end < nnz) t_lpart[tile] = tot;
+      else y[cur] = (float)tot;
+    }
+    if (lane == 0) {
+      uint8_t fl = 0;
+      if (cont) {
+        t_fpart[tile] = v;  // S_0: the first row's piece of this tile
+        fl |= T_PREV;
+        if (open_from(0)) fl |= T_SINGLE;
+      }
+      const int lrow = row[tile_end - 1];
+      if (tile_end < nnz && nxt == lrow) {
+        fl |= T_NEXT;
+        if (!((fl & T_SINGLE) && (fl & T_PREV))) fl |= T_OWN_LAST;
+      }
+      t_frow[tile] = hrow;
+      t_lrow[tile] = lrow;
+      t_flags[tile] = fl;
+    }
+  }
+}
+
 // rows spanning tiles: the tile where the row starts (T_OWN_LAST) adds the
 // pieces of the following tiles in tile order (fp64), rounds once
 __global__ void k_coo_fix(int64_t ntiles, const int32_t* __restrict__ t_frow,
@@ -251,7 +393,7 @@ void* dmalloc(size_t bytes) {
 void coo_build(spmv_plan_s* p, cudaStream_t s) {
   if (p->d_coo_row) return;
   const int64_t nz = p->nnz_local;
-  p->coo_tiles = (nz + COO_TILE - 1) / COO_TILE;
+  p->coo_tiles = (nz + CW_TILE - 1) / CW_TILE;  // the finer (warp) tiling bounds both
   p->d_coo_row = (int32_t*)dmalloc(sizeof(int32_t) * (size_t)(nz + 8));
   const int64_t T = std::max<int64_t>(p->coo_tiles, 1);
   p->d_coo_trow = (int32_t*)dmalloc(sizeof(int32_t) * 2 * (size_t)T);
@@ -276,19 +418,32 @@ void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s) {
     SPMV_CUDA(cudaMemsetAsync(y, 0, sizeof(float) * (size_t)p->nrows, s));
     return;
   }
-  const int64_t T = p->coo_tiles;
-  const unsigned g = (unsigned)std::min<int64_t>(T, (int64_t)sms(p->device) * 8);
+  int v = 2;
+  if (const char* e = getenv("SPMV_COO_V")) v = atoi(e) == 1 ? 1 : 2;  // dev knob
+  const int64_t T = v == 1 ? (p->nnz_local + COO_TILE - 1) / COO_TILE : p->coo_tiles;
   int32_t* frow = p->d_coo_trow;
   int32_t* lrow = p->d_coo_trow + T;
   double* fpart = p->d_coo_tpart;
   double* lpart = p->d_coo_tpart + T;
   // every chunk is read by exactly one thread, so evict_first never costs a refetch
-  if (p->opts.evict_first)
-    k_coo<1><<<g, CO_THREADS, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
-                                      p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
-  else
-    k_coo<0><<<g, CO_THREADS, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
-                                      p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
+  const int ef = p->opts.evict_first ? 1 : 0;
+  if (v == 1) {
+    const unsigned g = (unsigned)std::min<int64_t>(T, (int64_t)sms(p->device) * 8);
+    if (ef)
+      k_coo<1><<<g, CO_THREADS, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
+                                        p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
+    else
+      k_coo<0><<<g, CO_THREADS, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
+                                        p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
+  } else {
+    const unsigned g = (unsigned)std::min<int64_t>((T + 7) / 8, (int64_t)sms(p->device) * 16);
+    if (ef)
+      k_coo_w<1><<<g, 256, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
+                                   p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
+    else
+      k_coo_w<0><<<g, 256, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
+                                   p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
+  }
   k_coo_fix<<<(unsigned)((T + 255) / 256), 256, 0, s>>>(T, frow, lrow, fpart, lpart,
                                                         p->d_coo_tflag, y);
   SPMV_LAUNCH_CHECK();

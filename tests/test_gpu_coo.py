@@ -34,6 +34,9 @@ def _edge_matrices():
     L[3001] = 7
     L[3002] = 9
     L[4000] = 10000        # crosses 5+ tiles
+    L[4200:4264] = 512     # rows exactly one warp tile long
+    L[4300:4310] = 16      # one lane each
+    L[4400] = 513
     L[4001:4100] = rng.integers(0, 20, 99)
     L[8990] = 3
     rp = np.concatenate([[0], np.cumsum(L)])
@@ -51,8 +54,12 @@ def _edge_matrices():
 ALL = CASES + [(nm, (lambda m=m: m)) for nm, m in _edge_matrices()]
 
 
+@pytest.mark.parametrize("variant", ["1", "2"])
 @pytest.mark.parametrize("name,make", ALL)
-def test_coo_matches_oracle(dev, name, make):
+def test_coo_matches_oracle(dev, name, make, variant, monkeypatch):
+    """variant 1: CTA tiles of 2048 entries (k_coo); 2: warp tiles of 512
+    (k_coo_w, the default) -- SPMV_COO_V dev knob."""
+    monkeypatch.setenv("SPMV_COO_V", variant)
     A = make()
     perm = rabbit.random_perm(A.n, 21) if A.nnz and name not in ("edges", "lastrow") else None
     P = mk_plan(A, perm, dev)
