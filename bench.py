@@ -267,8 +267,26 @@ def run_gpu(args):
         e1.record(stream)
         torch.cuda.synchronize()
         warm_ms = e0.elapsed_time(e1) / K
+        graph_ms = None
+        if world == 1 and ideal < 256 * 2**20:
+            # small (L2-resident) matrices: launch overhead dominates a single
+            # exec, so also time G execs captured in one CUDA graph (warm)
+            G = 200
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                for _ in range(G):
+                    step()
+            g.replay()
+            torch.cuda.synchronize()
+            e0.record(stream)
+            for _ in range(5):
+                g.replay()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            graph_ms = e0.elapsed_time(e1) / (5 * G)
         gbs = ideal / (ms * 1e-3) / 1e9
         res = {"ms": ms, "ms_median": statistics.median(times), "warm_ms": warm_ms,
+               "graph_warm_ms": graph_ms,
                "gbs_ideal_over_t": gbs, "gflops": 2 * A.nnz / (ms * 1e-3) / 1e9,
                "runtime_over_ideal": hbm / gbs, "reorder_s": st.seconds, "plan_permute_s": plan_s,
                "insularity": st.insularity, "insular_frac": st.insular_frac,

@@ -541,6 +541,81 @@ __global__ void __launch_bounds__(256)
   if (threadIdx.x == 0) part[c] = (double)s;
 }
 
+// CTA rows and hub chunks with the hot-column set in shared memory (hot
+// mode 3): one persistent 1024-thread CTA per SM stages xh once; its four
+// 256-thread groups take work items (CTA rows first, then hub chunks) in a
+// fixed round robin and reduce each with the canonical W = 256 association of
+// cta_sum256 (group-local named barriers), so y is bitwise that of
+// k_cta_rows / k_hub_chunk.
+template <typename OT, bool SS>
+__global__ void __launch_bounds__(1024, 1)
+    k_long_rows_smem(const OT* __restrict__ rp, const int32_t* __restrict__ col,
+                     const float* __restrict__ val, const float* __restrict__ x,
+                     float* __restrict__ y, const int32_t* __restrict__ cta_rows, int64_t n_cta,
+                     const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_idx,
+                     int64_t n_chunks, double* __restrict__ part, const double* __restrict__ ss_in,
+                     double* __restrict__ row_ss, const float* __restrict__ xh, int hot_S) {
+  extern __shared__ float sx[];
+  __shared__ float red[4][256];
+  for (int i = threadIdx.x; i < hot_S; i += blockDim.x) sx[i] = xh[i];
+  __syncthreads();
+  const int grp = threadIdx.x >> 8, t0 = threadIdx.x & 255;
+  float* rd = red[grp];
+  const float alpha = alpha_of(ss_in);
+  auto g = [&](int c) { return c < 0 ? sx[~c] : __ldg(x + c); };
+  auto bar = [&]() { asm volatile("bar.sync %0, 256;" ::"r"(grp + 1) : "memory"); };
+  const int64_t total = n_cta + n_chunks;
+  for (int64_t it = (int64_t)blockIdx.x * 4 + grp; it < total; it += (int64_t)gridDim.x * 4) {
+    int64_t b, L;
+    int r = -1;
+    if (it < n_cta) {
+      r = cta_rows[it];
+      b = (int64_t)rp[r];
+      L = (int64_t)rp[r + 1] - b;
+    } else {
+      const int64_t c = it - n_cta;
+      const int hr = chunk_row[c];
+      const int64_t rb = (int64_t)rp[hr], RL = (int64_t)rp[hr + 1] - rb;
+      b = rb + (int64_t)chunk_idx[c] * HUB_CHUNK;
+      L = min((int64_t)HUB_CHUNK, rb + RL - b);
+    }
+    float s = 0.f;
+    int64_t t = t0;
+    for (; t + 768 < L; t += 1024) {
+      const int c0 = __ldcs(col + b + t), c1 = __ldcs(col + b + t + 256),
+                c2 = __ldcs(col + b + t + 512), c3 = __ldcs(col + b + t + 768);
+      const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256),
+                  v2 = __ldcs(val + b + t + 512), v3 = __ldcs(val + b + t + 768);
+      const float x0 = g(c0), x1 = g(c1), x2 = g(c2), x3 = g(c3);
+      s = __fadd_rn(s, __fmul_rn(v0, x0));
+      s = __fadd_rn(s, __fmul_rn(v1, x1));
+      s = __fadd_rn(s, __fmul_rn(v2, x2));
+      s = __fadd_rn(s, __fmul_rn(v3, x3));
+    }
+    for (; t < L; t += 256) s = __fadd_rn(s, __fmul_rn(__ldcs(val + b + t), g(__ldcs(col + b + t))));
+    rd[t0] = s;
+    bar();
+#pragma unroll
+    for (int o = 128; o >= 32; o >>= 1) {
+      if (t0 < o) rd[t0] = __fadd_rn(rd[t0], rd[t0 + o]);
+      bar();
+    }
+    if (t0 < 32) {
+      const float w = warp_tree(rd[t0]);
+      if (t0 == 0) {
+        if (it < n_cta) {
+          const float v = __fmul_rn(w, alpha);
+          y[r] = v;
+          if (SS) row_ss[it] = (double)v * (double)v;
+        } else {
+          part[it - n_cta] = (double)w;
+        }
+      }
+    }
+    bar();  // rd is reused by the group's next item
+  }
+}
+
 template <bool SS>
 __global__ void k_hub_fix(const int32_t* __restrict__ hub_rows, const int32_t* __restrict__ choff,
                           int64_t nh, const double* __restrict__ part,
@@ -810,14 +885,32 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
     const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
     k_warp_rows<OT, SS, HG><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh);
   }
-  if (p->n_cta)
+  const bool long_smem = HOT == 3 && (p->n_cta || p->n_chunks);
+  if (long_smem) {
+    static bool attr = false;
+    if (!attr) {
+      SPMV_CUDA(cudaFuncSetAttribute(k_long_rows_smem<OT, SS>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)(sizeof(float) * HOT_MAX)));
+      attr = true;
+    }
+    const size_t smem = sizeof(float) * (size_t)p->hot_S;
+    const int64_t items = p->n_cta + p->n_chunks;
+    const unsigned g = (unsigned)std::min<int64_t>((items + 3) / 4, num_sms(p->device));
+    k_long_rows_smem<OT, SS><<<g, 1024, smem, s2>>>(
+        rp, p->d_col_hot, p->d_val, x, y, p->d_cta_rows, p->n_cta, p->d_chunk_row,
+        p->d_chunk_idx, p->n_chunks, p->d_chunk_part, ss_in, p->d_cta_ss, p->d_xh,
+        (int)p->hot_S);
+  } else if (p->n_cta) {
     k_cta_rows<OT, SS, HG><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
                                                                p->d_cta_rows, ss_in, p->d_cta_ss,
                                                                p->d_xh);
+  }
   if (p->n_chunks) {
-    k_hub_chunk<OT, HG><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, col, p->d_val, x,
-                                                               p->d_chunk_row, p->d_chunk_idx,
-                                                               p->d_chunk_part, p->d_xh);
+    if (!long_smem)
+      k_hub_chunk<OT, HG><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, col, p->d_val, x,
+                                                                 p->d_chunk_row, p->d_chunk_idx,
+                                                                 p->d_chunk_part, p->d_xh);
     const unsigned g = (unsigned)((p->n_hub + 127) / 128);
     if (SS)
       k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
@@ -969,9 +1062,12 @@ void exec_streams(spmv_plan_s* p) { ensure_aux(p); }
 
 int exec_launches(const spmv_plan_s* p, bool ss) {
   const bool lane_mode = p->opts.variant != 1;
-  return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0) + (hot_mode(p) ? 1 : 0)
+  const int hot = lane_mode ? hot_mode(p) : 0;
+  const int longk = hot == 3 ? ((p->n_cta || p->n_chunks) ? 1 : 0) + (p->n_chunks ? 1 : 0)
+                             : (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0);
+  return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0) + (hot ? 1 : 0)
                     : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
-         (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0) + (ss ? 1 : 0);
+         longk + (ss ? 1 : 0);
 }
 
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,

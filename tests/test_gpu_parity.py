@@ -404,6 +404,8 @@ def test_hot_column_set_bitwise(dev, name, make, monkeypatch):
     P0.exec_scaled(xB, z0, None, s0)
     P1.exec_scaled(xB, z1, None, s1)
     assert torch.equal(z0, z1) and torch.equal(s0, s1)
-    assert P1.info()["exec_launches"] == P0.info()["exec_launches"] + 1
+    i0 = P0.info()
+    both = i0["n_cta_rows"] > 0 and i0["n_hub_chunks"] > 0  # mode 3 fuses their kernels
+    assert P1.info()["exec_launches"] == i0["exec_launches"] + 1 - (1 if both else 0)
     P0.close()
     P1.close()
