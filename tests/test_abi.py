@@ -111,3 +111,15 @@ def test_reorder_empty_and_isolated():
     assert sorted(perm.tolist()) == [0, 1, 2] and st.n_communities == 3
     perm, _ = spmv.reorder(np.zeros(1, np.int64), np.zeros(0, np.int32), "rabbit")
     assert perm.size == 0
+
+
+def test_table4_entry_points_reject_null_plan_without_gpu():
+    """spmv_exec_spmm4 / spmv_exec_coo / spmv_export_coo_rows validate their
+    arguments before touching the device (EINVAL + message)."""
+    L = spmv.lib()
+    for fn, args in (("spmv_exec_spmm4", (None, None, None, None)),
+                     ("spmv_exec_coo", (None, None, None, None)),
+                     ("spmv_export_coo_rows", (None, None, None))):
+        st = getattr(L, fn)(*args)
+        assert st == 1, fn
+        assert b"NULL" in L.spmv_last_error(), fn
