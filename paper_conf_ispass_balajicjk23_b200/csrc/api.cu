@@ -206,7 +206,7 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->rank = p->rank;
   info->permuted = p->permuted ? 1 : 0;
   info->l2_window_bytes = (int32_t)p->l2_window_bytes;
-  info->stream_evict_first = (p->opts.evict_first && p->stream_ef) ? 1 : 0;
+  info->stream_evict_first = spmv::lane_ef_mode(p);
   info->exec_launches = spmv::exec_launches(p, false);
   info->spmm4_launches = spmv::spmm4_launches(p);
   info->hot_cols = p->hot_S;

@@ -666,8 +666,8 @@ int num_sms(int dev) {
   return g_num_sms > 0 ? g_num_sms : 148;
 }
 
-// 0: no hot-column set; 1 / 2: gathers of every lane-mode kernel read hot
-// columns from the L1-resident copy (cold: __ldg / no L1 allocation);
+// 0: no hot-column set; 1 / 2: the MID / CTA / hub kernels read hot columns
+// from the L1-resident copy (cold: __ldg / no L1 allocation);
 // 3 (default): k_warp_rows_smem keeps the hot copy in shared memory, the other
 // kernels read the plain col array.  SPMV_HOT_MODE dev knob.
 int hot_mode(const spmv_plan_s* p) {
@@ -721,10 +721,12 @@ constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 // neighbouring row (the first / last chunk of a row) is read twice, by two
 // lanes at different times; evicting it first would make the second read a
 // DRAM refetch (measured: 2.3x DRAM traffic on the 27-point stencil), so
-// EF mode 2 marks only a row's interior chunks evict_first.
+// EF mode 2 loads a row's FIRST chunk normally and the rest evict_first: a
+// chunk shared by rows r and r + 1 is read first by lane r + 1 (as its first
+// chunk, kept) and last by lane r (its last chunk, then marked evict_first).
 template <int EF>
 __device__ __forceinline__ void ld_v8_stream(const int32_t* p, int (&r)[8]) {
-  if constexpr (EF)
+  if constexpr (EF == 1)
     asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.s32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
         : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
           "=r"(r[7])
@@ -738,7 +740,7 @@ __device__ __forceinline__ void ld_v8_stream(const int32_t* p, int (&r)[8]) {
 
 template <int EF>
 __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
-  if constexpr (EF)
+  if constexpr (EF == 1)
     asm("ld.global.nc.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
         : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]),
           "=f"(r[7])
@@ -798,8 +800,13 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
         for (int k = 0; k < hi; k += 8) {
           int cc[8];
           float vv[8];
-          ld_v8_stream<EF>(cp + k, cc);
-          ld_v8_stream<EF>(vp + k, vv);
+          if (EF == 2 && k == 0) {  // (warp-uniform: every lane starts at k = 0)
+            ld_v8_stream<0>(cp + k, cc);
+            ld_v8_stream<0>(vp + k, vv);
+          } else {
+            ld_v8_stream<EF == 0 ? 0 : 1>(cp + k, cc);
+            ld_v8_stream<EF == 0 ? 0 : 1>(vp + k, vv);
+          }
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
             const float xv = gx<HOT>(x, xh, cc[i]);
@@ -837,25 +844,29 @@ void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in
   const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
   const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
-  k_lane<OT, SS, EF, HOT><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, HOT ? p->d_col_hot : p->d_col,
+  k_lane<OT, SS, EF, HOT><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col,
                                                         p->d_val, x, y, p->nrows, ss_in,
                                                         p->d_blk_ss, p->d_xh);
 }
 
+}  // namespace
+
+int lane_ef_mode(const spmv_plan_s* p) {
+  return p->opts.evict_first && p->stream_ef ? 1 : 0;
+}
+
+namespace {
+
 template <typename OT, bool SS>
 void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
-  int ef = p->opts.evict_first && p->stream_ef ? 1 : 0;
-  if (const char* e = getenv("SPMV_LANE_EF")) ef = atoi(e);  // dev knob: 0 / 1
-  const int hot = hot_mode(p) == 3 ? 0 : hot_mode(p);
-  if (ef == 1) {
-    if (hot == 2) launch_lane_t<OT, SS, 1, 2>(p, x, y, ss_in, s);
-    else if (hot == 1) launch_lane_t<OT, SS, 1, 1>(p, x, y, ss_in, s);
-    else launch_lane_t<OT, SS, 1, 0>(p, x, y, ss_in, s);
-  } else {
-    if (hot == 2) launch_lane_t<OT, SS, 0, 2>(p, x, y, ss_in, s);
-    else if (hot == 1) launch_lane_t<OT, SS, 0, 1>(p, x, y, ss_in, s);
-    else launch_lane_t<OT, SS, 0, 0>(p, x, y, ss_in, s);
-  }
+  // stream policy (plan decision): evict_first on every chunk when no 8-entry
+  // chunk is shared by two rows (1), else none (0); 2 (first chunk of a row
+  // normal, the rest evict_first) via the SPMV_LANE_EF dev knob
+  int ef = lane_ef_mode(p);
+  if (const char* e = getenv("SPMV_LANE_EF")) ef = std::min(2, std::max(0, atoi(e)));  // dev knob
+  if (ef == 1) launch_lane_t<OT, SS, 1, 0>(p, x, y, ss_in, s);
+  else if (ef == 2) launch_lane_t<OT, SS, 2, 0>(p, x, y, ss_in, s);
+  else launch_lane_t<OT, SS, 0, 0>(p, x, y, ss_in, s);
 }
 
 // Row-class kernels other than the short-row one.  HOT 1/2: every gather
