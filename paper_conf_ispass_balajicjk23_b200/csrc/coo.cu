@@ -222,8 +222,8 @@ __global__ void __launch_bounds__(CO_THREADS)
 constexpr int CW_E = 16;
 constexpr int CW_TILE = 32 * CW_E;
 
-template <int EF>
-__global__ void __launch_bounds__(256)
+template <int EF, int MINB>
+__global__ void __launch_bounds__(256, MINB)
     k_coo_w(const int32_t* __restrict__ row, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
             int64_t nnz, int64_t nrows, int64_t ntiles, int32_t* __restrict__ t_frow,
@@ -437,12 +437,12 @@ void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s) {
                                         p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
   } else {
     const unsigned g = (unsigned)std::min<int64_t>((T + 7) / 8, (int64_t)sms(p->device) * 16);
-    if (ef)
-      k_coo_w<1><<<g, 256, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
-                                   p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
-    else
-      k_coo_w<0><<<g, 256, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local,
-                                   p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
+    int minb = 3;  // <= 85 registers: 3 CTAs (24 warps) per SM
+    if (const char* e = getenv("SPMV_COO_MINB")) minb = atoi(e) >= 4 ? 4 : 3;  // dev knob
+    auto k = ef ? (minb == 4 ? k_coo_w<1, 4> : k_coo_w<1, 3>)
+                : (minb == 4 ? k_coo_w<0, 4> : k_coo_w<0, 3>);
+    k<<<g, 256, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local, p->nrows, T, frow,
+                        lrow, fpart, lpart, p->d_coo_tflag);
   }
   k_coo_fix<<<(unsigned)((T + 255) / 256), 256, 0, s>>>(T, frow, lrow, fpart, lpart,
                                                         p->d_coo_tflag, y);
