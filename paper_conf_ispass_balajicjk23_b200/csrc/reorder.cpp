@@ -65,17 +65,26 @@ Sym symmetrize(int64_t n, const int64_t* rp, const int32_t* col) {
     std::sort(b, b + m);
     bl[i] = std::unique(b, b + m) - b;
   }
-  // transpose counts
+  // transpose: parallel counts and scatter with atomic cursors, then each
+  // transposed row sorted (the result is the same as a sequential transpose)
   std::vector<int64_t> tcnt(n + 1, 0);
+#pragma omp parallel for schedule(dynamic, 1024)
   for (int64_t i = 0; i < n; ++i)
-    for (int64_t k = 0; k < bl[i]; ++k) tcnt[bidx[rp[i] + k]]++;
+    for (int64_t k = 0; k < bl[i]; ++k)
+      __atomic_fetch_add(&tcnt[bidx[rp[i] + k]], (int64_t)1, __ATOMIC_RELAXED);
   std::vector<int64_t> tptr(tcnt);
   scan_inplace(tptr);
   std::vector<int32_t> tidx((size_t)tptr[n]);
   {
     std::vector<int64_t> cur(tptr.begin(), tptr.end() - 1);
-    for (int64_t i = 0; i < n; ++i)  // rows ascending -> transposed rows sorted
-      for (int64_t k = 0; k < bl[i]; ++k) tidx[cur[bidx[rp[i] + k]]++] = (int32_t)i;
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t i = 0; i < n; ++i)
+      for (int64_t k = 0; k < bl[i]; ++k) {
+        const int64_t pos = __atomic_fetch_add(&cur[bidx[rp[i] + k]], (int64_t)1, __ATOMIC_RELAXED);
+        tidx[pos] = (int32_t)i;
+      }
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t j = 0; j < n; ++j) std::sort(tidx.begin() + tptr[j], tidx.begin() + tptr[j + 1]);
   }
   // merge row i of Bp and Bp^T
   Sym S;
@@ -294,16 +303,19 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
       spmv::set_error("spmv_reorder: row_ptr inconsistent with nnz");
       return SPMV_EINVAL;
     }
-    for (int64_t i = 0; i < n; ++i)
-      if (rp[i + 1] < rp[i]) {
-        spmv::set_error("spmv_reorder: row_ptr not monotone");
-        return SPMV_EINVAL;
-      }
-    for (int64_t k = 0; k < nnz; ++k)
-      if (col[k] < 0 || col[k] >= n) {
-        spmv::set_error("spmv_reorder: column out of range");
-        return SPMV_EINVAL;
-      }
+    int64_t bad_rp = 0, bad_col = 0;
+#pragma omp parallel for schedule(static) reduction(+ : bad_rp)
+    for (int64_t i = 0; i < n; ++i) bad_rp += rp[i + 1] < rp[i];
+    if (bad_rp) {
+      spmv::set_error("spmv_reorder: row_ptr not monotone");
+      return SPMV_EINVAL;
+    }
+#pragma omp parallel for schedule(static) reduction(+ : bad_col)
+    for (int64_t k = 0; k < nnz; ++k) bad_col += col[k] < 0 || col[k] >= n;
+    if (bad_col) {
+      spmv::set_error("spmv_reorder: column out of range");
+      return SPMV_EINVAL;
+    }
     auto tp = std::chrono::steady_clock::now();
     phase("validate", tp);
     spmv_reorder_stats_t S0;
@@ -322,12 +334,16 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
     }
     // in-degree (column counts, diagonal and duplicates included: reading c13)
     std::vector<int64_t> colcnt(n, 0);
-    for (int64_t k = 0; k < nnz; ++k) colcnt[col[k]]++;
+#pragma omp parallel for schedule(static)
+    for (int64_t k = 0; k < nnz; ++k) __atomic_fetch_add(&colcnt[col[k]], (int64_t)1, __ATOMIC_RELAXED);
     std::vector<uint8_t> hub(n);
+    int64_t nh = 0;
+#pragma omp parallel for schedule(static) reduction(+ : nh)
     for (int64_t v = 0; v < n; ++v) {
       hub[v] = (__int128)colcnt[v] * n > (__int128)nnz;
-      S0.n_hubs += hub[v];
+      nh += hub[v];
     }
+    S0.n_hubs = nh;
     phase("skew+colcnt", tp);
 
     if (method == SPMV_ORDER_ORIGINAL) {
@@ -367,14 +383,28 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
         // modularity Q' = sum_c (2m in_c - tot_c^2) and insular flags
         g_cache.ins.assign(n, 1);
         {
+          // per-vertex sums in parallel, per-community accumulation in order
+          std::vector<int64_t> vin(n), vtot(n);
+          uint8_t* insp = g_cache.ins.data();  // g_cache is thread_local: no access in the region
+          const Rabbit& Rr = R;
+#pragma omp parallel for schedule(dynamic, 4096)
+          for (int64_t v = 0; v < n; ++v) {
+            const int32_t c = Rr.comm[v];
+            int64_t a = 0, t = 0;
+            uint8_t ins = 1;
+            for (int64_t k = S.ptr[v]; k < S.ptr[v + 1]; ++k) {
+              t += S.w[k];
+              if (Rr.comm[S.idx[k]] == c) a += S.w[k];
+              else ins = 0;
+            }
+            vin[v] = a;
+            vtot[v] = t;
+            insp[v] = ins;
+          }
           std::vector<__int128> inc(n, 0), totc(n, 0);
           for (int64_t v = 0; v < n; ++v) {
-            int32_t c = R.comm[v];
-            for (int64_t k = S.ptr[v]; k < S.ptr[v + 1]; ++k) {
-              totc[c] += S.w[k];
-              if (R.comm[S.idx[k]] == c) inc[c] += S.w[k];
-              else g_cache.ins[v] = 0;
-            }
+            inc[R.comm[v]] += vin[v];
+            totc[R.comm[v]] += vtot[v];
           }
           __int128 q = 0;
           for (int64_t c = 0; c < n; ++c)
