@@ -1,5 +1,6 @@
 // extern "C" entry points of include/spmv.h: argument checks, error
 // translation (no exception crosses the ABI), thread-local last error.
+#include <algorithm>
 #include <cstring>
 #include <string>
 
@@ -149,6 +150,63 @@ spmv_status spmv_exec_coo(spmv_plan_t p, const float* x_B, float* y_B, void* str
   if (p->nrows && (!x_B || !y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_coo: NULL vector");
   use_device(p);
   spmv::exec_coo(p, x_B, y_B, S(stream));
+  API_END
+}
+
+spmv_status spmv_exec_scaled_bcast(spmv_plan_t p, const float* x_B, float* const* x_next,
+                                   int n_next, const double* sumsq_in, double* sumsq_out,
+                                   void* stream) {
+  API_BEGIN
+  if (!p || !x_next) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled_bcast: NULL argument");
+  if (p->nrows && !x_B) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled_bcast: NULL vector");
+  if (n_next < 1 || n_next > 8 || n_next > p->world)
+    SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled_bcast: n_next must be in [1, min(world, 8)]");
+  use_device(p);
+  spmv::exec(p, x_B, nullptr, sumsq_in, sumsq_out, S(stream), x_next, n_next);
+  API_END
+}
+
+spmv_status spmv_dev_alloc(int device, int64_t bytes, void** dev_ptr) {
+  API_BEGIN
+  if (!dev_ptr || bytes < 0) SPMV_FAIL(SPMV_EINVAL, "spmv_dev_alloc: bad argument");
+  *dev_ptr = nullptr;
+  SPMV_CUDA(cudaSetDevice(device));
+  if (cudaMalloc(dev_ptr, (size_t)std::max<int64_t>(bytes, 256)) != cudaSuccess) {
+    cudaGetLastError();
+    SPMV_FAIL(SPMV_ENOMEM, "spmv_dev_alloc: cudaMalloc failed");
+  }
+  API_END
+}
+
+spmv_status spmv_dev_free(void* dev_ptr) {
+  API_BEGIN
+  if (dev_ptr) SPMV_CUDA(cudaFree(dev_ptr));
+  API_END
+}
+
+spmv_status spmv_ipc_handle(const void* dev_ptr, void* handle) {
+  API_BEGIN
+  if (!dev_ptr || !handle) SPMV_FAIL(SPMV_EINVAL, "spmv_ipc_handle: NULL argument");
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "64-byte IPC handle");
+  cudaIpcMemHandle_t h;
+  SPMV_CUDA(cudaIpcGetMemHandle(&h, const_cast<void*>(dev_ptr)));
+  std::memcpy(handle, &h, 64);
+  API_END
+}
+
+spmv_status spmv_ipc_open(const void* handle, void** dev_ptr) {
+  API_BEGIN
+  if (!handle || !dev_ptr) SPMV_FAIL(SPMV_EINVAL, "spmv_ipc_open: NULL argument");
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, 64);
+  SPMV_CUDA(cudaIpcOpenMemHandle(dev_ptr, h, cudaIpcMemLazyEnablePeerAccess));
+  API_END
+}
+
+spmv_status spmv_ipc_close(void* dev_ptr) {
+  API_BEGIN
+  if (!dev_ptr) SPMV_FAIL(SPMV_EINVAL, "spmv_ipc_close: NULL argument");
+  SPMV_CUDA(cudaIpcCloseMemHandle(dev_ptr));
   API_END
 }
 

@@ -87,6 +87,34 @@ __device__ __forceinline__ float alpha_of(const double* ss_in) {
   return v > 0.0 ? (float)(1.0 / sqrt(v)) : 1.f;
 }
 
+// Fused exchange (spmv_exec_scaled_bcast): the scaled y of a
+// row is stored straight into the next-x buffer of every rank (NVLink peer
+// stores through CUDA IPC mappings) instead of a local y + NCCL all-gather.
+// Only the exec_scaled (SS) instantiations look at it.
+struct YDst {
+  float* p[8];  // next-x buffers of ranks 0..n-1, each already offset by y_offset
+  int n;        // 0: plain local y
+};
+
+template <bool SS>
+__device__ __forceinline__ void store_y(float* __restrict__ y, const YDst& d, int64_t r, float v) {
+  if constexpr (SS) {
+    if (d.n) {
+#pragma unroll 1
+      for (int k = 0; k < d.n; ++k) d.p[k][r] = v;
+      return;
+    }
+  }
+  y[r] = v;
+}
+
+template <bool SS>
+__device__ __forceinline__ void fence_bcast(const YDst& d) {
+  if constexpr (SS) {
+    if (d.n) __threadfence_system();  // peer stores visible before the caller's collective
+  }
+}
+
 __device__ __forceinline__ float warp_tree(float s) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
@@ -391,7 +419,7 @@ __global__ void __launch_bounds__(256)
                 const float* __restrict__ val, const float* __restrict__ x,
                 float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
                 const double* __restrict__ ss_in, double* __restrict__ row_ss,
-                const float* __restrict__ xh) {
+                const float* __restrict__ xh, const YDst dst) {
   const int lane = threadIdx.x & 31;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float alpha = alpha_of(ss_in);
@@ -419,10 +447,11 @@ __global__ void __launch_bounds__(256)
     s = warp_tree(s);
     if (lane == 0) {
       const float v = __fmul_rn(s, alpha);
-      y[r] = v;
+      store_y<SS>(y, dst, r, v);
       if (SS) row_ss[q] = (double)v * (double)v;
     }
   }
+  fence_bcast<SS>(dst);
 }
 
 // k_warp_rows with the hot-column set in shared memory (hot mode 3): one
@@ -513,15 +542,16 @@ __global__ void __launch_bounds__(256)
     k_cta_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
                const int32_t* __restrict__ rows, const double* __restrict__ ss_in,
-               double* __restrict__ row_ss, const float* __restrict__ xh) {
+               double* __restrict__ row_ss, const float* __restrict__ xh, const YDst dst) {
   __shared__ float red[256];
   const int r = rows[blockIdx.x];
   const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
   const float s = cta_sum256<HOT>(col, val, x, b, L, red, xh);
   if (threadIdx.x == 0) {
     const float v = __fmul_rn(s, alpha_of(ss_in));
-    y[r] = v;
+    store_y<SS>(y, dst, r, v);
     if (SS) row_ss[blockIdx.x] = (double)v * (double)v;
+    fence_bcast<SS>(dst);
   }
 }
 
@@ -620,14 +650,15 @@ template <bool SS>
 __global__ void k_hub_fix(const int32_t* __restrict__ hub_rows, const int32_t* __restrict__ choff,
                           int64_t nh, const double* __restrict__ part,
                           const double* __restrict__ ss_in, float* __restrict__ y,
-                          double* __restrict__ hub_ss) {
+                          double* __restrict__ hub_ss, const YDst dst) {
   const int64_t h = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (h >= nh) return;
   double acc = 0.0;
   for (int c = choff[h]; c < choff[h + 1]; ++c) acc += part[c];
   const float v = __fmul_rn((float)acc, alpha_of(ss_in));
-  y[hub_rows[h]] = v;
+  store_y<SS>(y, dst, hub_rows[h], v);
   if (SS) hub_ss[h] = (double)v * (double)v;
+  fence_bcast<SS>(dst);
 }
 
 __global__ void __launch_bounds__(1024)
@@ -760,7 +791,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
            int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss,
-           const float* __restrict__ xh) {
+           const float* __restrict__ xh, const YDst dst) {
   __shared__ double wss[LN_WARPS];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
@@ -818,7 +849,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
     double ssacc = 0.0;
     if (mine) {
       const float o = __fmul_rn(res, alpha);
-      y[r] = o;
+      store_y<SS>(y, dst, r, o);
       if (SS) ssacc = (double)o * (double)o;
     }
     if (SS) {  // fixed-order per-block sum of y^2 (independent of the grid)
@@ -833,10 +864,12 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
       __syncthreads();
     }
   }
+  fence_bcast<SS>(dst);
 }
 
 template <typename OT, bool SS, int EF, int HOT>
-void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
+void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s,
+                   const YDst& dst) {
   // grid-stride with ~8 CTAs per resident slot (measured better than one
   // persistent wave on SBM, RMAT-26 and the stencil: r29, profiles/)
   int per_sm = LN_CTAS_PER_SM;
@@ -846,7 +879,7 @@ void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
   k_lane<OT, SS, EF, HOT><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col,
                                                         p->d_val, x, y, p->nrows, ss_in,
-                                                        p->d_blk_ss, p->d_xh);
+                                                        p->d_blk_ss, p->d_xh, dst);
 }
 
 }  // namespace
@@ -858,15 +891,16 @@ int lane_ef_mode(const spmv_plan_s* p) {
 namespace {
 
 template <typename OT, bool SS>
-void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
+void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s,
+                 const YDst& dst) {
   // stream policy (plan decision): evict_first on every chunk when no 8-entry
   // chunk is shared by two rows (1), else none (0); 2 (first chunk of a row
   // normal, the rest evict_first) via the SPMV_LANE_EF dev knob
   int ef = lane_ef_mode(p);
   if (const char* e = getenv("SPMV_LANE_EF")) ef = std::min(2, std::max(0, atoi(e)));  // dev knob
-  if (ef == 1) launch_lane_t<OT, SS, 1, 0>(p, x, y, ss_in, s);
-  else if (ef == 2) launch_lane_t<OT, SS, 2, 0>(p, x, y, ss_in, s);
-  else launch_lane_t<OT, SS, 0, 0>(p, x, y, ss_in, s);
+  if (ef == 1) launch_lane_t<OT, SS, 1, 0>(p, x, y, ss_in, s, dst);
+  else if (ef == 2) launch_lane_t<OT, SS, 2, 0>(p, x, y, ss_in, s, dst);
+  else launch_lane_t<OT, SS, 0, 0>(p, x, y, ss_in, s, dst);
 }
 
 // Row-class kernels other than the short-row one.  HOT 1/2: every gather
@@ -874,7 +908,7 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
 // in shared memory), the CTA / hub classes read the plain columns.
 template <typename OT, bool SS, int HOT>
 void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s1,
-                 cudaStream_t s2, bool lane_mode) {
+                 cudaStream_t s2, bool lane_mode, const YDst& dst) {
   constexpr int HG = HOT == 3 ? 0 : HOT;  // gather variant of the CTA / hub (and MID) kernels
   const OT* rp = (const OT*)p->d_rp;
   const int32_t* col = HG ? p->d_col_hot : p->d_col;
@@ -894,7 +928,8 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
         rp, p->d_col_hot, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh, (int)p->hot_S);
   } else if (nw) {
     const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
-    k_warp_rows<OT, SS, HG><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh);
+    k_warp_rows<OT, SS, HG><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh,
+                                               dst);
   }
   const bool long_smem = HOT == 3 && (p->n_cta || p->n_chunks);
   if (long_smem) {
@@ -915,7 +950,7 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   } else if (p->n_cta) {
     k_cta_rows<OT, SS, HG><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
                                                                p->d_cta_rows, ss_in, p->d_cta_ss,
-                                                               p->d_xh);
+                                                               p->d_xh, dst);
   }
   if (p->n_chunks) {
     if (!long_smem)
@@ -925,16 +960,16 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
     const unsigned g = (unsigned)((p->n_hub + 127) / 128);
     if (SS)
       k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
-                                         ss_in, y, p->d_hub_ss);
+                                         ss_in, y, p->d_hub_ss, dst);
     else
       k_hub_fix<false><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub,
-                                          p->d_chunk_part, ss_in, y, p->d_hub_ss);
+                                          p->d_chunk_part, ss_in, y, p->d_hub_ss, dst);
   }
 }
 
 template <typename OT>
 void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
-                cudaStream_t s) {
+                cudaStream_t s, const YDst& dst) {
   const bool SS = ss_out != nullptr;
   const bool lane_mode = p->opts.variant != 1;
   if (lane_mode && hot_mode(p)) {  // refresh the hot copy of x for this exec
@@ -961,8 +996,8 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   if (conc && early) fork();
   if (lane_mode) {
     if (p->nrows) {
-      if (SS) launch_lane<OT, true>(p, x, y, ss_in, s);
-      else launch_lane<OT, false>(p, x, y, ss_in, s);
+      if (SS) launch_lane<OT, true>(p, x, y, ss_in, s, dst);
+      else launch_lane<OT, false>(p, x, y, ss_in, s, dst);
     }
   } else if (p->K) {
     if (SS) launch_panel<OT, true>(p, x, y, ss_in, s);
@@ -972,15 +1007,15 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   {
     const int hot = lane_mode ? hot_mode(p) : 0;
     if (SS) {
-      if (hot == 3) launch_rows<OT, true, 3>(p, x, y, ss_in, s1, s2, lane_mode);
-      else if (hot == 2) launch_rows<OT, true, 2>(p, x, y, ss_in, s1, s2, lane_mode);
-      else if (hot == 1) launch_rows<OT, true, 1>(p, x, y, ss_in, s1, s2, lane_mode);
-      else launch_rows<OT, true, 0>(p, x, y, ss_in, s1, s2, lane_mode);
+      if (hot == 3) launch_rows<OT, true, 3>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+      else if (hot == 2) launch_rows<OT, true, 2>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+      else if (hot == 1) launch_rows<OT, true, 1>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+      else launch_rows<OT, true, 0>(p, x, y, ss_in, s1, s2, lane_mode, dst);
     } else {
-      if (hot == 3) launch_rows<OT, false, 3>(p, x, y, ss_in, s1, s2, lane_mode);
-      else if (hot == 2) launch_rows<OT, false, 2>(p, x, y, ss_in, s1, s2, lane_mode);
-      else if (hot == 1) launch_rows<OT, false, 1>(p, x, y, ss_in, s1, s2, lane_mode);
-      else launch_rows<OT, false, 0>(p, x, y, ss_in, s1, s2, lane_mode);
+      if (hot == 3) launch_rows<OT, false, 3>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+      else if (hot == 2) launch_rows<OT, false, 2>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+      else if (hot == 1) launch_rows<OT, false, 1>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+      else launch_rows<OT, false, 0>(p, x, y, ss_in, s1, s2, lane_mode, dst);
     }
   }
   if (conc) {
@@ -1082,13 +1117,25 @@ int exec_launches(const spmv_plan_s* p, bool ss) {
 }
 
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
-          cudaStream_t s) {
+          cudaStream_t s, float* const* bcast, int nbcast) {
   if (!p->permuted) SPMV_FAIL(SPMV_ESTATE, "spmv_exec before spmv_permute");
   if (ss_in && ss_in == ss_out) SPMV_FAIL(SPMV_EINVAL, "sumsq_in and sumsq_out alias");
+  YDst dst{};
+  if (nbcast) {
+    if (nbcast < 0 || nbcast > 8) SPMV_FAIL(SPMV_EINVAL, "bcast: 1..8 destination buffers");
+    if (!ss_out) SPMV_FAIL(SPMV_EINVAL, "bcast needs sumsq_out (exec_scaled)");
+    if (p->opts.variant == 1 || hot_mode(p))
+      SPMV_FAIL(SPMV_EUNSUPPORTED, "bcast: lane-mode kernels without the hot-column set only");
+    for (int k = 0; k < nbcast; ++k) {
+      if (!bcast[k]) SPMV_FAIL(SPMV_EINVAL, "bcast: NULL destination");
+      dst.p[k] = bcast[k] + p->y_offset;
+    }
+    dst.n = nbcast;
+  }
   ensure_aux(p);
   set_window(p, x, s);
-  if (p->off64) exec_typed<int64_t>(p, x, y, ss_in, ss_out, s);
-  else exec_typed<int32_t>(p, x, y, ss_in, ss_out, s);
+  if (p->off64) exec_typed<int64_t>(p, x, y, ss_in, ss_out, s, dst);
+  else exec_typed<int32_t>(p, x, y, ss_in, ss_out, s, dst);
 }
 
 void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s) {

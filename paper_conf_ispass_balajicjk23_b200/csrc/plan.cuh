@@ -113,7 +113,7 @@ void plan_free(spmv_plan_s* p);
 void permute_vec(spmv_plan_s* p, const float* in, float* out, int inverse, cudaStream_t s);
 void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStream_t s);
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
-          cudaStream_t s);
+          cudaStream_t s, float* const* bcast = nullptr, int nbcast = 0);
 void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s);
 int exec_launches(const spmv_plan_s* p, bool ss);
 void exec_spmm4(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s);

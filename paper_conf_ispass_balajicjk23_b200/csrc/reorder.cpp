@@ -180,10 +180,29 @@ Rabbit rabbit_detect(const Sym& S) {
       if (acc[r] == 0) touched.push_back(r);
       acc[r] += wt;
     };
-    for (int64_t k = S.ptr[u]; k < S.ptr[u + 1]; ++k) add(S.idx[k], S.w[k]);
+    // the loop is memory-latency bound (random parent / acc accesses):
+    // prefetch the union-find entry of a neighbour PF iterations ahead
+    constexpr int PF = 16;
+    {
+      const int64_t k0 = S.ptr[u], k1 = S.ptr[u + 1];
+      for (int64_t k = k0; k < k1; ++k) {
+        if (k + PF < k1) __builtin_prefetch(&parent[S.idx[k + PF]]);
+        add(S.idx[k], S.w[k]);
+      }
+    }
     for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) {
-      for (const Edge& e : agg[c]) add(e.v, e.w);
+      const std::vector<Edge>& L = agg[c];
+      const size_t m = L.size();
+      for (size_t i = 0; i < m; ++i) {
+        if (i + PF < m) __builtin_prefetch(&parent[L[i + PF].v]);
+        add(L[i].v, L[i].w);
+      }
       std::vector<Edge>().swap(agg[c]);
+    }
+    if (oi + 1 < n) {  // next vertex's row and union-find entry
+      const int32_t un = (int32_t)order[oi + 1];
+      __builtin_prefetch(&S.idx[S.ptr[un]]);
+      __builtin_prefetch(&first_child[un]);
     }
     int32_t best = -1;
     __int128 bestdq = 0;

@@ -1,4 +1,4 @@
-"""Row-block power iteration across ranks (SURVEY.md §8(e); reading c22).
+"""Row-block power iteration across ranks (SURVEY.md §8(e), §8(f1); reading c22).
 
 One process per GPU.  Rank k owns rows [b_k, b_{k+1}) of B (nnz-balanced
 partition computed by spmv_plan), a full replica of x in the padded layout
@@ -47,6 +47,69 @@ def iterate(local, x, iters: int, group=None):
         xa, xb = xb, xa
     local.scale(xa, xa, ss_in)
     return xa, math.sqrt(float(ss_in.item()))
+
+
+def _all_reduce_sum(t, group, host_staged):
+    import torch.distributed as dist
+    if host_staged:  # gloo: stage through the host (this also syncs the stream)
+        h = t.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+        t.copy_(h)
+    else:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+
+
+def iterate_fused(plan, x, iters: int, group=None, host_staged: bool = False):
+    """The same iteration with the exchange fused into the SpMV:
+    every rank maps every other rank's two next-x buffers (CUDA IPC over
+    NVLink / NVSwitch), and spmv_exec_scaled_bcast stores each y row straight
+    into all of them -- no all-gather.  Per iteration one collective remains,
+    the 8-byte all-reduce of sum y^2, which also orders every rank's next read
+    after all ranks' stores (and the previous read before the next stores:
+    a rank passes the all-reduce of step t only after every rank's step-t
+    kernels have completed).  Returns (x_iters, lambda) like iterate()."""
+    import torch
+    import torch.distributed as dist
+    from . import spmv
+
+    if iters < 1:
+        raise ValueError("iters must be >= 1")
+    i = plan.info()
+    world, rank, xlen = i["world"], i["rank"], i["x_len"]
+    dev = x.device
+    bufs = [spmv.DeviceBuffer(xlen, dev.index if dev.index is not None else 0) for _ in range(2)]
+    opened = []
+    try:
+        mine = [b.handle() for b in bufs]
+        allh = [None] * world
+        dist.all_gather_object(allh, mine, group=group)
+        dst = [[0] * world for _ in range(2)]
+        for k in range(world):
+            for j in range(2):
+                if k == rank:
+                    dst[j][k] = bufs[j].ptr
+                else:
+                    dst[j][k] = spmv.ipc_open(allh[k][j])
+                    opened.append(dst[j][k])
+        bufs[0].tensor.copy_(x)
+        ss = torch.zeros(2, dtype=torch.float64, device=dev)
+        ss_in, cur = None, 0
+        for t in range(iters):
+            ss_out = ss[t & 1:(t & 1) + 1]
+            plan.exec_scaled_bcast(bufs[cur].tensor, dst[1 - cur], ss_in, ss_out)
+            _all_reduce_sum(ss_out, group, host_staged)
+            ss_in, cur = ss_out, 1 - cur
+        out = torch.empty_like(x)
+        spmv.scale_vec(bufs[cur].tensor, out, ss_in)
+        lam = math.sqrt(float(ss_in.item()))
+        torch.cuda.synchronize(dev)
+        dist.barrier(group=group)  # nobody unmaps while a peer may still store
+    finally:
+        for q in opened:
+            spmv.ipc_close(q)
+        for b in bufs:
+            b.close()
+    return out, lam
 
 
 class PlanLocal:

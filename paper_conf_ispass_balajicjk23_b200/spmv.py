@@ -85,6 +85,12 @@ def lib() -> ctypes.CDLL:
             "spmv_exec_scaled": (i32, [vp, vp, vp, dp, dp, vp]),
             "spmv_exec_spmm4": (i32, [vp, vp, vp, vp]),
             "spmv_exec_coo": (i32, [vp, vp, vp, vp]),
+            "spmv_exec_scaled_bcast": (i32, [vp, vp, vp, i32, dp, dp, vp]),
+            "spmv_ipc_handle": (i32, [vp, vp]),
+            "spmv_dev_alloc": (i32, [i32, i64, ctypes.POINTER(vp)]),
+            "spmv_dev_free": (i32, [vp]),
+            "spmv_ipc_open": (i32, [vp, ctypes.POINTER(vp)]),
+            "spmv_ipc_close": (i32, [vp]),
             "spmv_export_coo_rows": (i32, [vp, vp, vp]),
             "spmv_iterate": (i32, [vp, vp, i32, ctypes.POINTER(ctypes.c_double), vp]),
             "spmv_scale_vec": (i32, [vp, vp, i64, dp, vp]),
@@ -231,6 +237,13 @@ class Plan:
         _check(lib().spmv_exec_spmm4(self._h, _ptr(X), _ptr(Y), _stream_ptr(stream)))
         return Y
 
+    def exec_scaled_bcast(self, x, x_next_ptrs, sumsq_in, sumsq_out, stream=None):
+        """Fused exec + exchange: rows scaled as exec_scaled, stored into every
+        buffer of x_next_ptrs (device addresses, padded x layout)."""
+        arr = (ctypes.c_void_p * len(x_next_ptrs))(*[int(a) for a in x_next_ptrs])
+        _check(lib().spmv_exec_scaled_bcast(self._h, _ptr(x), arr, len(x_next_ptrs),
+                                            _ptr(sumsq_in), _ptr(sumsq_out), _stream_ptr(stream)))
+
     def exec_scaled(self, x, y, sumsq_in=None, sumsq_out=None, stream=None):
         _check(lib().spmv_exec_scaled(self._h, _ptr(x), _ptr(y), _ptr(sumsq_in), _ptr(sumsq_out),
                                       _stream_ptr(stream)))
@@ -333,3 +346,38 @@ def reorder_last_comm(n: int) -> np.ndarray:
     out = np.empty(n, np.int32)
     _check(lib().spmv_reorder_last_comm(n, out.ctypes.data))
     return out
+
+
+class DeviceBuffer:
+    """fp32 device buffer from spmv_dev_alloc (a standalone cudaMalloc, so its
+    CUDA IPC handle names exactly this buffer); .tensor views it as torch."""
+
+    def __init__(self, n: int, device: int):
+        import torch
+        p = ctypes.c_void_p()
+        _check(lib().spmv_dev_alloc(int(device), 4 * int(n), ctypes.byref(p)))
+        self.ptr, self.n = int(p.value), int(n)
+        self.__cuda_array_interface__ = {"shape": (self.n,), "typestr": "<f4",
+                                         "data": (self.ptr, False), "version": 3}
+        self.tensor = torch.as_tensor(self, device=torch.device("cuda", int(device)))
+
+    def handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(64)
+        _check(lib().spmv_ipc_handle(ctypes.c_void_p(self.ptr), buf))
+        return buf.raw
+
+    def close(self):
+        if self.ptr:
+            self.tensor = None
+            lib().spmv_dev_free(ctypes.c_void_p(self.ptr))
+            self.ptr = 0
+
+
+def ipc_open(handle: bytes) -> int:
+    p = ctypes.c_void_p()
+    _check(lib().spmv_ipc_open(ctypes.create_string_buffer(handle, 64), ctypes.byref(p)))
+    return int(p.value)
+
+
+def ipc_close(ptr: int) -> None:
+    _check(lib().spmv_ipc_close(ctypes.c_void_p(ptr)))
