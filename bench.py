@@ -192,6 +192,7 @@ def run_gpu(args):
         ideal_p96 = 2 * A.n * 4 + (A.n + 1 + 2 * A.nnz) * 4
         launches = info["exec_launches"]
         is_main = ordering == main
+        fx = None
         K = args.steps if is_main else max(10, args.steps // 4)
         if world == 1:
             y = torch.empty(A.n, dtype=torch.float32, device=dev)
@@ -205,9 +206,18 @@ def run_gpu(args):
             state = {"t": 0, "xa": xa, "xb": xb, "ss_in": None}
             M, off, nr = loc.x_stride, loc.y_offset, loc.nrows
 
+            if args.exchange == "fused":  # y rows stored into every peer's x
+                fx = pdist.FusedExchange(P, dev, host_staged=args.backend != "nccl")
+                fx.x.copy_(xB)
+
             def step():
                 t = state["t"]
                 ss_out = ss[t & 1:(t & 1) + 1]
+                if fx is not None:
+                    fx.step(state["ss_in"], ss_out)
+                    state["ss_in"] = ss_out
+                    state["t"] = t + 1
+                    return
                 P.exec_scaled(state["xa"], state["xb"][off:off + nr], state["ss_in"], ss_out)
                 if args.backend == "nccl":
                     dist.all_reduce(ss_out)
@@ -307,6 +317,7 @@ def run_gpu(args):
             if world == 1:
                 e2e = e2e_measure(P, A, w.x, args, dev, ideal)
             else:
+                state["xcur"] = (lambda: fx.x) if fx is not None else (lambda: state["xa"])
                 e2e = e2e_dist_measure(P, loc, w.x, perm, step_state=state, step=step, args=args,
                                        dev=dev, ideal=ideal, world=world)
             line = dict(metric=METRIC, value=round(gbs, 2), unit="GB/s", n_gpus=world, steps=K,
@@ -317,7 +328,9 @@ def run_gpu(args):
                               "n": A.n, "nnz": A.nnz, "ordering": ordering,
                               "parallelism": f"row-block x{world}" if world > 1 else "1 GPU",
                               "step": "spmv_exec" if world == 1 else
-                              "exec_scaled + all_reduce + all_gather (power iteration)",
+                              ("exec_scaled_bcast (fused NVLink peer stores) + all_reduce (power iteration)"
+                                       if args.exchange == "fused" else
+                                       "exec_scaled + all_reduce + all_gather (power iteration)"),
                               "l2": "flushed before every step (512 MiB read, outside the events)",
                               "ideal_bytes": ideal, "ideal_bytes_paper_4B_offsets": ideal_p96,
                               "kernel_variant": ["lane", "panel"][args.variant],
@@ -337,6 +350,8 @@ def run_gpu(args):
             line["clocks"] = ck
             line["input_prep"] = {"generate_s": round(gen_s, 3), "reorder_s": round(st.seconds, 3),
                                   "plan_permute_s": round(plan_s, 4)}
+        if fx is not None:
+            fx.close()
         P.close()
     line["orderings"] = {k: {kk: (round(vv, 5) if isinstance(vv, float) else vv)
                              for kk, vv in v.items()} for k, v in results.items()}
@@ -446,7 +461,7 @@ def e2e_dist_measure(P, loc, x_host, perm, step_state, step, args, dev, ideal, w
     off = loc.y_offset
 
     def e2e_step():
-        step_state["xa"][off:off + (b1 - b0)].copy_(xs, non_blocking=True)
+        step_state["xcur"]()[off:off + (b1 - b0)].copy_(xs, non_blocking=True)
         step()
         ssh.copy_(step_state["ss_in"], non_blocking=True)
 
@@ -544,6 +559,8 @@ def main():
     ap.add_argument("--variant", type=int, default=0, help="short-row kernel: 0 lane, 1 panel")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="collectives for N > 1 (gloo: host-staged, test only)")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
+                    help="N > 1: NCCL all-gather of x, or the fused exec + NVLink peer stores")
     ap.add_argument("--single-device", action="store_true",
                     help="test only: put every rank on cuda:0 (with --backend gloo)")
     args = ap.parse_args()

@@ -59,56 +59,85 @@ def _all_reduce_sum(t, group, host_staged):
         dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
 
 
+class FusedExchange:
+    """Peer-mapped ping-pong x buffers for the fused exec + exchange (SURVEY
+    §8(f1)): every rank maps every other rank's two next-x buffers (CUDA IPC
+    over NVLink / NVSwitch), and spmv_exec_scaled_bcast stores each y row
+    straight into all of them -- no all-gather.  One collective remains per
+    step, the 8-byte all-reduce of sum y^2, which also orders the data: a rank
+    passes step t's all-reduce only after every rank's step-t kernels have
+    completed, so the next read sees all peers' stores and no peer overwrites a
+    buffer that is still being read."""
+
+    def __init__(self, plan, device, group=None, host_staged: bool = False):
+        import torch.distributed as dist
+        from . import spmv
+        self._spmv, self.plan, self.group, self.host_staged = spmv, plan, group, host_staged
+        i = plan.info()
+        self.world, self.rank, xlen = i["world"], i["rank"], i["x_len"]
+        idx = device.index if device.index is not None else 0
+        self.bufs = [spmv.DeviceBuffer(xlen, idx) for _ in range(2)]
+        self.opened = []
+        mine = [b.handle() for b in self.bufs]
+        allh = [None] * self.world
+        dist.all_gather_object(allh, mine, group=group)
+        self.dst = [[0] * self.world for _ in range(2)]
+        for k in range(self.world):
+            for j in range(2):
+                if k == self.rank:
+                    self.dst[j][k] = self.bufs[j].ptr
+                else:
+                    self.dst[j][k] = spmv.ipc_open(allh[k][j])
+                    self.opened.append(self.dst[j][k])
+        self.cur = 0
+
+    @property
+    def x(self):
+        """The current x (padded layout) -- the buffer the next step reads."""
+        return self.bufs[self.cur].tensor
+
+    def step(self, ss_in, ss_out):
+        """x <- B x / s (fused store into every rank's next buffer), then the
+        all-reduce of ss_out; flips the ping-pong."""
+        self.plan.exec_scaled_bcast(self.x, self.dst[1 - self.cur], ss_in, ss_out)
+        _all_reduce_sum(ss_out, self.group, self.host_staged)
+        self.cur = 1 - self.cur
+
+    def close(self):
+        import torch
+        import torch.distributed as dist
+        if self.bufs is None:
+            return
+        torch.cuda.synchronize()
+        dist.barrier(group=self.group)  # nobody unmaps while a peer may still store
+        for q in self.opened:
+            self._spmv.ipc_close(q)
+        for b in self.bufs:
+            b.close()
+        self.bufs = None
+
+
 def iterate_fused(plan, x, iters: int, group=None, host_staged: bool = False):
-    """The same iteration with the exchange fused into the SpMV:
-    every rank maps every other rank's two next-x buffers (CUDA IPC over
-    NVLink / NVSwitch), and spmv_exec_scaled_bcast stores each y row straight
-    into all of them -- no all-gather.  Per iteration one collective remains,
-    the 8-byte all-reduce of sum y^2, which also orders every rank's next read
-    after all ranks' stores (and the previous read before the next stores:
-    a rank passes the all-reduce of step t only after every rank's step-t
-    kernels have completed).  Returns (x_iters, lambda) like iterate()."""
+    """iterate() with the exchange fused into the SpMV (FusedExchange).
+    Returns (x_iters normalised, padded layout; lambda = s_iters)."""
     import torch
-    import torch.distributed as dist
-    from . import spmv
 
     if iters < 1:
         raise ValueError("iters must be >= 1")
-    i = plan.info()
-    world, rank, xlen = i["world"], i["rank"], i["x_len"]
-    dev = x.device
-    bufs = [spmv.DeviceBuffer(xlen, dev.index if dev.index is not None else 0) for _ in range(2)]
-    opened = []
+    fx = FusedExchange(plan, x.device, group, host_staged)
     try:
-        mine = [b.handle() for b in bufs]
-        allh = [None] * world
-        dist.all_gather_object(allh, mine, group=group)
-        dst = [[0] * world for _ in range(2)]
-        for k in range(world):
-            for j in range(2):
-                if k == rank:
-                    dst[j][k] = bufs[j].ptr
-                else:
-                    dst[j][k] = spmv.ipc_open(allh[k][j])
-                    opened.append(dst[j][k])
-        bufs[0].tensor.copy_(x)
-        ss = torch.zeros(2, dtype=torch.float64, device=dev)
-        ss_in, cur = None, 0
+        fx.x.copy_(x)
+        ss = torch.zeros(2, dtype=torch.float64, device=x.device)
+        ss_in = None
         for t in range(iters):
             ss_out = ss[t & 1:(t & 1) + 1]
-            plan.exec_scaled_bcast(bufs[cur].tensor, dst[1 - cur], ss_in, ss_out)
-            _all_reduce_sum(ss_out, group, host_staged)
-            ss_in, cur = ss_out, 1 - cur
+            fx.step(ss_in, ss_out)
+            ss_in = ss_out
         out = torch.empty_like(x)
-        spmv.scale_vec(bufs[cur].tensor, out, ss_in)
+        fx._spmv.scale_vec(fx.x, out, ss_in)
         lam = math.sqrt(float(ss_in.item()))
-        torch.cuda.synchronize(dev)
-        dist.barrier(group=group)  # nobody unmaps while a peer may still store
     finally:
-        for q in opened:
-            spmv.ipc_close(q)
-        for b in bufs:
-            b.close()
+        fx.close()
     return out, lam
 
 
