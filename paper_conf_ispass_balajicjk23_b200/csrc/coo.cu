@@ -18,7 +18,10 @@
 // y is rounded once from fp32 (<= 8 terms) or fp64 pieces, well inside the
 // north-star tolerance.  Empty rows: each gap between consecutive rows (and
 // before the first / after the last entry) is zeroed by the thread holding
-// the entry after it, so y is written exactly once and needs no memset.
+// the entry after it, so y is written exactly once and needs no memset --
+// unless the matrix has a run of more than 32 empty rows (e.g. RABBIT++ puts
+// the isolated vertices last), then y is memset first (4 N bytes) and the
+// variant-2 kernel skips the zeroing.
 #include <algorithm>
 #include <cstdlib>
 
@@ -41,6 +44,20 @@ __global__ void k_coo_rows(const OT* __restrict__ rp, int64_t nrows, int32_t* __
     const int64_t a = (int64_t)rp[r], e = (int64_t)rp[r + 1];
     for (int64_t k = a + lane; k < e; k += 32) row[k] = (int32_t)r;
   }
+}
+
+// a run of more than GAP_MAX empty rows somewhere (or before the first /
+// after the last entry)?  Such gaps are zeroed by a memset instead of by the
+// one thread that holds the entry after them.
+constexpr int GAP_MAX = 32;
+template <typename OT>
+__global__ void k_coo_long_gap(const OT* __restrict__ rp, int64_t nrows, int* __restrict__ flag) {
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r + GAP_MAX < nrows;
+       r += (int64_t)gridDim.x * blockDim.x)
+    if (rp[r] == rp[r + GAP_MAX + 1]) {
+      *flag = 1;
+      return;
+    }
 }
 
 template <int EF>
@@ -222,7 +239,7 @@ __global__ void __launch_bounds__(CO_THREADS)
 constexpr int CW_E = 16;
 constexpr int CW_TILE = 32 * CW_E;
 
-template <int EF, int MINB>
+template <int EF, int MINB, bool ZG>
 __global__ void __launch_bounds__(256, MINB)
     k_coo_w(const int32_t* __restrict__ row, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
@@ -287,7 +304,7 @@ __global__ void __launch_bounds__(256, MINB)
             }
             single = false;
           }
-          zero_rows(y, (int64_t)last + 1, r);
+          if (ZG) zero_rows(y, (int64_t)last + 1, r);
           cur = r;
           run = 0.f;
         }
@@ -295,7 +312,7 @@ __global__ void __launch_bounds__(256, MINB)
         last = r;
       }
     }
-    if (nh > 0 && eb + nh == nnz) zero_rows(y, (int64_t)cur + 1, nrows);
+    if (ZG && nh > 0 && eb + nh == nnz) zero_rows(y, (int64_t)cur + 1, nrows);
     if (single) {
       hrow = cur;
       hsum = run;
@@ -407,6 +424,17 @@ void coo_build(spmv_plan_s* p, cudaStream_t s) {
     else
       k_coo_rows<int32_t><<<g, 256, 0, s>>>((const int32_t*)p->d_rp, p->nrows, p->d_coo_row);
     SPMV_LAUNCH_CHECK();
+    int* dflag = (int*)dmalloc(sizeof(int));
+    SPMV_CUDA(cudaMemsetAsync(dflag, 0, sizeof(int), s));
+    const unsigned gg = (unsigned)std::min<int64_t>((p->nrows + 255) / 256, (int64_t)sms(p->device) * 8);
+    if (p->off64) k_coo_long_gap<int64_t><<<gg, 256, 0, s>>>((const int64_t*)p->d_rp, p->nrows, dflag);
+    else k_coo_long_gap<int32_t><<<gg, 256, 0, s>>>((const int32_t*)p->d_rp, p->nrows, dflag);
+    SPMV_LAUNCH_CHECK();
+    int hflag = 0;
+    SPMV_CUDA(cudaMemcpyAsync(&hflag, dflag, sizeof(int), cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA(cudaStreamSynchronize(s));
+    cudaFree(dflag);
+    p->coo_memset = hflag != 0;
   }
 }
 
@@ -439,8 +467,12 @@ void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s) {
     const unsigned g = (unsigned)std::min<int64_t>((T + 7) / 8, (int64_t)sms(p->device) * 16);
     int minb = 3;  // <= 85 registers: 3 CTAs (24 warps) per SM
     if (const char* e = getenv("SPMV_COO_MINB")) minb = atoi(e) >= 4 ? 4 : 3;  // dev knob
-    auto k = ef ? (minb == 4 ? k_coo_w<1, 4> : k_coo_w<1, 3>)
-                : (minb == 4 ? k_coo_w<0, 4> : k_coo_w<0, 3>);
+    const bool zg = !p->coo_memset;
+    if (!zg) SPMV_CUDA(cudaMemsetAsync(y, 0, sizeof(float) * (size_t)p->nrows, s));
+    auto k = zg ? (ef ? (minb == 4 ? k_coo_w<1, 4, true> : k_coo_w<1, 3, true>)
+                      : (minb == 4 ? k_coo_w<0, 4, true> : k_coo_w<0, 3, true>))
+                : (ef ? (minb == 4 ? k_coo_w<1, 4, false> : k_coo_w<1, 3, false>)
+                      : (minb == 4 ? k_coo_w<0, 4, false> : k_coo_w<0, 3, false>));
     k<<<g, 256, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local, p->nrows, T, frow,
                         lrow, fpart, lpart, p->d_coo_tflag);
   }

@@ -75,6 +75,7 @@ struct spmv_plan_s {
   int32_t* d_coo_trow = nullptr;   // [2 coo_tiles] first / last row of each tile
   double* d_coo_tpart = nullptr;   // [2 coo_tiles] fp64 pieces (first / last row)
   uint8_t* d_coo_tflag = nullptr;  // [coo_tiles]
+  bool coo_memset = false;         // a run of > 32 empty rows: memset y, no in-kernel zeroing
   double* d_tile_ss = nullptr;     // [K]
   double* d_blk_ss = nullptr;      // [ceil(nrows/64)] per-block sumsq (lane variant)
   double* d_warp_ss = nullptr;     // [n_warp]
