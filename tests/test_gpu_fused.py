@@ -4,8 +4,9 @@ dist.iterate_fused) against the single-GPU power iteration.
 Two processes share cuda:0 (CUDA IPC maps the peer's buffers exactly as it
 would across NVLink-connected GPUs; only the link differs), gloo carries the
 8-byte all-reduce and the handle exchange.  The fused iteration must give the
-single-GPU spmv_iterate result bitwise (same kernels, same association; the
-partition never changes y)."""
+single-GPU spmv_iterate result: y rows bitwise (same kernels, same
+association; the partition never changes y), the fp64 norm up
+to its summation order across ranks."""
 import os
 import socket
 
@@ -69,8 +70,12 @@ def test_fused_exchange_equals_single_gpu(tmp_path, cfg):
     ref = x.cpu().numpy()
     for r in range(world):
         d = np.load(tmp_path / f"r{r}.npz")
-        assert np.array_equal(d["x"].view(np.int32), ref.view(np.int32)), f"rank {r}"
-        assert float(d["lam"]) == lam
+        # every y row is bitwise that of the single-GPU exec; the fp64 norm is
+        # summed per rank then all-reduced (another association), so s_t can
+        # differ in its last bits, and x = fp32(u / s) by at most one ulp
+        err = np.abs(d["x"].astype(np.float64) - ref.astype(np.float64))
+        assert np.all(err <= 2.0 ** -23 * np.abs(ref.astype(np.float64))), f"rank {r}"
+        assert abs(float(d["lam"]) - lam) <= 1e-12 * lam
     P.close()
 
 
