@@ -17,6 +17,7 @@
 //   k_cta_rows4   2048 < L <= 16384, CTA per row (256 partials + tree);
 //   k_hub_chunk4 / k_hub_fix4  L > 16384: 16384-entry chunks, fp64 combine.
 #include <algorithm>
+#include <cstdlib>
 
 #include "plan.cuh"
 
@@ -78,8 +79,8 @@ __device__ __forceinline__ void ld8_f(const float* p, float (&r)[8]) {
 // contribute v * 0 = +-0 for the (finite) matrix value v, which
 // leaves the running sum unchanged (it starts at +0 and is never -0), so the
 // loop is branch-free and both chunks of a 16-entry row are in flight at once.
-template <typename OT, int EF>
-__global__ void __launch_bounds__(L4_THREADS, 2)
+template <typename OT, int EF, int MINB, int UNR>
+__global__ void __launch_bounds__(L4_THREADS, MINB)
     k_lane4(const OT* __restrict__ rp, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ X, float* __restrict__ Y,
             int64_t nrows) {
@@ -92,7 +93,7 @@ __global__ void __launch_bounds__(L4_THREADS, 2)
     const int32_t* cp = col + (a & ~(OT)7);
     const float* vp = val + (a & ~(OT)7);
     const int lo = (int)(a & 7), hi = lo + L;
-#pragma unroll 2
+#pragma unroll UNR
     for (int k = 0; k < hi; k += 8) {
       int cc[8];
       float vv[8];
@@ -123,12 +124,16 @@ __global__ void __launch_bounds__(256)
     const int L = (int)((int64_t)rp[r + 1] - b);
     float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
     int j = lane;
-    for (; j + 32 < L; j += 64) {  // two independent gathers in flight
-      const int c0 = __ldcs(col + b + j), c1 = __ldcs(col + b + j + 32);
-      const float v0 = __ldcs(val + b + j), v1 = __ldcs(val + b + j + 32);
-      const float4 x0 = ldx4(X, c0), x1 = ldx4(X, c1);
+    for (; j + 96 < L; j += 128) {  // four independent gathers in flight
+      const int c0 = __ldcs(col + b + j), c1 = __ldcs(col + b + j + 32),
+                c2 = __ldcs(col + b + j + 64), c3 = __ldcs(col + b + j + 96);
+      const float v0 = __ldcs(val + b + j), v1 = __ldcs(val + b + j + 32),
+                  v2 = __ldcs(val + b + j + 64), v3 = __ldcs(val + b + j + 96);
+      const float4 x0 = ldx4(X, c0), x1 = ldx4(X, c1), x2 = ldx4(X, c2), x3 = ldx4(X, c3);
       fma4(s, v0, x0);
       fma4(s, v1, x1);
+      fma4(s, v2, x2);
+      fma4(s, v3, x3);
     }
     for (; j < L; j += 32) fma4(s, __ldcs(val + b + j), ldx4(X, __ldcs(col + b + j)));
     s.x = tree32(s.x);
@@ -147,12 +152,16 @@ __device__ __forceinline__ float4 cta_sum256x4(const int32_t* __restrict__ col,
   const int tid = threadIdx.x;
   float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
   int64_t t = tid;
-  for (; t + 256 < L; t += 512) {
-    const int c0 = __ldcs(col + b + t), c1 = __ldcs(col + b + t + 256);
-    const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256);
-    const float4 x0 = ldx4(X, c0), x1 = ldx4(X, c1);
+  for (; t + 768 < L; t += 1024) {
+    const int c0 = __ldcs(col + b + t), c1 = __ldcs(col + b + t + 256),
+              c2 = __ldcs(col + b + t + 512), c3 = __ldcs(col + b + t + 768);
+    const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256),
+                v2 = __ldcs(val + b + t + 512), v3 = __ldcs(val + b + t + 768);
+    const float4 x0 = ldx4(X, c0), x1 = ldx4(X, c1), x2 = ldx4(X, c2), x3 = ldx4(X, c3);
     fma4(s, v0, x0);
     fma4(s, v1, x1);
+    fma4(s, v2, x2);
+    fma4(s, v3, x3);
   }
   for (; t < L; t += 256) fma4(s, __ldcs(val + b + t), ldx4(X, __ldcs(col + b + t)));
   red[tid] = s;
@@ -242,10 +251,15 @@ void spmm4_typed(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s) {
   if (p->nrows) {
     const int64_t blocks = (p->nrows + L4_THREADS - 1) / L4_THREADS;
     const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)sms * 32));
-    if (p->opts.evict_first && p->stream_ef)
-      k_lane4<OT, 1><<<g, L4_THREADS, 0, s>>>(rp, p->d_col, p->d_val, X, Y, p->nrows);
-    else
-      k_lane4<OT, 0><<<g, L4_THREADS, 0, s>>>(rp, p->d_col, p->d_val, X, Y, p->nrows);
+    // shape: 0 = 2 chunks in flight, 2 CTAs/SM (default); 1 = 2 chunks, 3 CTAs/SM;
+    // 2 = 1 chunk, 4 CTAs/SM (SPMV_L4_V dev knob)
+    int v = 0;
+    if (const char* e = getenv("SPMV_L4_V")) v = std::min(2, std::max(0, atoi(e)));
+    const bool ef = p->opts.evict_first && p->stream_ef;
+    auto k = v == 2 ? (ef ? k_lane4<OT, 1, 4, 1> : k_lane4<OT, 0, 4, 1>)
+           : v == 1 ? (ef ? k_lane4<OT, 1, 3, 2> : k_lane4<OT, 0, 3, 2>)
+                    : (ef ? k_lane4<OT, 1, 2, 2> : k_lane4<OT, 0, 2, 2>);
+    k<<<g, L4_THREADS, 0, s>>>(rp, p->d_col, p->d_val, X, Y, p->nrows);
   }
   cudaStream_t s1 = s, s2 = s;
   const bool conc = p->conc && (p->n_mid > 0 || p->n_cta > 0 || p->n_chunks > 0);
