@@ -531,7 +531,7 @@ def run_reference(args):
                       steps=args.steps, warmup=args.warmup)
     ms = cb["ms_per_spmv"]
     line = dict(metric=METRIC, value=cb["value"], unit="GB/s", n_gpus=world, steps=args.steps,
-                warmup=args.warmup, ms_per_step=ms, higher_is_better=True, scaling="weak",
+                warmup=args.warmup, ms_per_step=ms, higher_is_better=True, scaling="strong",
                 vs_baseline=None, dtype="f64", data="synthetic", impl="reference",
                 config={"workload": f"{w.name} (BASELINE configs[{args.config - 1}])", "n": A.n,
                         "nnz": A.nnz, "ordering": args.orderings.split(",")[-1],

@@ -69,6 +69,7 @@ for o in ords:
     perm_d = torch.from_numpy(perm).to(dev)
     xB = None
     ref = None
+    kind = os.environ.get("KIND", "exec")  # exec | spmm4 | coo
     for c in combos:
         saved = {k: os.environ.get(k) for k in c}
         os.environ.update({k: str(v) for k, v in c.items()})
@@ -76,15 +77,20 @@ for o in ords:
         if xB is None:
             xB = P.permute_vec(torch.from_numpy(w.x).to(dev))
             y = torch.empty(A.n, device=dev)
-        P.exec(xB, y)
+            X4 = xB[:, None].repeat(1, 4).contiguous() if kind == "spmm4" else None
+            Y4 = torch.empty_like(X4) if kind == "spmm4" else None
+        run = {"exec": lambda: P.exec(xB, y), "coo": lambda: P.exec_coo(xB, y),
+               "spmm4": lambda: P.exec_spmm4(X4, Y4)}[kind]
+        run()
         torch.cuda.synchronize()
+        out = Y4 if kind == "spmm4" else y
         if ref is None:
-            ref = y.clone()
-        same = bool(torch.equal(ref, y))
-        cold = timeit(lambda: P.exec(xB, y), lambda: torch.sum(buf, dim=0, out=sink))
-        warm = timeit(lambda: P.exec(xB, y), lambda: None)
+            ref = out.clone()
+        same = bool(torch.equal(ref, out))
+        cold = timeit(run, lambda: torch.sum(buf, dim=0, out=sink))
+        warm = timeit(run, lambda: None)
         info = P.info()
-        print(json.dumps({"ord": o, **c, "cold_us": cold, "warm_us": warm,
+        print(json.dumps({"ord": o, "kind": kind, **c, "cold_us": cold, "warm_us": warm,
                           "x_ideal": round(cold / (ideal / 6539.2e9 * 1e6), 3),
                           "win_bytes": info["l2_window_bytes"], "bitwise_same": same}), flush=True)
         P.close()
