@@ -251,9 +251,10 @@ void spmm4_typed(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s) {
   if (p->nrows) {
     const int64_t blocks = (p->nrows + L4_THREADS - 1) / L4_THREADS;
     const unsigned g = (unsigned)std::max<int64_t>(1, std::min<int64_t>(blocks, (int64_t)sms * 32));
-    // shape: 0 = 2 chunks in flight, 2 CTAs/SM (default); 1 = 2 chunks, 3 CTAs/SM;
+    // shape: 0 = 2 chunks in flight, 2 CTAs/SM; 1 = 2 chunks, 3 CTAs/SM (80
+    // registers, default: SBM 0.178 vs 0.189 ms, RMAT-26 6.74 vs 7.23 ms, r41);
     // 2 = 1 chunk, 4 CTAs/SM (SPMV_L4_V dev knob)
-    int v = 0;
+    int v = 1;
     if (const char* e = getenv("SPMV_L4_V")) v = std::min(2, std::max(0, atoi(e)));
     const bool ef = p->opts.evict_first && p->stream_ef;
     auto k = v == 2 ? (ef ? k_lane4<OT, 1, 4, 1> : k_lane4<OT, 0, 4, 1>)
