@@ -100,8 +100,9 @@ template <bool SS>
 __device__ __forceinline__ void store_y(float* __restrict__ y, const YDst& d, int64_t r, float v) {
   if constexpr (SS) {
     if (d.n) {
-#pragma unroll 1
-      for (int k = 0; k < d.n; ++k) d.p[k][r] = v;
+#pragma unroll
+      for (int k = 0; k < 8; ++k)  // constant indices: the pointers stay in the param space
+        if (k < d.n) d.p[k][r] = v;
       return;
     }
   }
@@ -430,20 +431,22 @@ __global__ void __launch_bounds__(256)
     const int32_t* cc = col + b;
     const float* vv = val + b;
     float s = 0.f;
-    int j = lane;
-    for (; j + 96 < L; j += 128) {
-      const int c0 = __ldcs(cc + j), c1 = __ldcs(cc + j + 32), c2 = __ldcs(cc + j + 64),
-                c3 = __ldcs(cc + j + 96);
-      const float v0 = __ldcs(vv + j), v1 = __ldcs(vv + j + 32), v2 = __ldcs(vv + j + 64),
-                  v3 = __ldcs(vv + j + 96);
-      const float x0 = gx<HOT>(x, xh, c0), x1 = gx<HOT>(x, xh, c1), x2 = gx<HOT>(x, xh, c2),
-                  x3 = gx<HOT>(x, xh, c3);
+    // four strided entries in flight per lane, the ragged end guarded: a slot
+    // past the row adds +0, which leaves s unchanged (s starts at +0 and is
+    // never -0), so the association is exactly j, j+32, j+64, ...
+    for (int j = lane; j < L; j += 128) {
+      const bool p1 = j + 32 < L, p2 = j + 64 < L, p3 = j + 96 < L;
+      const int c0 = __ldcs(cc + j), c1 = p1 ? __ldcs(cc + j + 32) : 0,
+                c2 = p2 ? __ldcs(cc + j + 64) : 0, c3 = p3 ? __ldcs(cc + j + 96) : 0;
+      const float v0 = __ldcs(vv + j), v1 = p1 ? __ldcs(vv + j + 32) : 0.f,
+                  v2 = p2 ? __ldcs(vv + j + 64) : 0.f, v3 = p3 ? __ldcs(vv + j + 96) : 0.f;
+      const float x0 = gx<HOT>(x, xh, c0), x1 = p1 ? gx<HOT>(x, xh, c1) : 0.f,
+                  x2 = p2 ? gx<HOT>(x, xh, c2) : 0.f, x3 = p3 ? gx<HOT>(x, xh, c3) : 0.f;
       s = __fadd_rn(s, __fmul_rn(v0, x0));
       s = __fadd_rn(s, __fmul_rn(v1, x1));
       s = __fadd_rn(s, __fmul_rn(v2, x2));
       s = __fadd_rn(s, __fmul_rn(v3, x3));
     }
-    for (; j < L; j += 32) s = __fadd_rn(s, __fmul_rn(__ldcs(vv + j), gx<HOT>(x, xh, __ldcs(cc + j))));
     s = warp_tree(s);
     if (lane == 0) {
       const float v = __fmul_rn(s, alpha);
