@@ -513,21 +513,21 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             float* red, const float* __restrict__ xh) {
   const int tid = threadIdx.x;
   float s = 0.f;
-  int64_t t = tid;
-  for (; t + 768 < L; t += 1024) {
-    const int c0 = __ldcs(col + b + t), c1 = __ldcs(col + b + t + 256),
-              c2 = __ldcs(col + b + t + 512), c3 = __ldcs(col + b + t + 768);
-    const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256),
-                v2 = __ldcs(val + b + t + 512), v3 = __ldcs(val + b + t + 768);
-    const float x0 = gx<HOT>(x, xh, c0), x1 = gx<HOT>(x, xh, c1), x2 = gx<HOT>(x, xh, c2),
-                x3 = gx<HOT>(x, xh, c3);
+  // four strided entries in flight, ragged end guarded (+0 slots, as k_warp_rows)
+  for (int64_t t = tid; t < L; t += 1024) {
+    const bool p1 = t + 256 < L, p2 = t + 512 < L, p3 = t + 768 < L;
+    const int c0 = __ldcs(col + b + t), c1 = p1 ? __ldcs(col + b + t + 256) : 0,
+              c2 = p2 ? __ldcs(col + b + t + 512) : 0, c3 = p3 ? __ldcs(col + b + t + 768) : 0;
+    const float v0 = __ldcs(val + b + t), v1 = p1 ? __ldcs(val + b + t + 256) : 0.f,
+                v2 = p2 ? __ldcs(val + b + t + 512) : 0.f,
+                v3 = p3 ? __ldcs(val + b + t + 768) : 0.f;
+    const float x0 = gx<HOT>(x, xh, c0), x1 = p1 ? gx<HOT>(x, xh, c1) : 0.f,
+                x2 = p2 ? gx<HOT>(x, xh, c2) : 0.f, x3 = p3 ? gx<HOT>(x, xh, c3) : 0.f;
     s = __fadd_rn(s, __fmul_rn(v0, x0));
     s = __fadd_rn(s, __fmul_rn(v1, x1));
     s = __fadd_rn(s, __fmul_rn(v2, x2));
     s = __fadd_rn(s, __fmul_rn(v3, x3));
   }
-  for (; t < L; t += 256)
-    s = __fadd_rn(s, __fmul_rn(__ldcs(val + b + t), gx<HOT>(x, xh, __ldcs(col + b + t))));
   red[tid] = s;
   __syncthreads();
 #pragma unroll
