@@ -123,19 +123,20 @@ __global__ void __launch_bounds__(256)
     const int64_t b = (int64_t)rp[r];
     const int L = (int)((int64_t)rp[r + 1] - b);
     float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
-    int j = lane;
-    for (; j + 96 < L; j += 128) {  // four independent gathers in flight
-      const int c0 = __ldcs(col + b + j), c1 = __ldcs(col + b + j + 32),
-                c2 = __ldcs(col + b + j + 64), c3 = __ldcs(col + b + j + 96);
-      const float v0 = __ldcs(val + b + j), v1 = __ldcs(val + b + j + 32),
-                  v2 = __ldcs(val + b + j + 64), v3 = __ldcs(val + b + j + 96);
-      const float4 x0 = ldx4(X, c0), x1 = ldx4(X, c1), x2 = ldx4(X, c2), x3 = ldx4(X, c3);
+    const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int j = lane; j < L; j += 128) {  // four gathers in flight, ragged end guarded (+0)
+      const bool p1 = j + 32 < L, p2 = j + 64 < L, p3 = j + 96 < L;
+      const int c0 = __ldcs(col + b + j), c1 = p1 ? __ldcs(col + b + j + 32) : 0,
+                c2 = p2 ? __ldcs(col + b + j + 64) : 0, c3 = p3 ? __ldcs(col + b + j + 96) : 0;
+      const float v0 = __ldcs(val + b + j), v1 = p1 ? __ldcs(val + b + j + 32) : 0.f,
+                  v2 = p2 ? __ldcs(val + b + j + 64) : 0.f, v3 = p3 ? __ldcs(val + b + j + 96) : 0.f;
+      const float4 x0 = ldx4(X, c0), x1 = p1 ? ldx4(X, c1) : z4, x2 = p2 ? ldx4(X, c2) : z4,
+                   x3 = p3 ? ldx4(X, c3) : z4;
       fma4(s, v0, x0);
       fma4(s, v1, x1);
       fma4(s, v2, x2);
       fma4(s, v3, x3);
     }
-    for (; j < L; j += 32) fma4(s, __ldcs(val + b + j), ldx4(X, __ldcs(col + b + j)));
     s.x = tree32(s.x);
     s.y = tree32(s.y);
     s.z = tree32(s.z);
@@ -151,19 +152,20 @@ __device__ __forceinline__ float4 cta_sum256x4(const int32_t* __restrict__ col,
                                                int64_t L, float4* red) {
   const int tid = threadIdx.x;
   float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
-  int64_t t = tid;
-  for (; t + 768 < L; t += 1024) {
-    const int c0 = __ldcs(col + b + t), c1 = __ldcs(col + b + t + 256),
-              c2 = __ldcs(col + b + t + 512), c3 = __ldcs(col + b + t + 768);
-    const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256),
-                v2 = __ldcs(val + b + t + 512), v3 = __ldcs(val + b + t + 768);
-    const float4 x0 = ldx4(X, c0), x1 = ldx4(X, c1), x2 = ldx4(X, c2), x3 = ldx4(X, c3);
+  const float4 z4 = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int64_t t = tid; t < L; t += 1024) {  // ragged end guarded (+0), as k_warp_rows4
+    const bool p1 = t + 256 < L, p2 = t + 512 < L, p3 = t + 768 < L;
+    const int c0 = __ldcs(col + b + t), c1 = p1 ? __ldcs(col + b + t + 256) : 0,
+              c2 = p2 ? __ldcs(col + b + t + 512) : 0, c3 = p3 ? __ldcs(col + b + t + 768) : 0;
+    const float v0 = __ldcs(val + b + t), v1 = p1 ? __ldcs(val + b + t + 256) : 0.f,
+                v2 = p2 ? __ldcs(val + b + t + 512) : 0.f, v3 = p3 ? __ldcs(val + b + t + 768) : 0.f;
+    const float4 x0 = ldx4(X, c0), x1 = p1 ? ldx4(X, c1) : z4, x2 = p2 ? ldx4(X, c2) : z4,
+                 x3 = p3 ? ldx4(X, c3) : z4;
     fma4(s, v0, x0);
     fma4(s, v1, x1);
     fma4(s, v2, x2);
     fma4(s, v3, x3);
   }
-  for (; t < L; t += 256) fma4(s, __ldcs(val + b + t), ldx4(X, __ldcs(col + b + t)));
   red[tid] = s;
   __syncthreads();
 #pragma unroll
