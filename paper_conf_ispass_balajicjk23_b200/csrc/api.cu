@@ -136,6 +136,19 @@ spmv_status spmv_exec(spmv_plan_t p, const float* x_B, float* y_B, void* stream)
   API_END
 }
 
+spmv_status spmv_rabbitpp_gpu(const spmv_csr_t* A, const int32_t* perm_rabbit,
+                              const int32_t* comm, int32_t* perm_out, void* stream) {
+  API_BEGIN
+  if (!A || (A->n && (!perm_rabbit || !comm || !perm_out)))
+    SPMV_FAIL(SPMV_EINVAL, "spmv_rabbitpp_gpu: NULL argument");
+  if (A->n < 0 || A->nnz < 0 || (A->row_ptr32 == nullptr) == (A->row_ptr64 == nullptr) ||
+      (A->nnz && !A->col_idx))
+    SPMV_FAIL(SPMV_EINVAL, "spmv_rabbitpp_gpu: malformed CSR descriptor");
+  if (A->n > (int64_t)INT32_MAX) SPMV_FAIL(SPMV_EUNSUPPORTED, "spmv_rabbitpp_gpu: n > INT32_MAX");
+  spmv::rabbitpp_gpu(A, perm_rabbit, comm, perm_out, S(stream));
+  API_END
+}
+
 spmv_status spmv_exec_spmm4(spmv_plan_t p, const float* X_B, float* Y_B, void* stream) {
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_spmm4: NULL plan");

@@ -953,6 +953,88 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
   }
 }
 
+// ---------------------------------------------- RABBIT++ post-pass (GPU)
+// SURVEY §8(f4).  Inputs by OLD vertex id: the RABBIT
+// permutation and the top-level community of every vertex.
+template <typename AT>
+__global__ void k_pp_scan_entries(const AT* rp, const int32_t* col, int64_t n,
+                                  const int32_t* comm, unsigned long long* colcnt,
+                                  uint8_t* insular) {
+  // warp per row: column counts (diagonal and duplicates included, reading
+  // c13) and insularity (an off-diagonal entry (i, j) with comm[i] != comm[j]
+  // makes both i and j non-insular: S = Bp + Bp^T, reading c5)
+  const int lane = threadIdx.x & 31;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += W) {
+    const int64_t a = (int64_t)rp[i], e = (int64_t)rp[i + 1];
+    const int32_t ci = comm[i];
+    for (int64_t k = a + lane; k < e; k += 32) {
+      const int32_t j = col[k];
+      atomicAdd(&colcnt[j], 1ull);
+      if (j != i && comm[j] != ci) {
+        insular[i] = 0;
+        insular[j] = 0;
+      }
+    }
+  }
+}
+
+// group of the vertex at RABBIT position q: 0 non-insular hub, 1 non-insular
+// non-hub, 2 insular; flags[g * n + q] = (group == g)
+__global__ void k_pp_groups(const int32_t* perm_rabbit, const unsigned long long* colcnt,
+                            const uint8_t* insular, int64_t n, int64_t nnz, int32_t* flags) {
+  GRID_STRIDE(v, n) {
+    const int64_t q = perm_rabbit[v];
+    const bool hub = (__int128)colcnt[v] * n > (__int128)nnz;  // P:181, reading c14
+    const int g = insular[v] ? 2 : (hub ? 0 : 1);
+    flags[q] = g == 0;
+    flags[n + q] = g == 1;
+    flags[2 * n + q] = g == 2;
+  }
+}
+
+// new id = start of the vertex's group + its rank among the group in RABBIT order
+__global__ void k_pp_assign(const int32_t* perm_rabbit, const int32_t* flags, const int64_t* pos,
+                            int64_t n, int32_t* perm_out) {
+  const int64_t c0 = pos[n], c1 = pos[2 * n + 1];
+  GRID_STRIDE(v, n) {
+    const int64_t q = perm_rabbit[v];
+    int64_t id;
+    if (flags[q]) id = pos[q];
+    else if (flags[n + q]) id = c0 + pos[n + 1 + q];
+    else id = c0 + c1 + pos[2 * n + 2 + q];
+    perm_out[v] = (int32_t)id;
+  }
+}
+
+void rabbitpp_gpu(const spmv_csr_t* A, const int32_t* perm_rabbit, const int32_t* comm,
+                  int32_t* perm_out, cudaStream_t s) {
+  const int64_t n = A->n, nnz = A->nnz;
+  if (n == 0) return;
+  unsigned long long* cnt = dalloc<unsigned long long>(n);
+  uint8_t* ins = dalloc<uint8_t>(n);
+  int32_t* flags = dalloc<int32_t>(3 * n);
+  int64_t* pos = dalloc<int64_t>(3 * (n + 1));
+  int64_t* tmp = dalloc<int64_t>(scan_temp_len(n));
+  SPMV_CUDA(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * n, s));
+  SPMV_CUDA(cudaMemsetAsync(ins, 1, (size_t)n, s));
+  const unsigned gw = (unsigned)std::min<int64_t>((n + 7) / 8, 148 * 64);
+  if (A->row_ptr64)
+    k_pp_scan_entries<int64_t><<<gw, 256, 0, s>>>(A->row_ptr64, A->col_idx, n, comm, cnt, ins);
+  else
+    k_pp_scan_entries<int32_t><<<gw, 256, 0, s>>>(A->row_ptr32, A->col_idx, n, comm, cnt, ins);
+  k_pp_groups<<<grid_for(n), TPB, 0, s>>>(perm_rabbit, cnt, ins, n, nnz, flags);
+  for (int g = 0; g < 3; ++g) exclusive_scan<int32_t>(flags + g * n, n, pos + g * (n + 1), tmp, s);
+  k_pp_assign<<<grid_for(n), TPB, 0, s>>>(perm_rabbit, flags, pos, n, perm_out);
+  SPMV_LAUNCH_CHECK();
+  SPMV_CUDA(cudaStreamSynchronize(s));  // scratch lifetime
+  dfree(cnt);
+  dfree(ins);
+  dfree(flags);
+  dfree(pos);
+  dfree(tmp);
+}
+
 // ------------------------------------------------------------------ public
 void plan_build(spmv_plan_s* p, const spmv_csr_t* A, const int32_t* perm) {
   const int64_t n = p->n;

@@ -109,6 +109,8 @@ struct spmv_plan_s {
 
 namespace spmv {
 void plan_build(spmv_plan_s* p, const spmv_csr_t* A, const int32_t* perm);
+void rabbitpp_gpu(const spmv_csr_t* A, const int32_t* perm_rabbit, const int32_t* comm,
+                  int32_t* perm_out, cudaStream_t s);
 void plan_permute(spmv_plan_s* p, cudaStream_t s);
 void plan_free(spmv_plan_s* p);
 void permute_vec(spmv_plan_s* p, const float* in, float* out, int inverse, cudaStream_t s);

@@ -85,6 +85,7 @@ def lib() -> ctypes.CDLL:
             "spmv_exec_scaled": (i32, [vp, vp, vp, dp, dp, vp]),
             "spmv_exec_spmm4": (i32, [vp, vp, vp, vp]),
             "spmv_exec_coo": (i32, [vp, vp, vp, vp]),
+            "spmv_rabbitpp_gpu": (i32, [ctypes.POINTER(_Csr), vp, vp, vp, vp]),
             "spmv_exec_scaled_bcast": (i32, [vp, vp, vp, i32, dp, dp, vp]),
             "spmv_ipc_handle": (i32, [vp, vp]),
             "spmv_dev_alloc": (i32, [i32, i64, ctypes.POINTER(vp)]),
@@ -381,3 +382,19 @@ def ipc_open(handle: bytes) -> int:
 
 def ipc_close(ptr: int) -> None:
     _check(lib().spmv_ipc_close(ctypes.c_void_p(ptr)))
+
+
+def rabbitpp_gpu(row_ptr, col, perm_rabbit, comm, stream=None):
+    """RABBIT++ post-pass on the GPU (spmv_rabbitpp_gpu): device tensors in,
+    device int32 permutation out."""
+    import torch
+    n = row_ptr.numel() - 1
+    A = _Csr(n, col.numel(), None, None, _ptr(col), None)
+    if row_ptr.dtype == torch.int64:
+        A.row_ptr64 = _ptr(row_ptr)
+    else:
+        A.row_ptr32 = _ptr(row_ptr)
+    out = torch.empty(n, dtype=torch.int32, device=col.device)
+    _check(lib().spmv_rabbitpp_gpu(ctypes.byref(A), _ptr(perm_rabbit), _ptr(comm), _ptr(out),
+                                   _stream_ptr(stream)))
+    return out

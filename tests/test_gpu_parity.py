@@ -409,3 +409,21 @@ def test_hot_column_set_bitwise(dev, name, make, monkeypatch):
     assert P1.info()["exec_launches"] == i0["exec_launches"] + 1 - (1 if both else 0)
     P0.close()
     P1.close()
+
+
+@pytest.mark.parametrize("name,make", [c for c in CASES if c[0] != "longrows"])
+def test_rabbitpp_gpu_postpass_bitexact(dev, name, make):
+    """spmv_rabbitpp_gpu from the host RABBIT order and top-level
+    communities equals the host RABBIT++ (and hence the oracle's, test_abi)."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = make()
+    pr, _ = spmv.reorder(A.row_ptr, A.col, "rabbit")
+    comm = spmv.reorder_last_comm(A.n)
+    ppp, _ = spmv.reorder(A.row_ptr, A.col, "rabbitpp")
+    out = spmv.rabbitpp_gpu(torch.from_numpy(A.row_ptr).to(dev), torch.from_numpy(A.col).to(dev),
+                            torch.from_numpy(pr).to(dev), torch.from_numpy(comm).to(dev))
+    assert np.array_equal(out.cpu().numpy(), ppp)
+    out32 = spmv.rabbitpp_gpu(torch.from_numpy(A.row_ptr).to(dev, torch.int32),
+                              torch.from_numpy(A.col).to(dev), torch.from_numpy(pr).to(dev),
+                              torch.from_numpy(comm).to(dev))
+    assert np.array_equal(out32.cpu().numpy(), ppp)
