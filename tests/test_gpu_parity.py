@@ -318,6 +318,13 @@ def test_rmat26_full_size(dev):
     _full_size_check(dev, 3, "original")
 
 
+def test_stencil464_full_size(dev):
+    """BASELINE configs[3] (27-point stencil 464^3, 99.9 M rows, 2.69 G nnz) at
+    full size as generated (random labels): the int64 row-pointer path
+    (NZ >= 2^31), lane rows with shared 8-entry chunks, x = 400 MB > L2."""
+    _full_size_check(dev, 4, "original", nsample=1000)
+
+
 @pytest.mark.parametrize("name,make", CASES)
 def test_smem_window_and_l2_options_bitwise(dev, name, make):
     """The x window, L2 policies and an unaligned x (window disabled) change
