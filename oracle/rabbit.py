@@ -127,6 +127,7 @@ def rabbit(n, row_ptr, col) -> RabbitResult:
 
 # RABBIT++ variants (Table II design space)
 RABBITPP, HUBSORT, INSULAR_ONLY, HUBGROUP_ONLY = "rabbitpp", "hubsort", "insular", "hubgroup"
+HUBSORT_ONLY = "hubsort_only"
 
 
 def insular_flags(n, row_ptr, col, comm) -> np.ndarray:
@@ -171,6 +172,11 @@ def rabbitpp(n, row_ptr, col, rabbit_perm, comm, variant=RABBITPP) -> np.ndarray
         groups = [[v for v in seq if not ins[v]], [v for v in seq if ins[v]]]
     elif variant == HUBGROUP_ONLY:      # modification 2 only, no insular grouping
         groups = [[v for v in seq if hub[v]], [v for v in seq if not hub[v]]]
+    elif variant == HUBSORT_ONLY:       # hubs by decreasing in-degree, no insular grouping
+        g0 = [v for v in seq if hub[v]]  # (Table II, left half, RABBIT+HUBSORT)
+        pos = {v: i for i, v in enumerate(seq)}
+        g0.sort(key=lambda v: (-int(colcnt[v]), pos[v]))
+        groups = [g0, [v for v in seq if not hub[v]]]
     else:
         raise ValueError(variant)
     perm = np.empty(n, np.int64)

@@ -375,7 +375,8 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
       std::stable_sort(seq.begin(), seq.end(),
                        [&](int32_t a, int32_t b) { return colcnt[a] > colcnt[b]; });
       for (int64_t i = 0; i < n; ++i) perm_out[seq[i]] = (int32_t)i;
-    } else if (method >= SPMV_ORDER_RABBIT && method <= SPMV_ORDER_HUBGROUP) {
+    } else if ((method >= SPMV_ORDER_RABBIT && method <= SPMV_ORDER_HUBGROUP) ||
+               method == SPMV_ORDER_HUBSORT_ONLY) {
       // community detection is shared by RABBIT and every RABBIT++ variant:
       // reuse the last detection on this thread when the input is identical
       const uint64_t key = input_key(n, nnz, rp, col);
@@ -500,9 +501,12 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
         } else if (method == SPMV_ORDER_INSULAR) {
           take([&](int32_t v) { return !ins[v]; });
           take([&](int32_t v) { return (bool)ins[v]; });
-        } else {  // HUBGROUP only
+        } else {  // HUBGROUP only / HUBSORT only (no insular grouping)
           take([&](int32_t v) { return (bool)hub[v]; });
           S0.n_group0 = (int64_t)out.size();
+          if (method == SPMV_ORDER_HUBSORT_ONLY)
+            std::stable_sort(out.begin(), out.end(),
+                             [&](int32_t a, int32_t b) { return colcnt[a] > colcnt[b]; });
           take([&](int32_t v) { return !hub[v]; });
         }
         for (int64_t i = 0; i < n; ++i) perm_out[out[i]] = (int32_t)i;

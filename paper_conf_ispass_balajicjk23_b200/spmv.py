@@ -17,9 +17,10 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 SO_PATH = os.path.join(_HERE, "libspmv.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "spmv.h")
 
-ORIGINAL, RANDOM, RABBIT, RABBITPP, HUBSORT, INSULAR, HUBGROUP, DEGSORT = range(8)
+ORIGINAL, RANDOM, RABBIT, RABBITPP, HUBSORT, INSULAR, HUBGROUP, DEGSORT, HUBSORT_ONLY = range(9)
 METHODS = {"original": ORIGINAL, "random": RANDOM, "rabbit": RABBIT, "rabbitpp": RABBITPP,
-           "hubsort": HUBSORT, "insular": INSULAR, "hubgroup": HUBGROUP, "degsort": DEGSORT}
+           "hubsort": HUBSORT, "insular": INSULAR, "hubgroup": HUBGROUP, "degsort": DEGSORT,
+           "hubsort_only": HUBSORT_ONLY}
 STATUS = {0: "SPMV_OK", 1: "SPMV_EINVAL", 2: "SPMV_EPERM", 3: "SPMV_ENOMEM", 4: "SPMV_ECUDA",
           5: "SPMV_ENCCL", 6: "SPMV_EUNSUPPORTED", 7: "SPMV_ESTATE"}
 

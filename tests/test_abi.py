@@ -62,7 +62,8 @@ def test_reorder_rabbit_bitexact(name, A):
 @pytest.mark.parametrize("variant,method", [(rabbit.RABBITPP, "rabbitpp"),
                                             (rabbit.HUBSORT, "hubsort"),
                                             (rabbit.INSULAR_ONLY, "insular"),
-                                            (rabbit.HUBGROUP_ONLY, "hubgroup")])
+                                            (rabbit.HUBGROUP_ONLY, "hubgroup"),
+                                            (rabbit.HUBSORT_ONLY, "hubsort_only")])
 def test_reorder_rabbitpp_bitexact(name, A, variant, method):
     r = rabbit.rabbit(A.n, A.row_ptr, A.col)
     ref = rabbit.rabbitpp(A.n, A.row_ptr, A.col, r.perm, r.comm, variant)

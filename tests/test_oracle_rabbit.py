@@ -177,6 +177,15 @@ def test_rabbitpp_variants():
     seq = order_of(hs)
     cc = np.bincount(col, minlength=n)
     assert all(cc[seq[i]] >= cc[seq[i + 1]] for i in range(g0 - 1))
+    # HUBSORT_ONLY: every hub first, in non-increasing in-degree, then the rest
+    # in RABBIT order (no insular grouping)
+    hso = rabbit.rabbitpp(n, rp, col, r.perm, r.comm, rabbit.HUBSORT_ONLY)
+    assert permute.is_bijection(hso, n)
+    s2 = order_of(hso)
+    nh = int(hub.sum())
+    assert all(hub[v] for v in s2[:nh]) and all(cc[s2[i]] >= cc[s2[i + 1]] for i in range(nh - 1))
+    rest = [v for v in order_of(r.perm) if not hub[v]]
+    assert list(s2[nh:]) == rest
 
 
 def test_fig5_hub_arithmetic():
