@@ -230,16 +230,15 @@ __global__ void __launch_bounds__(CO_THREADS)
   }
 }
 
-// k_coo_w (variant 2): warp tiles of CW_TILE = 512 entries, 16 per lane (two
+// k_coo_w (variant 2): warp tiles of 32 E entries, E = 16 per lane (two
 // 256-bit chunks of row / col / val, 16 gathers in flight), no shared memory
 // and no CTA barrier.  Lane pieces of a row crossing lanes are combined with
 // a segmented suffix scan over the warp in fp64 (shuffles; the association is
 // fixed by the lane layout); pieces crossing warp tiles go through k_coo_fix
 // exactly like the CTA tiles of k_coo.
-constexpr int CW_E = 16;
-constexpr int CW_TILE = 32 * CW_E;
+constexpr int CW_TILE_MIN = 32 * 8;  // finest warp tile (8 entries per lane): sizes the tile arrays
 
-template <int EF, int MINB, bool ZG>
+template <int EF, int MINB, bool ZG, int E>
 __global__ void __launch_bounds__(256, MINB)
     k_coo_w(const int32_t* __restrict__ row, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
@@ -250,16 +249,17 @@ __global__ void __launch_bounds__(256, MINB)
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t tile = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < ntiles;
        tile += W) {
-    const int64_t e0 = tile * CW_TILE;
-    const int64_t eb = e0 + (int64_t)lane * CW_E;
-    const int nh = (int)max((int64_t)0, min((int64_t)CW_E, nnz - eb));
-    int rr[16], cc[16];
-    float vv[16];
-    if (nh == CW_E) {
+    constexpr int TILE = 32 * E;
+    const int64_t e0 = tile * TILE;
+    const int64_t eb = e0 + (int64_t)lane * E;
+    const int nh = (int)max((int64_t)0, min((int64_t)E, nnz - eb));
+    int rr[E], cc[E];
+    float vv[E];
+    if (nh == E) {
       int r8[8], c8[8];
       float v8[8];
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
+      for (int h = 0; h < E / 8; ++h) {
         ld8<EF>(row + eb + 8 * h, r8);
         ld8<EF>(col + eb + 8 * h, c8);
         ld8<EF>(val + eb + 8 * h, v8);
@@ -272,25 +272,25 @@ __global__ void __launch_bounds__(256, MINB)
       }
     } else {
 #pragma unroll
-      for (int i = 0; i < 16; ++i) {
+      for (int i = 0; i < E; ++i) {
         rr[i] = i < nh ? row[eb + i] : -1;
         cc[i] = i < nh ? col[eb + i] : 0;
         vv[i] = i < nh ? val[eb + i] : 0.f;
       }
     }
-    float xv[16];
+    float xv[E];
 #pragma unroll
-    for (int i = 0; i < 16; ++i) xv[i] = i < nh ? __ldg(x + cc[i]) : 0.f;
+    for (int i = 0; i < E; ++i) xv[i] = i < nh ? __ldg(x + cc[i]) : 0.f;
     int mylast = -1;
 #pragma unroll
-    for (int i = 0; i < 16; ++i) mylast = i < nh ? rr[i] : mylast;
+    for (int i = 0; i < E; ++i) mylast = i < nh ? rr[i] : mylast;
     int prow = __shfl_up_sync(0xffffffffu, mylast, 1);
     if (lane == 0) prow = e0 > 0 && nh > 0 ? row[e0 - 1] : -1;
     int hrow = -1, cur = -1, last = prow;
     float hsum = 0.f, run = 0.f;
     bool single = true;
 #pragma unroll
-    for (int i = 0; i < 16; ++i) {
+    for (int i = 0; i < E; ++i) {
       if (i < nh) {
         const int r = rr[i];
         if (r != cur) {
@@ -317,7 +317,7 @@ __global__ void __launch_bounds__(256, MINB)
       hrow = cur;
       hsum = run;
     }
-    const int64_t tile_end = min(nnz, e0 + CW_TILE);
+    const int64_t tile_end = min(nnz, e0 + TILE);
     // first row of the next warp tile (decides whether lane 31's chain is open)
     int nxt = -1;
     if (lane == 31 && tile_end < nnz) nxt = row[tile_end];
@@ -410,7 +410,7 @@ void* dmalloc(size_t bytes) {
 void coo_build(spmv_plan_s* p, cudaStream_t s) {
   if (p->d_coo_row) return;
   const int64_t nz = p->nnz_local;
-  p->coo_tiles = (nz + CW_TILE - 1) / CW_TILE;  // the finer (warp) tiling bounds both
+  p->coo_tiles = (nz + CW_TILE_MIN - 1) / CW_TILE_MIN;  // the finest tiling bounds every variant
   p->d_coo_row = (int32_t*)dmalloc(sizeof(int32_t) * (size_t)(nz + 8));
   const int64_t T = std::max<int64_t>(p->coo_tiles, 1);
   p->d_coo_trow = (int32_t*)dmalloc(sizeof(int32_t) * 2 * (size_t)T);
@@ -448,7 +448,10 @@ void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s) {
   }
   int v = 2;
   if (const char* e = getenv("SPMV_COO_V")) v = atoi(e) == 1 ? 1 : 2;  // dev knob
-  const int64_t T = v == 1 ? (p->nnz_local + COO_TILE - 1) / COO_TILE : p->coo_tiles;
+  int E = 16;  // entries per lane of k_coo_w
+  if (const char* e = getenv("SPMV_COO_E")) E = atoi(e) == 8 ? 8 : 16;  // dev knob
+  const int64_t tile = v == 1 ? COO_TILE : 32 * E;
+  const int64_t T = (p->nnz_local + tile - 1) / tile;
   int32_t* frow = p->d_coo_trow;
   int32_t* lrow = p->d_coo_trow + T;
   double* fpart = p->d_coo_tpart;
@@ -465,14 +468,14 @@ void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s) {
                                         p->nrows, T, frow, lrow, fpart, lpart, p->d_coo_tflag);
   } else {
     const unsigned g = (unsigned)std::min<int64_t>((T + 7) / 8, (int64_t)sms(p->device) * 16);
-    int minb = 3;  // <= 85 registers: 3 CTAs (24 warps) per SM
-    if (const char* e = getenv("SPMV_COO_MINB")) minb = atoi(e) >= 4 ? 4 : 3;  // dev knob
     const bool zg = !p->coo_memset;
     if (!zg) SPMV_CUDA(cudaMemsetAsync(y, 0, sizeof(float) * (size_t)p->nrows, s));
-    auto k = zg ? (ef ? (minb == 4 ? k_coo_w<1, 4, true> : k_coo_w<1, 3, true>)
-                      : (minb == 4 ? k_coo_w<0, 4, true> : k_coo_w<0, 3, true>))
-                : (ef ? (minb == 4 ? k_coo_w<1, 4, false> : k_coo_w<1, 3, false>)
-                      : (minb == 4 ? k_coo_w<0, 4, false> : k_coo_w<0, 3, false>));
+    // 16 entries per lane: <= 85 registers, 3 CTAs (24 warps) per SM;
+    // 8 entries per lane: <= 51 registers, 5 CTAs (40 warps) per SM
+    auto k = E == 8 ? (zg ? (ef ? k_coo_w<1, 5, true, 8> : k_coo_w<0, 5, true, 8>)
+                          : (ef ? k_coo_w<1, 5, false, 8> : k_coo_w<0, 5, false, 8>))
+                    : (zg ? (ef ? k_coo_w<1, 3, true, 16> : k_coo_w<0, 3, true, 16>)
+                          : (ef ? k_coo_w<1, 3, false, 16> : k_coo_w<0, 3, false, 16>));
     k<<<g, 256, 0, s>>>(p->d_coo_row, p->d_col, p->d_val, x, y, p->nnz_local, p->nrows, T, frow,
                         lrow, fpart, lpart, p->d_coo_tflag);
   }

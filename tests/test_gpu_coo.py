@@ -54,12 +54,14 @@ def _edge_matrices():
 ALL = CASES + [(nm, (lambda m=m: m)) for nm, m in _edge_matrices()]
 
 
-@pytest.mark.parametrize("variant", ["1", "2"])
+@pytest.mark.parametrize("variant", ["1", "2", "2e8"])
 @pytest.mark.parametrize("name,make", ALL)
 def test_coo_matches_oracle(dev, name, make, variant, monkeypatch):
-    """variant 1: CTA tiles of 2048 entries (k_coo); 2: warp tiles of 512
-    (k_coo_w, the default) -- SPMV_COO_V dev knob."""
-    monkeypatch.setenv("SPMV_COO_V", variant)
+    """variant 1: CTA tiles of 2048 entries (k_coo); 2: warp tiles of 32 x 16
+    entries (k_coo_w, the default); 2e8: warp tiles of 32 x 8 -- SPMV_COO_V /
+    SPMV_COO_E dev knobs."""
+    monkeypatch.setenv("SPMV_COO_V", variant[0])
+    monkeypatch.setenv("SPMV_COO_E", "8" if variant == "2e8" else "16")
     A = make()
     perm = rabbit.random_perm(A.n, 21) if A.nnz and name not in ("edges", "lastrow") else None
     P = mk_plan(A, perm, dev)
