@@ -414,7 +414,7 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 }
 
 // ------------------------------------------------------------- long rows
-template <typename OT, bool SS, int HOT>
+template <typename OT, bool SS, int HOT, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
@@ -431,21 +431,22 @@ __global__ void __launch_bounds__(256)
     const int32_t* cc = col + b;
     const float* vv = val + b;
     float s = 0.f;
-    // four strided entries in flight per lane, the ragged end guarded: a slot
+    // UNR strided entries in flight per lane, the ragged end guarded: a slot
     // past the row adds +0, which leaves s unchanged (s starts at +0 and is
-    // never -0), so the association is exactly j, j+32, j+64, ...
-    for (int j = lane; j < L; j += 128) {
-      const bool p1 = j + 32 < L, p2 = j + 64 < L, p3 = j + 96 < L;
-      const int c0 = __ldcs(cc + j), c1 = p1 ? __ldcs(cc + j + 32) : 0,
-                c2 = p2 ? __ldcs(cc + j + 64) : 0, c3 = p3 ? __ldcs(cc + j + 96) : 0;
-      const float v0 = __ldcs(vv + j), v1 = p1 ? __ldcs(vv + j + 32) : 0.f,
-                  v2 = p2 ? __ldcs(vv + j + 64) : 0.f, v3 = p3 ? __ldcs(vv + j + 96) : 0.f;
-      const float x0 = gx<HOT>(x, xh, c0), x1 = p1 ? gx<HOT>(x, xh, c1) : 0.f,
-                  x2 = p2 ? gx<HOT>(x, xh, c2) : 0.f, x3 = p3 ? gx<HOT>(x, xh, c3) : 0.f;
-      s = __fadd_rn(s, __fmul_rn(v0, x0));
-      s = __fadd_rn(s, __fmul_rn(v1, x1));
-      s = __fadd_rn(s, __fmul_rn(v2, x2));
-      s = __fadd_rn(s, __fmul_rn(v3, x3));
+    // never -0), so the association is exactly j, j+32, j+64, ... for any UNR
+    for (int j = lane; j < L; j += 32 * UNR) {
+      int c[UNR];
+      float v[UNR], xv[UNR];
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) {
+        const bool pu = j + 32 * u < L;
+        c[u] = pu ? __ldcs(cc + j + 32 * u) : 0;
+        v[u] = pu ? __ldcs(vv + j + 32 * u) : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) xv[u] = (j + 32 * u < L) ? gx<HOT>(x, xh, c[u]) : 0.f;
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
     }
     s = warp_tree(s);
     if (lane == 0) {
@@ -506,27 +507,27 @@ __global__ void __launch_bounds__(1024, 1)
 }
 
 // canonical W = 256 sum of entries [b, b + L) of a row
-template <int HOT>
+template <int HOT, int UNR = 4>
 __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             const float* __restrict__ val,
                                             const float* __restrict__ x, int64_t b, int64_t L,
                                             float* red, const float* __restrict__ xh) {
   const int tid = threadIdx.x;
   float s = 0.f;
-  // four strided entries in flight, ragged end guarded (+0 slots, as k_warp_rows)
-  for (int64_t t = tid; t < L; t += 1024) {
-    const bool p1 = t + 256 < L, p2 = t + 512 < L, p3 = t + 768 < L;
-    const int c0 = __ldcs(col + b + t), c1 = p1 ? __ldcs(col + b + t + 256) : 0,
-              c2 = p2 ? __ldcs(col + b + t + 512) : 0, c3 = p3 ? __ldcs(col + b + t + 768) : 0;
-    const float v0 = __ldcs(val + b + t), v1 = p1 ? __ldcs(val + b + t + 256) : 0.f,
-                v2 = p2 ? __ldcs(val + b + t + 512) : 0.f,
-                v3 = p3 ? __ldcs(val + b + t + 768) : 0.f;
-    const float x0 = gx<HOT>(x, xh, c0), x1 = p1 ? gx<HOT>(x, xh, c1) : 0.f,
-                x2 = p2 ? gx<HOT>(x, xh, c2) : 0.f, x3 = p3 ? gx<HOT>(x, xh, c3) : 0.f;
-    s = __fadd_rn(s, __fmul_rn(v0, x0));
-    s = __fadd_rn(s, __fmul_rn(v1, x1));
-    s = __fadd_rn(s, __fmul_rn(v2, x2));
-    s = __fadd_rn(s, __fmul_rn(v3, x3));
+  // UNR strided entries in flight, ragged end guarded (+0 slots, as k_warp_rows)
+  for (int64_t t = tid; t < L; t += 256 * UNR) {
+    int c[UNR];
+    float v[UNR], xv[UNR];
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) {
+      const bool pu = t + 256 * u < L;
+      c[u] = pu ? __ldcs(col + b + t + 256 * u) : 0;
+      v[u] = pu ? __ldcs(val + b + t + 256 * u) : 0.f;
+    }
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) xv[u] = (t + 256 * u < L) ? gx<HOT>(x, xh, c[u]) : 0.f;
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
   }
   red[tid] = s;
   __syncthreads();
@@ -540,7 +541,7 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
   return r;  // valid in thread 0
 }
 
-template <typename OT, bool SS, int HOT>
+template <typename OT, bool SS, int HOT, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_cta_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
@@ -549,7 +550,7 @@ __global__ void __launch_bounds__(256)
   __shared__ float red[256];
   const int r = rows[blockIdx.x];
   const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
-  const float s = cta_sum256<HOT>(col, val, x, b, L, red, xh);
+  const float s = cta_sum256<HOT, UNR>(col, val, x, b, L, red, xh);
   if (threadIdx.x == 0) {
     const float v = __fmul_rn(s, alpha_of(ss_in));
     store_y<SS>(y, dst, r, v);
@@ -558,7 +559,7 @@ __global__ void __launch_bounds__(256)
   }
 }
 
-template <typename OT, int HOT>
+template <typename OT, int HOT, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_hub_chunk(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
@@ -570,7 +571,7 @@ __global__ void __launch_bounds__(256)
   const int64_t rb = (int64_t)rp[r], L = (int64_t)rp[r + 1] - rb;
   const int64_t b = rb + (int64_t)chunk_idx[c] * HUB_CHUNK;
   const int64_t m = min((int64_t)HUB_CHUNK, rb + L - b);
-  const float s = cta_sum256<HOT>(col, val, x, b, m, red, xh);
+  const float s = cta_sum256<HOT, UNR>(col, val, x, b, m, red, xh);
   if (threadIdx.x == 0) part[c] = (double)s;
 }
 
@@ -931,8 +932,14 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
         rp, p->d_col_hot, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh, (int)p->hot_S);
   } else if (nw) {
     const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
-    k_warp_rows<OT, SS, HG><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh,
-                                               dst);
+    int unr = 4;  // entries in flight per lane (same association for any value)
+    if (const char* e = getenv("SPMV_WARP_UNR")) unr = atoi(e) == 8 ? 8 : 4;  // dev knob
+    if (unr == 8)
+      k_warp_rows<OT, SS, HG, 8><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss,
+                                                    p->d_xh, dst);
+    else
+      k_warp_rows<OT, SS, HG, 4><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss,
+                                                    p->d_xh, dst);
   }
   const bool long_smem = HOT == 3 && (p->n_cta || p->n_chunks);
   if (long_smem) {
@@ -950,16 +957,24 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
         rp, p->d_col_hot, p->d_val, x, y, p->d_cta_rows, p->n_cta, p->d_chunk_row,
         p->d_chunk_idx, p->n_chunks, p->d_chunk_part, ss_in, p->d_cta_ss, p->d_xh,
         (int)p->hot_S);
-  } else if (p->n_cta) {
-    k_cta_rows<OT, SS, HG><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
-                                                               p->d_cta_rows, ss_in, p->d_cta_ss,
-                                                               p->d_xh, dst);
+  }
+  int cunr = 4;  // entries in flight per thread (same association for any value)
+  if (const char* e = getenv("SPMV_CTA_UNR")) cunr = atoi(e) == 8 ? 8 : 4;  // dev knob
+  if (!long_smem && p->n_cta) {
+    if (cunr == 8)
+      k_cta_rows<OT, SS, HG, 8><<<(unsigned)p->n_cta, 256, 0, s2>>>(
+          rp, col, p->d_val, x, y, p->d_cta_rows, ss_in, p->d_cta_ss, p->d_xh, dst);
+    else
+      k_cta_rows<OT, SS, HG, 4><<<(unsigned)p->n_cta, 256, 0, s2>>>(
+          rp, col, p->d_val, x, y, p->d_cta_rows, ss_in, p->d_cta_ss, p->d_xh, dst);
   }
   if (p->n_chunks) {
-    if (!long_smem)
-      k_hub_chunk<OT, HG><<<(unsigned)p->n_chunks, 256, 0, s2>>>(rp, col, p->d_val, x,
-                                                                 p->d_chunk_row, p->d_chunk_idx,
-                                                                 p->d_chunk_part, p->d_xh);
+    if (!long_smem && cunr == 8)
+      k_hub_chunk<OT, HG, 8><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
+          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part, p->d_xh);
+    else if (!long_smem)
+      k_hub_chunk<OT, HG, 4><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
+          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part, p->d_xh);
     const unsigned g = (unsigned)((p->n_hub + 127) / 128);
     if (SS)
       k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
