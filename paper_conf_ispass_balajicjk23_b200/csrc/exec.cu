@@ -18,6 +18,7 @@
 //   k_ss_final   fixed-order fp64 sum of per-tile / per-row y^2 partials
 //                (power-iteration norm; deterministic).
 // No tensor cores: SpMV is not a dense contraction (AI <= 0.25 flop/B).
+#include <atomic>
 #include <cmath>
 #include <cstdlib>
 
@@ -712,15 +713,21 @@ int hot_mode(const spmv_plan_s* p) {
   return m;
 }
 
+// cudaFuncSetAttribute acts on the current device, so the max-dynamic-smem
+// opt-in is remembered per (kernel instantiation, device), thread-safely
+template <auto K>
+void max_dyn_smem(int bytes, int device) {
+  static std::atomic<uint64_t> done{0};
+  const uint64_t bit = 1ull << (device & 63);
+  if (done.load(std::memory_order_acquire) & bit) return;
+  SPMV_CUDA(cudaFuncSetAttribute(K, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes));
+  done.fetch_or(bit, std::memory_order_release);
+}
+
 template <typename OT, bool SS>
 void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s) {
   constexpr size_t smem = sizeof(PanelSmem);
-  static bool attr = false;
-  if (!attr) {
-    SPMV_CUDA(cudaFuncSetAttribute(k_panel<OT, SS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                   (int)smem));
-    attr = true;
-  }
+  max_dyn_smem<k_panel<OT, SS>>((int)smem, p->device);
   static int per_sm = 0;
   if (!per_sm) {
     SPMV_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_panel<OT, SS>, PT_THREADS,
@@ -920,13 +927,7 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
   double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
   if (nw && HOT == 3) {
-    static bool attr = false;
-    if (!attr) {
-      SPMV_CUDA(cudaFuncSetAttribute(k_warp_rows_smem<OT, SS>,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)(sizeof(float) * HOT_MAX)));
-      attr = true;
-    }
+    max_dyn_smem<k_warp_rows_smem<OT, SS>>((int)(sizeof(float) * HOT_MAX), p->device);
     const size_t smem = sizeof(float) * (size_t)p->hot_S;
     k_warp_rows_smem<OT, SS><<<(unsigned)num_sms(p->device), 1024, smem, s1>>>(
         rp, p->d_col_hot, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh, (int)p->hot_S);
@@ -943,13 +944,7 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   }
   const bool long_smem = HOT == 3 && (p->n_cta || p->n_chunks);
   if (long_smem) {
-    static bool attr = false;
-    if (!attr) {
-      SPMV_CUDA(cudaFuncSetAttribute(k_long_rows_smem<OT, SS>,
-                                     cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     (int)(sizeof(float) * HOT_MAX)));
-      attr = true;
-    }
+    max_dyn_smem<k_long_rows_smem<OT, SS>>((int)(sizeof(float) * HOT_MAX), p->device);
     const size_t smem = sizeof(float) * (size_t)p->hot_S;
     const int64_t items = p->n_cta + p->n_chunks;
     const unsigned g = (unsigned)std::min<int64_t>((items + 3) / 4, num_sms(p->device));
