@@ -24,8 +24,11 @@ here from DESIGN.md §Plan, not imported from the library:
 H: the length of the leading run of columns j of B with
 colcnt_B[j] * N > NZ_B (the hot, hub-grouped prefix of x under RABBIT++).
 
-Partition: b_0 = 0, b_G = N,
-b_k = lower_bound(row_ptr_B, ceil(k * NZ / G)) for 0 < k < G.
+Partition (SURVEY.md §8(e) "nnz-balanced" row blocks, refined by reading c29 of
+DESIGN.md §2 to balance each rank's compulsory bytes of PAPER.md:96 -- 8 B per
+entry (col, val) and w_off + 8 B per row (row_ptr, x, y), w_off = 8 when
+NZ >= 2^31 else 4): with c(r) = 8 * row_ptr_B[r] + (w_off + 8) * r,
+b_0 = 0, b_G = N, b_k = min{ r : c(r) >= ceil(k * c(N) / G) } for 0 < k < G.
 
 TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).
 """
@@ -117,9 +120,11 @@ def partition(row_ptr, G: int) -> np.ndarray:
     row_ptr = np.asarray(row_ptr, np.int64)
     n = len(row_ptr) - 1
     nnz = int(row_ptr[-1])
+    w_off = 8 if nnz >= 2**31 else 4
+    cost = 8 * row_ptr + (w_off + 8) * np.arange(n + 1, dtype=np.int64)   # c(r), r = 0..N
     b = np.zeros(G + 1, np.int64)
     b[G] = n
     for k in range(1, G):
-        target = -(-(k * nnz) // G)
-        b[k] = int(np.searchsorted(row_ptr, target, side="left"))
+        target = -(-(k * int(cost[n])) // G)
+        b[k] = int(np.searchsorted(cost, target, side="left"))
     return b

@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 SO = os.path.join(HERE, "libspmv.so")
-SOURCES = ["api.cu", "plan.cu", "exec.cu", "spmm.cu", "coo.cu", "reorder.cpp"]
+SOURCES = ["api.cu", "plan.cu", "exec.cu", "iterate.cu", "spmm.cu", "coo.cu", "reorder.cpp"]
 HEADERS = ["common.cuh", "plan.cuh"]
 
 
@@ -57,7 +57,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
             sys.stderr.write(r.stderr)
         objs.append(obj)
     tmp = SO + ".tmp"
-    cmd = [cc, "-shared", "-o", tmp] + objs + ["-Xcompiler", "-fopenmp", "-lgomp", "-lcudart"]
+    cmd = [cc, "-shared", "-o", tmp] + objs + ["-Xcompiler", "-fopenmp", "-lgomp", "-lcudart", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)

@@ -18,6 +18,10 @@ const char* get_error() { return g_err.c_str(); }
   catch (const spmv::Err& e) {                              \
     return e.st;                                            \
   }                                                         \
+  catch (const std::bad_alloc&) {                           \
+    spmv::set_error("out of host memory");                  \
+    return SPMV_ENOMEM;                                     \
+  }                                                         \
   catch (const std::exception& e) {                         \
     spmv::set_error(std::string("internal: ") + e.what());  \
     return SPMV_EINVAL;                                     \
@@ -132,6 +136,7 @@ spmv_status spmv_exec(spmv_plan_t p, const float* x_B, float* y_B, void* stream)
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec: NULL plan");
   if (p->nrows && (!x_B || !y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec: NULL vector");
+  use_device(p);
   spmv::exec(p, x_B, y_B, nullptr, nullptr, S(stream));
   API_END
 }
@@ -153,6 +158,7 @@ spmv_status spmv_exec_spmm4(spmv_plan_t p, const float* X_B, float* Y_B, void* s
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_spmm4: NULL plan");
   if (p->nrows && (!X_B || !Y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_spmm4: NULL matrix");
+  use_device(p);
   spmv::exec_spmm4(p, X_B, Y_B, S(stream));
   API_END
 }
@@ -228,6 +234,7 @@ spmv_status spmv_exec_scaled(spmv_plan_t p, const float* x_B, float* y_B,
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled: NULL plan");
   if (p->nrows && (!x_B || !y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled: NULL vector");
+  use_device(p);
   spmv::exec(p, x_B, y_B, sumsq_in, sumsq_out, S(stream));
   API_END
 }
@@ -246,6 +253,15 @@ spmv_status spmv_scale_vec(const float* u, float* x, int64_t n, const double* su
   API_BEGIN
   if (n < 0 || (n && (!u || !x))) SPMV_FAIL(SPMV_EINVAL, "spmv_scale_vec: bad argument");
   spmv::scale_vec(u, x, n, sumsq_in, S(stream));
+  API_END
+}
+
+spmv_status spmv_iterate_finish(const float* u, float* x, int64_t n, const double* sumsq_dev,
+                                double* lambda_out, void* stream) {
+  API_BEGIN
+  if (n < 0 || (n && (!u || !x)) || !sumsq_dev)
+    SPMV_FAIL(SPMV_EINVAL, "spmv_iterate_finish: bad argument");
+  spmv::iterate_finish(u, x, n, sumsq_dev, lambda_out, S(stream));
   API_END
 }
 

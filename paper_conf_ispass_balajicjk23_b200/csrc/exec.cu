@@ -687,14 +687,6 @@ __global__ void __launch_bounds__(1024)
   }
 }
 
-__global__ void k_scale(const float* __restrict__ u, float* __restrict__ x, int64_t n,
-                        const double* __restrict__ ss) {
-  const float a = alpha_of(ss);
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (int64_t)gridDim.x * blockDim.x)
-    x[i] = __fmul_rn(u[i], a);
-}
-
 int g_num_sms = 0;
 
 int num_sms(int dev) {
@@ -833,8 +825,10 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
       if (L <= SHORT_MAX) {  // longer rows: k_warp_rows / k_cta_rows / k_hub_*
         mine = true;
         // Every slot of a chunk holds a valid column of some row (or the zero
-        // tail padding), so its x read is always safe; slots outside [a, e)
-        // get x = 0, an exact +-0 product (res starts at +0, never -0).
+        // tail padding), so its x read is always safe; a slot outside [a, e)
+        // contributes the product +0 (selected, not computed: a neighbouring
+        // row's Inf / NaN value never reaches this row, Alg. 1), which leaves
+        // res unchanged (it starts at +0 and is never -0).
         const int32_t* cp = col + (a & ~(OT)7);
         const float* vp = val + (a & ~(OT)7);
         const int lo = (int)(a & 7), hi = lo + L;
@@ -852,7 +846,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
             const float xv = gx<HOT>(x, xh, cc[i]);
-            res = __fadd_rn(res, __fmul_rn(vv[i], (k + i >= lo && k + i < hi) ? xv : 0.f));
+            res = __fadd_rn(res, (k + i >= lo && k + i < hi) ? __fmul_rn(vv[i], xv) : 0.f);
           }
         }
       }
@@ -1149,47 +1143,6 @@ void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double*
   set_window(p, x, s);
   if (p->off64) exec_typed<int64_t>(p, x, y, ss_in, ss_out, s, dst);
   else exec_typed<int32_t>(p, x, y, ss_in, ss_out, s, dst);
-}
-
-void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s) {
-  if (iters < 1) SPMV_FAIL(SPMV_EINVAL, "iters must be >= 1");
-  if (p->world != 1)
-    SPMV_FAIL(SPMV_EUNSUPPORTED,
-              "spmv_iterate drives world == 1; use spmv_exec_scaled + collectives for world > 1");
-  if (!p->permuted) SPMV_FAIL(SPMV_ESTATE, "spmv_iterate before spmv_permute");
-  if (!p->d_u) {
-    void* q = nullptr;
-    if (cudaMalloc(&q, sizeof(float) * (size_t)std::max<int64_t>(p->x_len, 1)) != cudaSuccess) {
-      cudaGetLastError();
-      SPMV_FAIL(SPMV_ENOMEM, "iterate buffer allocation failed");
-    }
-    p->d_u = (float*)q;
-  }
-  float* a = x;
-  float* b = p->d_u;
-  const double* sin = nullptr;
-  for (int t = 0; t < iters; ++t) {
-    double* sout = p->d_ss + (t & 1);
-    exec(p, a, b, sin, sout, s);
-    sin = sout;
-    std::swap(a, b);
-  }
-  if (p->n) {
-    int g = (int)std::min<int64_t>((p->n + 255) / 256, 148 * 16);
-    k_scale<<<g, 256, 0, s>>>(a, x, p->n, sin);
-    SPMV_LAUNCH_CHECK();
-  }
-  double ss = 0.0;
-  SPMV_CUDA(cudaMemcpyAsync(&ss, sin, sizeof(double), cudaMemcpyDeviceToHost, s));
-  SPMV_CUDA(cudaStreamSynchronize(s));
-  if (lambda) *lambda = std::sqrt(ss);
-}
-
-void scale_vec(const float* u, float* x, int64_t n, const double* ss, cudaStream_t s) {
-  if (n <= 0) return;
-  int g = (int)std::min<int64_t>((n + 255) / 256, 148 * 16);
-  k_scale<<<g, 256, 0, s>>>(u, x, n, ss);
-  SPMV_LAUNCH_CHECK();
 }
 
 }  // namespace spmv

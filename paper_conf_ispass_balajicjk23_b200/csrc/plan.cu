@@ -176,18 +176,26 @@ void exclusive_scan(const T* in, int64_t n, int64_t* out, int64_t* temp, cudaStr
 int64_t scan_temp_len(int64_t n) { return (n + SCAN_B - 1) / SCAN_B + 2; }
 
 // ---------------------------------------------------------------- partition
-__global__ void k_partition(const int64_t* rpB, int64_t n, int64_t nnz, int G, int64_t* b) {
-  int k = threadIdx.x;
-  if (k > G) return;
-  if (k == 0) { b[0] = 0; return; }
-  if (k == G) { b[G] = n; return; }
-  int64_t target = ((int64_t)k * nnz + G - 1) / G;
-  int64_t lo = 0, hi = n;
-  while (lo < hi) {
-    int64_t mid = (lo + hi) >> 1;
-    if (rpB[mid] >= target) hi = mid; else lo = mid + 1;
+// Row blocks balanced on compulsory bytes (reading c29): row r
+// starts at byte offset cost(r) = 8 row_ptr_B[r] + (w_off + 8) r of the P:96
+// traffic (col + val per entry; row_ptr, x and y per row), and
+// b_k = lower_bound(cost, ceil(k * cost(n) / G)).  cost is strictly increasing,
+// so every block is a contiguous row range and b_0 = 0, b_G = n.  Grid-stride
+// over k in [0, G] (G + 1 bounds).
+__global__ void k_partition(const int64_t* rpB, int64_t n, int64_t nnz, int G, int64_t w_off,
+                            int64_t* b) {
+  const int64_t wr = w_off + 8, total = 8 * nnz + wr * n;
+  for (int k = blockIdx.x * blockDim.x + threadIdx.x; k <= G; k += gridDim.x * blockDim.x) {
+    if (k == 0) { b[0] = 0; continue; }
+    if (k == G) { b[G] = n; continue; }
+    const int64_t target = ((int64_t)k * total + G - 1) / G;
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+      const int64_t mid = (lo + hi) >> 1;
+      if (8 * rpB[mid] + wr * mid >= target) hi = mid; else lo = mid + 1;
+    }
+    b[k] = lo;
   }
-  b[k] = lo;
 }
 
 template <typename OT>
@@ -735,9 +743,10 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   exclusive_scan<int64_t>(lenB, n, rpB, tmp, s);
   dfree(lenB);
 
-  // partition: b_k = lower_bound(row_ptr_B, ceil(k NZ / G))
+  // partition (reading c29): compulsory bytes balanced
   int64_t* d_part = dalloc<int64_t>(p->world + 1);
-  k_partition<<<1, 1024, 0, s>>>(rpB, n, nnz, p->world, d_part);
+  k_partition<<<(unsigned)((p->world + 256) / 256), 256, 0, s>>>(rpB, n, nnz, p->world,
+                                                                  p->off64 ? 8 : 4, d_part);
   p->part.assign(p->world + 1, 0);
   SPMV_CUDA(cudaMemcpyAsync(p->part.data(), d_part, sizeof(int64_t) * (p->world + 1),
                             cudaMemcpyDeviceToHost, s));
@@ -752,7 +761,7 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   SPMV_CUDA(cudaStreamSynchronize(s));
   p->nnz_before = lo_nz;
   p->nnz_local = hi_nz - lo_nz;
-  if (p->world > 1) {
+  if (p->world > 1 && p->opts.x_layout == SPMV_XLAYOUT_PADDED) {
     int64_t M = 0;
     for (int k = 0; k < p->world; ++k) M = std::max<int64_t>(M, p->part[k + 1] - p->part[k]);
     M = (M + 31) / 32 * 32;
@@ -761,10 +770,10 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
     p->x_stride = M;
     p->x_len = (int64_t)p->world * M;
     p->y_offset = (int64_t)p->rank * M;
-  } else {
+  } else {  // global layout: x_B indexed by B's row id, this rank's y at row_begin
     p->x_stride = n;
     p->x_len = n;
-    p->y_offset = 0;
+    p->y_offset = p->row_begin;
   }
 
   // local row pointer
@@ -942,7 +951,7 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
                                                         p->d_col_hot);
     SPMV_LAUNCH_CHECK();
   }
-  if (p->world > 1 && p->nnz_local) {
+  if (padded(p) && p->nnz_local) {
     int64_t* d_part = dalloc<int64_t>(p->world + 1);
     SPMV_CUDA(cudaMemcpyAsync(d_part, p->part.data(), 8 * (p->world + 1), cudaMemcpyHostToDevice, s));
     k_pad_cols<<<grid_for(p->nnz_local), TPB, 0, s>>>(p->d_col, p->nnz_local, d_part, p->world,
@@ -1074,6 +1083,10 @@ void permute_vec(spmv_plan_s* p, const float* in, float* out, int inverse, cudaS
 
 void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStream_t s) {
   if (p->n == 0) return;
+  if (!padded(p)) {  // global layout: the padded form is the vector itself
+    SPMV_CUDA(cudaMemcpyAsync(out, in, 4 * p->n, cudaMemcpyDeviceToDevice, s));
+    return;
+  }
   int64_t* d_part = dalloc<int64_t>(p->world + 1);
   SPMV_CUDA(cudaMemcpyAsync(d_part, p->part.data(), 8 * (p->world + 1), cudaMemcpyHostToDevice, s));
   k_pad_vec<<<grid_for(p->n), TPB, 0, s>>>(d_part, p->world, p->x_stride, p->n, in, out, to_padded);

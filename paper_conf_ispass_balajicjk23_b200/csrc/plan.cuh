@@ -100,6 +100,13 @@ struct spmv_plan_s {
   bool conc = false, conc_init = false;
   bool stream_ef = false;  // k_lane streams col/val with L2::evict_first (plan decision)
 
+  // power iteration across ranks (iterate.cu): collective backend
+  // (spmv_set_coll, else NCCL on opts.nccl_comm) and the peer next-x buffers
+  // of SPMV_EXCHANGE_PEER (spmv_set_peers), [j * world + k]
+  spmv_coll_t coll{};
+  bool has_coll = false;
+  std::vector<float*> peers;
+
   // state
   bool permuted = false;
   int64_t l2_window_bytes = 0;
@@ -108,6 +115,11 @@ struct spmv_plan_s {
 };
 
 namespace spmv {
+// x layout of a multi-rank plan (opts.x_layout): padded slices of M floats per
+// rank, or (default) B's own row ids, x_len = n
+inline bool padded(const spmv_plan_s* p) {
+  return p->world > 1 && p->opts.x_layout == SPMV_XLAYOUT_PADDED;
+}
 void plan_build(spmv_plan_s* p, const spmv_csr_t* A, const int32_t* perm);
 void rabbitpp_gpu(const spmv_csr_t* A, const int32_t* perm_rabbit, const int32_t* comm,
                   int32_t* perm_out, cudaStream_t s);
@@ -118,6 +130,8 @@ void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStr
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
           cudaStream_t s, float* const* bcast = nullptr, int nbcast = 0);
 void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s);
+void iterate_finish(const float* u, float* x, int64_t n, const double* ss, double* lambda,
+                    cudaStream_t s);
 int exec_launches(const spmv_plan_s* p, bool ss);
 void exec_spmm4(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s);
 int spmm4_launches(const spmv_plan_s* p);

@@ -19,12 +19,15 @@
 #include <omp.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdio>
 #include <cstdlib>
 #include <chrono>
 #include <cmath>
 #include <cstring>
+#include <memory>
 #include <numeric>
+#include <stdexcept>
 #include <string>
 #include <vector>
 
@@ -125,12 +128,55 @@ struct Edge {
   int64_t w;
 };
 
-struct Rabbit {
-  std::vector<int32_t> perm, comm;
-  int64_t two_m = 0, n_merges = 0, n_top = 0;
+struct MergeRec {  // one merge of the dendrogram: child u into root v, exact gain dQ'
+  int32_t u, v;
+  __int128 dq;
 };
 
-Rabbit rabbit_detect(const Sym& S) {
+struct Rabbit {
+  std::vector<int32_t> perm, comm;
+  int64_t two_m = 0, n_merges = 0, n_top = 0, n_deferred = 0, n_retries = 0;
+  bool parallel = false;
+  std::vector<MergeRec> log;  // filled when requested (SPMV_REORDER_LOG)
+};
+
+// ascending (deg, id) order of the vertices (reading c7): stable counting sort
+std::vector<int64_t> degree_order(const std::vector<int64_t>& deg) {
+  const int64_t n = (int64_t)deg.size();
+  int64_t maxd = 0;
+  for (int64_t v = 0; v < n; ++v) maxd = std::max(maxd, deg[v]);
+  std::vector<int64_t> order(n);
+  std::vector<int64_t> c(maxd + 2, 0);
+  for (int64_t v = 0; v < n; ++v) c[deg[v] + 1]++;
+  for (int64_t d = 0; d <= maxd; ++d) c[d + 1] += c[d];
+  for (int64_t v = 0; v < n; ++v) order[c[deg[v]]++] = v;
+  return order;
+}
+
+// pre-order DFS of the dendrogram (reading c10): roots in `top` order,
+// children in merge order
+void dendrogram_ids(const std::vector<int32_t>& top, const std::vector<int32_t>& first_child,
+                    const std::vector<int32_t>& next_sib, Rabbit& R, int64_t n) {
+  R.perm.assign(n, -1);
+  R.comm.assign(n, -1);
+  int32_t nxt = 0;
+  std::vector<int32_t> st;
+  for (int32_t r : top) {
+    st.push_back(r);
+    while (!st.empty()) {
+      int32_t x = st.back();
+      st.pop_back();
+      R.perm[x] = nxt++;
+      R.comm[x] = r;
+      size_t mark = st.size();
+      for (int32_t c = first_child[x]; c != -1; c = next_sib[c]) st.push_back(c);
+      std::reverse(st.begin() + mark, st.end());
+    }
+  }
+  R.n_top = (int64_t)top.size();
+}
+
+Rabbit rabbit_detect(const Sym& S, bool want_log) {
   const int64_t n = S.n;
   std::vector<int64_t> deg(n);
 #pragma omp parallel for schedule(static)
@@ -141,16 +187,7 @@ Rabbit rabbit_detect(const Sym& S) {
   }
   int64_t two_m = 0;
   for (int64_t v = 0; v < n; ++v) two_m += deg[v];
-  // ascending (deg, id): stable counting sort by degree
-  int64_t maxd = 0;
-  for (int64_t v = 0; v < n; ++v) maxd = std::max(maxd, deg[v]);
-  std::vector<int64_t> order(n);
-  {
-    std::vector<int64_t> c(maxd + 2, 0);
-    for (int64_t v = 0; v < n; ++v) c[deg[v] + 1]++;
-    for (int64_t d = 0; d <= maxd; ++d) c[d + 1] += c[d];
-    for (int64_t v = 0; v < n; ++v) order[c[deg[v]]++] = v;
-  }
+  const std::vector<int64_t> order = degree_order(deg);
   std::vector<int32_t> parent(n);
   std::iota(parent.begin(), parent.end(), 0);
   auto find = [&](int32_t v) {
@@ -222,30 +259,241 @@ Rabbit rabbit_detect(const Sym& S) {
       agg[u].reserve(touched.size());
       for (int32_t r : touched) agg[u].push_back({r, acc[r]});
       R.n_merges++;
+      if (want_log) R.log.push_back({u, best, bestdq});
     } else {
       top.push_back(u);
     }
     for (int32_t r : touched) acc[r] = 0;
   }
-  // pre-order DFS of the dendrogram
-  R.perm.assign(n, -1);
-  R.comm.assign(n, -1);
-  int32_t nxt = 0;
-  std::vector<int32_t> st;
-  for (int32_t r : top) {
-    st.push_back(r);
-    while (!st.empty()) {
-      int32_t x = st.back();
-      st.pop_back();
-      R.perm[x] = nxt++;
-      R.comm[x] = r;
-      // push children in reverse merge order so they pop in merge order
-      size_t mark = st.size();
-      for (int32_t c = first_child[x]; c != -1; c = next_sib[c]) st.push_back(c);
-      std::reverse(st.begin() + mark, st.end());
+  dendrogram_ids(top, first_child, next_sib, R, n);
+  return R;
+}
+
+// ------------------------------------------------ concurrent merges (f4)
+// Rabbit Order's parallel incremental aggregation (ref [1], PAPER.md:259;
+// SURVEY §8(f4)): threads take vertices in the same ascending (deg, id) order
+// (dynamic chunks) and run the sequential step on each, with three states in
+// tot[] besides a community's total degree:
+//   PROC    u is being aggregated: nothing merges into u meanwhile, so u's
+//           children (all merged before) are final;
+//   MLOCK   short critical section of a merge into v;
+//   MERGED  u is no longer a root.
+// A merge u -> v locks v (CAS from a valid total), recomputes the EXACT
+// weight w(C_u, C_v) from u's aggregated list with the current union-find
+// roots (v's community cannot change under the lock, u's cannot change while
+// PROC), and merges only if dQ' = 2m w - tot_u tot_v > 0 -- so every recorded
+// gain is the exact change of Q'/2 and Q'_final - Q'_init = 2 sum dQ' holds.
+// A target that is being processed (PROC) defers u; deferred vertices are
+// processed sequentially afterwards, in order.  The result depends on thread
+// timing (not bit-exact with the oracle); tests check it by these invariants.
+struct HashAcc {  // per-thread (root -> summed weight) map, open addressing
+  std::vector<int32_t> key;
+  std::vector<int64_t> val;
+  std::vector<uint32_t> used;
+  uint32_t mask = 0;
+  void prepare(size_t expect) {
+    size_t cap = 64;
+    while (cap < 2 * expect) cap <<= 1;
+    if (cap > key.size()) {
+      key.assign(cap, -1);
+      val.assign(cap, 0);
+      mask = (uint32_t)(cap - 1);
     }
   }
-  R.n_top = (int64_t)top.size();
+  inline void add(int32_t r, int64_t w) {
+    uint32_t h = ((uint32_t)r * 2654435761u) & mask;
+    while (key[h] != -1 && key[h] != r) h = (h + 1) & mask;
+    if (key[h] == -1) {
+      key[h] = r;
+      used.push_back(h);
+    }
+    val[h] += w;
+  }
+  void clear() {
+    for (uint32_t h : used) {
+      key[h] = -1;
+      val[h] = 0;
+    }
+    used.clear();
+  }
+};
+
+Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
+  const int64_t n = S.n;
+  constexpr int64_t PROC = -1, MLOCK = -2, MERGED = -3;
+  std::vector<int64_t> deg(n);
+#pragma omp parallel for schedule(static)
+  for (int64_t v = 0; v < n; ++v) {
+    int64_t d = 0;
+    for (int64_t k = S.ptr[v]; k < S.ptr[v + 1]; ++k) d += S.w[k];
+    deg[v] = d;
+  }
+  int64_t two_m = 0;
+#pragma omp parallel for reduction(+ : two_m) schedule(static)
+  for (int64_t v = 0; v < n; ++v) two_m += deg[v];
+  const std::vector<int64_t> order = degree_order(deg);
+  std::vector<int64_t> pos(n);
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < n; ++i) pos[order[i]] = i;
+  std::unique_ptr<std::atomic<int64_t>[]> tot(new std::atomic<int64_t>[n]);
+  std::unique_ptr<std::atomic<int32_t>[]> parent(new std::atomic<int32_t>[n]);
+#pragma omp parallel for schedule(static)
+  for (int64_t v = 0; v < n; ++v) {
+    tot[v].store(deg[v], std::memory_order_relaxed);
+    parent[v].store((int32_t)v, std::memory_order_relaxed);
+  }
+  // written only under the target's MLOCK (or by u's own thread while PROC)
+  std::vector<int32_t> first_child(n, -1), last_child(n, -1), next_sib(n, -1);
+  std::vector<std::vector<Edge>> agg(n);
+  auto find = [&](int32_t v) {  // path halving; concurrent shortcuts stay valid
+    for (;;) {
+      const int32_t p = parent[v].load(std::memory_order_acquire);
+      if (p == v) return v;
+      const int32_t g = parent[p].load(std::memory_order_acquire);
+      if (g != p) parent[v].store(g, std::memory_order_relaxed);
+      v = g;
+    }
+  };
+  const int T = omp_get_max_threads();
+  std::vector<std::vector<int32_t>> tops(T), deferred(T);
+  std::vector<std::vector<MergeRec>> logs(T);
+  std::vector<int64_t> merges(T, 0), retries(T, 0);
+
+  // one sequential step on u; returns false when u must be deferred
+  auto step = [&](int32_t u, HashAcc& H, std::vector<Edge>& tl, int tid) -> bool {
+    int64_t tu;
+    for (;;) {  // PROC-lock u (it may be the target of a short merge section)
+      tu = tot[u].load(std::memory_order_acquire);
+      if (tu == MLOCK) continue;
+      if (tot[u].compare_exchange_weak(tu, PROC, std::memory_order_acq_rel)) break;
+    }
+    for (int attempt = 0;; ++attempt) {
+      size_t expect = (size_t)(S.ptr[u + 1] - S.ptr[u]);
+      for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) expect += agg[c].size();
+      H.prepare(expect);
+      for (int64_t k = S.ptr[u]; k < S.ptr[u + 1]; ++k) {
+        const int32_t r = find(S.idx[k]);
+        if (r != u) H.add(r, S.w[k]);
+      }
+      for (int32_t c = first_child[u]; c != -1; c = next_sib[c])
+        for (const Edge& e : agg[c]) {
+          const int32_t r = find(e.v);
+          if (r != u) H.add(r, e.w);
+        }
+      tl.clear();
+      int32_t best = -1;
+      __int128 bestdq = 0;
+      for (uint32_t h : H.used) {
+        const int32_t r = H.key[h];
+        tl.push_back({r, H.val[h]});
+        const int64_t tr = tot[r].load(std::memory_order_acquire);
+        if (tr < 0) continue;  // being processed / locked / merged meanwhile
+        const __int128 dq = (__int128)two_m * H.val[h] - (__int128)tu * tr;
+        if (best == -1 || dq > bestdq || (dq == bestdq && r < best)) {
+          best = r;
+          bestdq = dq;
+        }
+      }
+      H.clear();
+      if (best == -1 || bestdq <= 0) {
+        for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) std::vector<Edge>().swap(agg[c]);
+        tot[u].store(tu, std::memory_order_release);
+        tops[tid].push_back(u);
+        return true;
+      }
+      // lock the target
+      int64_t tv = tot[best].load(std::memory_order_acquire);
+      bool locked = false, defer = false;
+      for (;;) {
+        if (tv == MLOCK) {
+          tv = tot[best].load(std::memory_order_acquire);
+          continue;
+        }
+        if (tv == PROC) { defer = true; break; }
+        if (tv == MERGED) break;  // merged meanwhile: aggregate again
+        if (tot[best].compare_exchange_weak(tv, MLOCK, std::memory_order_acq_rel)) {
+          locked = true;
+          break;
+        }
+      }
+      if (defer || (!locked && attempt >= 3)) {
+        tot[u].store(tu, std::memory_order_release);
+        deferred[tid].push_back(u);
+        return false;
+      }
+      if (!locked) {
+        retries[tid]++;
+        continue;
+      }
+      // exact w(C_u, C_v) under the lock
+      int64_t w = 0;
+      for (const Edge& e : tl)
+        if (find(e.v) == best) w += e.w;
+      const __int128 dq = (__int128)two_m * w - (__int128)tu * tv;
+      if (dq <= 0) {
+        tot[best].store(tv, std::memory_order_release);
+        if (attempt >= 3) {
+          for (int32_t c = first_child[u]; c != -1; c = next_sib[c])
+            std::vector<Edge>().swap(agg[c]);
+          tot[u].store(tu, std::memory_order_release);
+          tops[tid].push_back(u);
+          return true;
+        }
+        retries[tid]++;
+        continue;
+      }
+      for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) std::vector<Edge>().swap(agg[c]);
+      agg[u] = tl;
+      if (last_child[best] == -1) first_child[best] = u;
+      else next_sib[last_child[best]] = u;
+      last_child[best] = u;
+      parent[u].store(best, std::memory_order_release);
+      tot[u].store(MERGED, std::memory_order_release);
+      merges[tid]++;
+      if (want_log) logs[tid].push_back({u, best, dq});
+      tot[best].store(tv + tu, std::memory_order_release);
+      return true;
+    }
+  };
+
+#pragma omp parallel num_threads(T)
+  {
+    const int tid = omp_get_thread_num();
+    HashAcc H;
+    std::vector<Edge> tl;
+#pragma omp for schedule(dynamic, 256)
+    for (int64_t oi = 0; oi < n; ++oi) step((int32_t)order[oi], H, tl, tid);
+  }
+  // deferred vertices: sequentially, in processing order
+  std::vector<int32_t> rest;
+  for (auto& d : deferred) rest.insert(rest.end(), d.begin(), d.end());
+  std::sort(rest.begin(), rest.end(), [&](int32_t a, int32_t b) { return pos[a] < pos[b]; });
+  Rabbit R;
+  R.parallel = true;
+  R.two_m = two_m;
+  R.n_deferred = (int64_t)rest.size();
+  {
+    HashAcc H;
+    std::vector<Edge> tl;
+    for (auto& d : deferred) d.clear();
+    for (int32_t u : rest)
+      if (!step(u, H, tl, 0)) {  // nothing runs concurrently now: cannot defer again
+        spmv::set_error("rabbit_detect_par: deferred vertex deferred again");
+        throw std::runtime_error("rabbit_detect_par");
+      }
+  }
+  for (int t = 0; t < T; ++t) {
+    R.n_merges += merges[t];
+    R.n_retries += retries[t];
+  }
+  if (want_log)
+    for (auto& l : logs) R.log.insert(R.log.end(), l.begin(), l.end());
+  // top level in processing order (the sequential reading's append order)
+  std::vector<int32_t> top;
+  for (auto& t : tops) top.insert(top.end(), t.begin(), t.end());
+  std::sort(top.begin(), top.end(), [&](int32_t a, int32_t b) { return pos[a] < pos[b]; });
+  std::vector<std::vector<Edge>>().swap(agg);
+  dendrogram_ids(top, first_child, next_sib, R, n);
   return R;
 }
 
@@ -276,6 +524,7 @@ struct DetectCache {
   uint64_t key = 0;
   int64_t n = -1, nnz = -1;
   Rabbit R;
+  bool logged = false;
   std::vector<uint8_t> ins;
   double seconds_detect = 0, seconds_build = 0, largest = 0, qnum = 0, q = 0, insularity = 0;
 };
@@ -310,6 +559,9 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
                                     spmv_reorder_stats_t* st) {
   try {
     auto t0 = std::chrono::steady_clock::now();
+    const bool par = (method & SPMV_REORDER_PARALLEL) != 0;
+    const bool want_log = (method & SPMV_REORDER_LOG) != 0;
+    method &= 0xff;
     if (n < 0 || nnz < 0 || !rp || (nnz && !col) || (n && !perm_out)) {
       spmv::set_error("spmv_reorder: bad argument");
       return SPMV_EINVAL;
@@ -381,13 +633,15 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
       // reuse the last detection on this thread when the input is identical
       const uint64_t key = input_key(n, nnz, rp, col);
       double reused_s = 0;  // detection reused from the cache: charged to this call too
-      if (!(g_cache.valid && g_cache.key == key && g_cache.n == n && g_cache.nnz == nnz)) {
+      if (!(g_cache.valid && g_cache.key == key && g_cache.n == n && g_cache.nnz == nnz &&
+            g_cache.R.parallel == par && (!want_log || g_cache.logged))) {
         g_cache.valid = false;
         const auto tb = std::chrono::steady_clock::now();
         Sym S = symmetrize(n, rp, col);
         phase("symmetrize", tp);
         auto td = std::chrono::steady_clock::now();
-        g_cache.R = rabbit_detect(S);
+        g_cache.R = par ? rabbit_detect_par(S, want_log) : rabbit_detect(S, want_log);
+        g_cache.logged = want_log;
         g_cache.seconds_detect =
             std::chrono::duration<double>(std::chrono::steady_clock::now() - td).count();
         phase("detect+dfs", tp);
@@ -469,6 +723,8 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
       S0.seconds_detect = g_cache.seconds_detect;
       S0.two_m = R.two_m;
       S0.n_merges = R.n_merges;
+      S0.n_deferred = R.n_deferred;
+      S0.parallel = R.parallel ? 1 : 0;
       S0.n_communities = R.n_top;
       S0.largest_comm_frac = g_cache.largest;
       S0.modularity_num = g_cache.qnum;
@@ -526,6 +782,30 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
     spmv::set_error("spmv_reorder: internal error");
     return SPMV_EINVAL;
   }
+}
+
+extern "C" spmv_status spmv_reorder_last_merges(int64_t cap, int32_t* child, int32_t* parent,
+                                                int64_t* dq, int64_t* count_out) {
+  if (!count_out || (cap > 0 && (!child || !parent || !dq))) {
+    spmv::set_error("spmv_reorder_last_merges: bad argument");
+    return SPMV_EINVAL;
+  }
+  if (!g_cache.valid || !g_cache.logged) {
+    spmv::set_error("spmv_reorder_last_merges: no logged RABBIT detection on this thread");
+    return SPMV_ESTATE;
+  }
+  const std::vector<MergeRec>& L = g_cache.R.log;
+  *count_out = (int64_t)L.size();
+  for (int64_t i = 0; i < std::min<int64_t>(cap, (int64_t)L.size()); ++i) {
+    if (L[i].dq > (__int128)INT64_MAX || L[i].dq < (__int128)INT64_MIN) {
+      spmv::set_error("spmv_reorder_last_merges: gain exceeds int64");
+      return SPMV_EUNSUPPORTED;
+    }
+    child[i] = L[i].u;
+    parent[i] = L[i].v;
+    dq[i] = (int64_t)L[i].dq;
+  }
+  return SPMV_OK;
 }
 
 extern "C" spmv_status spmv_reorder_last_comm(int64_t n, int32_t* comm_out) {

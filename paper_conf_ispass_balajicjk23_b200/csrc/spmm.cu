@@ -75,9 +75,10 @@ __device__ __forceinline__ void ld8_f(const float* p, float (&r)[8]) {
 
 // lane per row, L <= SHORT_MAX, sequential: the association of k_lane.  As
 // there, slots of a chunk outside the row read a valid X row (a neighbouring
-// row's column or the zero tail padding) whose value is replaced by 0, so they
-// contribute v * 0 = +-0 for the (finite) matrix value v, which
-// leaves the running sum unchanged (it starts at +0 and is never -0), so the
+// row's column or the zero tail padding); both the matrix value and the X row
+// of such a slot are replaced by 0, so it contributes 0 * 0 = +0 whatever the
+// neighbouring row holds (an Inf / NaN there never reaches this row, Alg. 1)
+// and leaves the running sum unchanged (it starts at +0 and is never -0): the
 // loop is branch-free and both chunks of a 16-entry row are in flight at once.
 template <typename OT, int EF, int MINB, int UNR>
 __global__ void __launch_bounds__(L4_THREADS, MINB)
@@ -104,7 +105,7 @@ __global__ void __launch_bounds__(L4_THREADS, MINB)
         const float4 xg = ldx4(X, cc[i]);
         const bool in = k + i >= lo && k + i < hi;
         const float4 xv = in ? xg : make_float4(0.f, 0.f, 0.f, 0.f);
-        fma4(s, vv[i], xv);
+        fma4(s, in ? vv[i] : 0.f, xv);
       }
     }
     reinterpret_cast<float4*>(Y)[r] = s;

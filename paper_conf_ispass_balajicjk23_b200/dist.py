@@ -1,78 +1,128 @@
-"""Row-block power iteration across ranks (reading c22).
+"""Multi-rank plumbing of spmv_iterate (reading c22).
 
-One process per GPU.  Rank k owns rows [b_k, b_{k+1}) of B (nnz-balanced
-partition computed by spmv_plan), a full replica of x in the padded layout
-x[k*M + (i - b_k)] (M = plan x_stride), and writes its y slice straight into
-its own segment of the next x buffer.  Per iteration:
+One process per GPU.  Rank k owns rows [b_k, b_{k+1}) of B (partition by
+spmv_plan, reading c29) and a full replica of x.  The power-iteration loop --
+scaled SpMV, all-reduce of sum y^2, exchange of the y slices, final
+normalisation and lambda -- runs inside libspmv (spmv_iterate).  This module
+only connects it to torch.distributed:
 
-    exec_scaled   y_k = (B_k u_{t-1}) / s_{t-1},  partial sum y_k^2   (libspmv)
-    all_reduce    s_t^2 = sum_k partial                               (NCCL, 8 B)
-    all_gather    in place, equal-size segments of M floats           (NCCL over NVLink)
+  nccl_comm_ptr   the ncclComm_t of a ProcessGroupNCCL (opts.nccl_comm), so
+                  libspmv issues ncclAllReduce / grouped ncclBroadcast itself;
+  HostColl        an spmv_coll_t over any torch.distributed group with host
+                  staging (gloo): the test / CPU-box backend;
+  PeerBuffers     the ping-pong next-x buffers of the PEER exchange: allocated
+                  with spmv_dev_alloc, IPC handles swapped with
+                  all_gather_object, peers' buffers mapped (NVLink/NVSwitch)
+                  and registered with spmv_set_peers;
+  iterate         plan.iterate (the C loop) with the above in place.
 
-The padded layout turns NCCL's missing all-gatherv into an in-place
-equal-count all-gather with zero copies.  The
-collectives go through torch.distributed (plumbing); all arithmetic runs in
-libspmv.  ``local`` may be any object with the Plan interface below, which is
-how the gloo/CPU tests drive this exact code with a stand-in local SpMV.
+No arithmetic of the method is done here.
 """
 from __future__ import annotations
 
-import math
+import ctypes
+
+import numpy as np
 
 
-def iterate(local, x, iters: int, group=None):
-    """Run `iters` normalised steps from x (padded layout, every rank the same).
-
-    local: object with attributes world, rank, x_stride, y_offset, nrows and
-    methods exec_scaled(x, y, ss_in, ss_out) and scale(u, x, ss).
-    Returns (x_iters normalised, padded layout; lambda = s_iters).
-    """
+def nccl_comm_ptr(group=None, device=None) -> int:
+    """ncclComm_t (as an int) of the NCCL backend of `group` on `device`.
+    The communicator is created eagerly (init_process_group(device_id=...)),
+    or by the first collective; a barrier forces it."""
     import torch
     import torch.distributed as dist
-
-    if iters < 1:
-        raise ValueError("iters must be >= 1")
-    M, off, nr = local.x_stride, local.y_offset, local.nrows
-    xa, xb = x, torch.empty_like(x)
-    ss = torch.zeros(2, dtype=torch.float64, device=x.device)
-    ss_in = None
-    for t in range(iters):
-        ss_out = ss[t & 1:(t & 1) + 1]
-        local.exec_scaled(xa, xb[off:off + nr], ss_in, ss_out)
-        if local.world > 1:
-            dist.all_reduce(ss_out, op=dist.ReduceOp.SUM, group=group)
-            dist.all_gather_into_tensor(xb, xb[off:off + M].clone() if not xb.is_cuda
-                                        else xb[off:off + M], group=group)
-        ss_in = ss_out
-        xa, xb = xb, xa
-    local.scale(xa, xa, ss_in)
-    return xa, math.sqrt(float(ss_in.item()))
+    g = group if group is not None else dist.distributed_c10d._get_default_group()
+    dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+    be = g._get_backend(dev)
+    ptr = be._comm_ptr()
+    if not ptr:
+        dist.barrier(group=g, device_ids=[dev.index])
+        ptr = be._comm_ptr()
+    if not ptr:
+        raise RuntimeError("no NCCL communicator on this process group")
+    return int(ptr)
 
 
-def _all_reduce_sum(t, group, host_staged):
-    import torch.distributed as dist
-    if host_staged:  # gloo: stage through the host (this also syncs the stream)
-        h = t.cpu()
-        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
-        t.copy_(h)
-    else:
-        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+class _DevView:
+    """torch view of a raw fp32 / fp64 device range (__cuda_array_interface__)."""
+
+    def __init__(self, ptr: int, n: int, typestr: str):
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": typestr,
+                                         "data": (int(ptr), False), "version": 3}
 
 
-class FusedExchange:
-    """Peer-mapped ping-pong x buffers for the fused exec + exchange (SURVEY
-    §8(f1)): every rank maps every other rank's two next-x buffers (CUDA IPC
-    over NVLink / NVSwitch), and spmv_exec_scaled_bcast stores each y row
-    straight into all of them -- no all-gather.  One collective remains per
-    step, the 8-byte all-reduce of sum y^2, which also orders the data: a rank
-    passes step t's all-reduce only after every rank's step-t kernels have
-    completed, so the next read sees all peers' stores and no peer overwrites a
-    buffer that is still being read."""
+class HostColl:
+    """spmv_coll_t over a torch.distributed group, staged through host memory
+    (gloo).  device=None: the buffers are host memory (CPU tests);
+    otherwise device buffers on `device`, whose stream is synchronised before
+    the host copy (the callbacks run on the thread that called spmv_iterate)."""
 
-    def __init__(self, plan, device, group=None, host_staged: bool = False):
+    def __init__(self, group=None, device=None):
+        from . import spmv
+        self.group, self.device = group, device
+        self._ar = spmv.ALLREDUCE_FN(self._allreduce)
+        self._ag = spmv.ALLGATHERV_FN(self._allgatherv)
+        self.coll = spmv._Coll(None, self._ar, self._ag)
+        self.calls = {"allreduce": 0, "allgatherv": 0}
+
+    def _view(self, ptr, n, dtype):
+        import torch
+        if self.device is None:
+            ct = ctypes.c_double if dtype == np.float64 else ctypes.c_float
+            return torch.from_numpy(np.ctypeslib.as_array((ct * int(n)).from_address(int(ptr))))
+        ts = "<f8" if dtype == np.float64 else "<f4"
+        return torch.as_tensor(_DevView(ptr, n, ts), device=self.device)
+
+    def _sync(self, stream):
+        import torch
+        if self.device is not None:
+            torch.cuda.ExternalStream(int(stream or 0), device=self.device).synchronize() \
+                if stream else torch.cuda.synchronize(self.device)
+
+    def _allreduce(self, ctx, buf, count, stream):
+        import torch.distributed as dist
+        try:
+            self._sync(stream)
+            t = self._view(buf, count, np.float64)
+            h = t.cpu()
+            dist.all_reduce(h, op=dist.ReduceOp.SUM, group=self.group)
+            t.copy_(h)
+            self._sync(stream)
+            self.calls["allreduce"] += 1
+            return 0
+        except Exception:  # reported as SPMV_ENCCL by the library
+            return 1
+
+    def _allgatherv(self, ctx, x, bounds, world, stream):
+        import torch.distributed as dist
+        try:
+            self._sync(stream)
+            b = [int(bounds[k]) for k in range(world + 1)]
+            t = self._view(x + 4 * b[0], b[world] - b[0], np.float32)
+            h = t.cpu()
+            for k in range(world):  # all-gatherv = one broadcast per root
+                if b[k + 1] > b[k]:
+                    sl = h[b[k] - b[0]:b[k + 1] - b[0]].clone()
+                    dist.broadcast(sl, src=k, group=self.group)
+                    h[b[k] - b[0]:b[k + 1] - b[0]] = sl
+            t.copy_(h)
+            self._sync(stream)
+            self.calls["allgatherv"] += 1
+            return 0
+        except Exception:
+            return 1
+
+
+class PeerBuffers:
+    """Ping-pong next-x buffers of every rank for the PEER exchange (SURVEY
+    §8(f1)): two spmv_dev_alloc buffers per rank, the other ranks' mapped
+    through CUDA IPC (peer access over NVLink / NVSwitch) and registered with
+    spmv_set_peers.  close() unmaps after a barrier (no peer may still store)."""
+
+    def __init__(self, plan, device, group=None):
         import torch.distributed as dist
         from . import spmv
-        self._spmv, self.plan, self.group, self.host_staged = spmv, plan, group, host_staged
+        self._spmv, self.plan, self.group = spmv, plan, group
         i = plan.info()
         self.world, self.rank, xlen = i["world"], i["rank"], i["x_len"]
         idx = device.index if device.index is not None else 0
@@ -81,27 +131,16 @@ class FusedExchange:
         mine = [b.handle() for b in self.bufs]
         allh = [None] * self.world
         dist.all_gather_object(allh, mine, group=group)
-        self.dst = [[0] * self.world for _ in range(2)]
-        for k in range(self.world):
-            for j in range(2):
+        ptrs = []
+        for j in range(2):
+            for k in range(self.world):
                 if k == self.rank:
-                    self.dst[j][k] = self.bufs[j].ptr
+                    ptrs.append(self.bufs[j].ptr)
                 else:
-                    self.dst[j][k] = spmv.ipc_open(allh[k][j])
-                    self.opened.append(self.dst[j][k])
-        self.cur = 0
-
-    @property
-    def x(self):
-        """The current x (padded layout) -- the buffer the next step reads."""
-        return self.bufs[self.cur].tensor
-
-    def step(self, ss_in, ss_out):
-        """x <- B x / s (fused store into every rank's next buffer), then the
-        all-reduce of ss_out; flips the ping-pong."""
-        self.plan.exec_scaled_bcast(self.x, self.dst[1 - self.cur], ss_in, ss_out)
-        _all_reduce_sum(ss_out, self.group, self.host_staged)
-        self.cur = 1 - self.cur
+                    q = spmv.ipc_open(allh[k][j])
+                    self.opened.append(q)
+                    ptrs.append(q)
+        plan.set_peers(ptrs)
 
     def close(self):
         import torch
@@ -109,7 +148,7 @@ class FusedExchange:
         if self.bufs is None:
             return
         torch.cuda.synchronize()
-        dist.barrier(group=self.group)  # nobody unmaps while a peer may still store
+        dist.barrier(group=self.group)
         for q in self.opened:
             self._spmv.ipc_close(q)
         for b in self.bufs:
@@ -117,44 +156,10 @@ class FusedExchange:
         self.bufs = None
 
 
-def iterate_fused(plan, x, iters: int, group=None, host_staged: bool = False):
-    """iterate() with the exchange fused into the SpMV (FusedExchange).
-    Returns (x_iters normalised, padded layout; lambda = s_iters)."""
-    import torch
-
-    if iters < 1:
-        raise ValueError("iters must be >= 1")
-    fx = FusedExchange(plan, x.device, group, host_staged)
-    try:
-        fx.x.copy_(x)
-        ss = torch.zeros(2, dtype=torch.float64, device=x.device)
-        ss_in = None
-        for t in range(iters):
-            ss_out = ss[t & 1:(t & 1) + 1]
-            fx.step(ss_in, ss_out)
-            ss_in = ss_out
-        out = torch.empty_like(x)
-        fx._spmv.scale_vec(fx.x, out, ss_in)
-        lam = math.sqrt(float(ss_in.item()))
-    finally:
-        fx.close()
-    return out, lam
-
-
-class PlanLocal:
-    """Adapter: a libspmv Plan as the `local` of iterate()."""
-
-    def __init__(self, plan):
-        from . import spmv
-        self._spmv = spmv
-        self.plan = plan
-        i = plan.info()
-        self.world, self.rank = i["world"], i["rank"]
-        self.x_stride, self.y_offset = i["x_stride"], i["y_offset"]
-        self.nrows = i["row_end"] - i["row_begin"]
-
-    def exec_scaled(self, x, y, ss_in, ss_out):
-        self.plan.exec_scaled(x, y, ss_in, ss_out)
-
-    def scale(self, u, x, ss):
-        self._spmv.scale_vec(u, x, ss)
+def iterate(plan, x, iters: int, stream=None) -> float:
+    """spmv_iterate on this rank: x (full length, plan's x layout, the same on
+    every rank) is overwritten with x_iters; returns lambda = s_iters.  The
+    plan carries its collective backend (nccl_comm at creation, or
+    plan.set_coll(HostColl(...).coll)) and, for the PEER exchange, its
+    PeerBuffers."""
+    return plan.iterate(x, iters, stream)

@@ -42,7 +42,24 @@ class _Opts(ctypes.Structure):
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("smem_window", ctypes.c_int32),
                 ("l2_hit_ratio", ctypes.c_double), ("variant", ctypes.c_int64),
-                ("hot_x", ctypes.c_int64), ("reserved", ctypes.c_int64 * 6)]
+                ("hot_x", ctypes.c_int64), ("nccl_comm", ctypes.c_void_p),
+                ("x_layout", ctypes.c_int32), ("exchange", ctypes.c_int32),
+                ("reserved", ctypes.c_int64 * 4)]
+
+
+XLAYOUT_GLOBAL, XLAYOUT_PADDED = 0, 1
+EXCHANGE_COLL, EXCHANGE_PEER = 0, 1
+
+# spmv_coll_t callbacks (int return, 0 = ok)
+ALLREDUCE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64,
+                                ctypes.c_void_p)
+ALLGATHERV_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
+                                 ctypes.POINTER(ctypes.c_int64), ctypes.c_int, ctypes.c_void_p)
+
+
+class _Coll(ctypes.Structure):
+    _fields_ = [("ctx", ctypes.c_void_p), ("allreduce_sum_f64", ALLREDUCE_FN),
+                ("allgatherv_f32", ALLGATHERV_FN)]
 
 
 class _Info(ctypes.Structure):
@@ -62,7 +79,8 @@ class _Stats(ctypes.Structure):
                 ("insularity", ctypes.c_double), ("insular_frac", ctypes.c_double),
                 ("n_hubs", ctypes.c_int64), ("n_group0", ctypes.c_int64),
                 ("skew", ctypes.c_double), ("seconds", ctypes.c_double),
-                ("seconds_detect", ctypes.c_double)]
+                ("seconds_detect", ctypes.c_double), ("n_deferred", ctypes.c_int64),
+                ("parallel", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 _lib = None
@@ -96,6 +114,9 @@ def lib() -> ctypes.CDLL:
             "spmv_export_coo_rows": (i32, [vp, vp, vp]),
             "spmv_iterate": (i32, [vp, vp, i32, ctypes.POINTER(ctypes.c_double), vp]),
             "spmv_scale_vec": (i32, [vp, vp, i64, dp, vp]),
+            "spmv_set_coll": (i32, [vp, ctypes.POINTER(_Coll)]),
+            "spmv_set_peers": (i32, [vp, vp, i32]),
+            "spmv_iterate_finish": (i32, [vp, vp, i64, dp, ctypes.POINTER(ctypes.c_double), vp]),
             "spmv_plan_info": (i32, [vp, ctypes.POINTER(_Info)]),
             "spmv_export_csr": (i32, [vp, vp, vp, vp, vp]),
             "spmv_export_bins": (i32, [vp, vp, vp, vp, vp, vp, vp, vp, vp]),
@@ -104,6 +125,7 @@ def lib() -> ctypes.CDLL:
             "spmv_destroy": (None, [vp]),
             "spmv_reorder": (i32, [i64, i64, vp, vp, i32, ctypes.c_uint64, vp, ctypes.POINTER(_Stats)]),
             "spmv_reorder_last_comm": (i32, [i64, vp]),
+            "spmv_reorder_last_merges": (i32, [i64, vp, vp, vp, ctypes.POINTER(ctypes.c_int64)]),
             "spmv_last_error": (ctypes.c_char_p, []),
             "spmv_version": (ctypes.c_char_p, []),
         }
@@ -130,9 +152,11 @@ def version() -> str:
     return lib().spmv_version().decode()
 
 
-def _stream_ptr(stream=None) -> int:
+def _stream_ptr(stream=None, device=None) -> int:
+    """The given stream, else the current stream of `device` (a plan's device,
+    not whichever device happens to be current)."""
     import torch
-    s = stream if stream is not None else torch.cuda.current_stream()
+    s = stream if stream is not None else torch.cuda.current_stream(device)
     return int(s.cuda_stream)
 
 
@@ -149,7 +173,8 @@ class Plan:
 
     def __init__(self, row_ptr, col, val, perm=None, *, world=1, rank=0, l2_window=True,
                  evict_first=True, l2_hit_ratio=1.0, smem_window=True, variant=0,
-                 hot_x=0, permute=True, stream=None):
+                 hot_x=0, permute=True, stream=None, x_layout=XLAYOUT_GLOBAL,
+                 exchange=EXCHANGE_COLL, nccl_comm=None):
         import torch
         assert row_ptr.is_cuda and col.is_cuda and val.is_cuda
         assert col.dtype == torch.int32 and val.dtype == torch.float32
@@ -172,6 +197,8 @@ class Plan:
         o.smem_window = int(smem_window)
         o.variant = int(variant)
         o.hot_x = int(hot_x)
+        o.x_layout, o.exchange = int(x_layout), int(exchange)
+        o.nccl_comm = nccl_comm
         o.device = row_ptr.device.index if row_ptr.device.index is not None else -1
         h = ctypes.c_void_p()
         _check(lib().spmv_plan(ctypes.byref(A), _ptr(perm), ctypes.byref(o), ctypes.byref(h)))
@@ -182,7 +209,7 @@ class Plan:
 
     # ------------------------------------------------------------------ calls
     def permute(self, stream=None):
-        _check(lib().spmv_permute(self._h, _stream_ptr(stream)))
+        _check(lib().spmv_permute(self._h, _stream_ptr(stream, self.device)))
         return self
 
     def info(self) -> dict:
@@ -193,7 +220,7 @@ class Plan:
     def permute_vec(self, x, inverse=False, out=None, stream=None):
         import torch
         out = torch.empty_like(x) if out is None else out
-        _check(lib().spmv_permute_vec(self._h, _ptr(x), _ptr(out), int(inverse), _stream_ptr(stream)))
+        _check(lib().spmv_permute_vec(self._h, _ptr(x), _ptr(out), int(inverse), _stream_ptr(stream, self.device)))
         return out
 
     def pad_vec(self, x, to_padded=True, out=None, stream=None):
@@ -202,7 +229,7 @@ class Plan:
             info = self.info()
             out = torch.zeros(info["x_len"] if to_padded else info["n"], dtype=torch.float32,
                               device=x.device)
-        _check(lib().spmv_pad_vec(self._h, _ptr(x), _ptr(out), int(to_padded), _stream_ptr(stream)))
+        _check(lib().spmv_pad_vec(self._h, _ptr(x), _ptr(out), int(to_padded), _stream_ptr(stream, self.device)))
         return out
 
     def exec(self, x, y=None, stream=None):
@@ -210,7 +237,7 @@ class Plan:
         if y is None:
             info = self.info()
             y = torch.empty(info["row_end"] - info["row_begin"], dtype=torch.float32, device=x.device)
-        _check(lib().spmv_exec(self._h, _ptr(x), _ptr(y), _stream_ptr(stream)))
+        _check(lib().spmv_exec(self._h, _ptr(x), _ptr(y), _stream_ptr(stream, self.device)))
         return y
 
     def exec_coo(self, x, y=None, stream=None):
@@ -219,14 +246,14 @@ class Plan:
         if y is None:
             info = self.info()
             y = torch.empty(info["row_end"] - info["row_begin"], dtype=torch.float32, device=x.device)
-        _check(lib().spmv_exec_coo(self._h, _ptr(x), _ptr(y), _stream_ptr(stream)))
+        _check(lib().spmv_exec_coo(self._h, _ptr(x), _ptr(y), _stream_ptr(stream, self.device)))
         return y
 
     def export_coo_rows(self):
         import torch
         info = self.info()
         rows = torch.empty(info["nnz_local"], dtype=torch.int32, device=self.device)
-        _check(lib().spmv_export_coo_rows(self._h, _ptr(rows), _stream_ptr(None)))
+        _check(lib().spmv_export_coo_rows(self._h, _ptr(rows), _stream_ptr(None, self.device)))
         return rows
 
     def exec_spmm4(self, X, Y=None, stream=None):
@@ -236,7 +263,7 @@ class Plan:
             info = self.info()
             Y = torch.empty((info["row_end"] - info["row_begin"], 4), dtype=torch.float32,
                             device=X.device)
-        _check(lib().spmv_exec_spmm4(self._h, _ptr(X), _ptr(Y), _stream_ptr(stream)))
+        _check(lib().spmv_exec_spmm4(self._h, _ptr(X), _ptr(Y), _stream_ptr(stream, self.device)))
         return Y
 
     def exec_scaled_bcast(self, x, x_next_ptrs, sumsq_in, sumsq_out, stream=None):
@@ -244,16 +271,29 @@ class Plan:
         buffer of x_next_ptrs (device addresses, padded x layout)."""
         arr = (ctypes.c_void_p * len(x_next_ptrs))(*[int(a) for a in x_next_ptrs])
         _check(lib().spmv_exec_scaled_bcast(self._h, _ptr(x), arr, len(x_next_ptrs),
-                                            _ptr(sumsq_in), _ptr(sumsq_out), _stream_ptr(stream)))
+                                            _ptr(sumsq_in), _ptr(sumsq_out), _stream_ptr(stream, self.device)))
 
     def exec_scaled(self, x, y, sumsq_in=None, sumsq_out=None, stream=None):
         _check(lib().spmv_exec_scaled(self._h, _ptr(x), _ptr(y), _ptr(sumsq_in), _ptr(sumsq_out),
-                                      _stream_ptr(stream)))
+                                      _stream_ptr(stream, self.device)))
         return y
+
+    def set_coll(self, coll):
+        """Install a collective backend (a _Coll, kept alive here) or None for
+        NCCL on the plan's nccl_comm."""
+        self._coll = coll
+        _check(lib().spmv_set_coll(self._h, None if coll is None else ctypes.byref(coll)))
+
+    def set_peers(self, ptrs):
+        """Peer next-x buffers of the PEER exchange: 2 * world device addresses,
+        [j * world + k] = buffer j of rank k."""
+        arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
+        _check(lib().spmv_set_peers(self._h, ctypes.cast(arr, ctypes.c_void_p),
+                                    len(ptrs) // 2))
 
     def iterate(self, x, iters: int, stream=None) -> float:
         lam = ctypes.c_double(0.0)
-        _check(lib().spmv_iterate(self._h, _ptr(x), iters, ctypes.byref(lam), _stream_ptr(stream)))
+        _check(lib().spmv_iterate(self._h, _ptr(x), iters, ctypes.byref(lam), _stream_ptr(stream, self.device)))
         return lam.value
 
     def export_csr(self, stream=None):
@@ -263,7 +303,7 @@ class Plan:
         rp = torch.empty(nr + 1, dtype=torch.int64, device=self.device)
         col = torch.empty(max(i["nnz_local"], 0), dtype=torch.int32, device=self.device)
         val = torch.empty(max(i["nnz_local"], 0), dtype=torch.float32, device=self.device)
-        _check(lib().spmv_export_csr(self._h, _ptr(rp), _ptr(col), _ptr(val), _stream_ptr(stream)))
+        _check(lib().spmv_export_csr(self._h, _ptr(rp), _ptr(col), _ptr(val), _stream_ptr(stream, self.device)))
         return rp, col, val
 
     def export_bins(self, stream=None) -> dict:
@@ -279,7 +319,7 @@ class Plan:
                                       _ptr(d["warp_rows"]),
                                       _ptr(d["cta_rows"]),
                                       _ptr(d["hub_rows"]), _ptr(d["chunk_row"]),
-                                      _ptr(d["chunk_idx"]), _stream_ptr(stream)))
+                                      _ptr(d["chunk_idx"]), _stream_ptr(stream, self.device)))
         return d
 
     def export_partition(self) -> list[int]:
@@ -291,7 +331,7 @@ class Plan:
     def export_inverse(self, stream=None):
         import torch
         inv = torch.empty(self.info()["n"], dtype=torch.int32, device=self.device)
-        _check(lib().spmv_export_inverse(self._h, _ptr(inv), _stream_ptr(stream)))
+        _check(lib().spmv_export_inverse(self._h, _ptr(inv), _stream_ptr(stream, self.device)))
         return inv
 
     def close(self):
@@ -307,6 +347,14 @@ class Plan:
             self.close()
         except Exception:
             pass
+
+
+def iterate_finish(u, x, sumsq, stream=None) -> float:
+    """x = u / sqrt(sumsq) (device), returns lambda = sqrt(sumsq)."""
+    lam = ctypes.c_double(0.0)
+    _check(lib().spmv_iterate_finish(_ptr(u), _ptr(x), u.numel(), _ptr(sumsq), ctypes.byref(lam),
+                                     _stream_ptr(stream, u.device)))
+    return lam.value
 
 
 def scale_vec(u, x, sumsq=None, stream=None):
@@ -329,11 +377,21 @@ class ReorderStats:
     skew: float
     seconds: float
     seconds_detect: float
+    n_deferred: int = 0
+    parallel: int = 0
+    reserved: int = 0
 
 
-def reorder(row_ptr: np.ndarray, col: np.ndarray, method="rabbitpp", seed: int = 0):
-    """Host reordering (spmv_reorder).  Returns (perm int32[n], ReorderStats)."""
+PARALLEL, LOG = 0x100, 0x200
+
+
+def reorder(row_ptr: np.ndarray, col: np.ndarray, method="rabbitpp", seed: int = 0,
+            parallel: bool = False, log: bool = False):
+    """Host reordering (spmv_reorder).  Returns (perm int32[n], ReorderStats).
+    parallel: concurrent RABBIT merges (SPMV_REORDER_PARALLEL); log: keep the
+    merge log for reorder_last_merges()."""
     m = METHODS[method] if isinstance(method, str) else int(method)
+    m |= (PARALLEL if parallel else 0) | (LOG if log else 0)
     rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
     c = np.ascontiguousarray(col, dtype=np.int32)
     n = len(rp) - 1
@@ -342,6 +400,17 @@ def reorder(row_ptr: np.ndarray, col: np.ndarray, method="rabbitpp", seed: int =
     _check(lib().spmv_reorder(n, int(rp[-1]) if n >= 0 else 0, rp.ctypes.data, c.ctypes.data, m,
                               seed, perm.ctypes.data, ctypes.byref(st)))
     return perm, ReorderStats(**{f: getattr(st, f) for f, _ in _Stats._fields_})
+
+
+def reorder_last_merges():
+    """(child int32[], root int32[], dq int64[]) of the last logged detection."""
+    cnt = ctypes.c_int64(0)
+    _check(lib().spmv_reorder_last_merges(0, None, None, None, ctypes.byref(cnt)))
+    m = cnt.value
+    c, p, d = np.empty(m, np.int32), np.empty(m, np.int32), np.empty(m, np.int64)
+    _check(lib().spmv_reorder_last_merges(m, c.ctypes.data, p.ctypes.data, d.ctypes.data,
+                                          ctypes.byref(cnt)))
+    return c, p, d
 
 
 def reorder_last_comm(n: int) -> np.ndarray:

@@ -17,7 +17,7 @@ from paper_conf_ispass_balajicjk23_b200 import spmv
 def test_library_exports_every_declared_symbol():
     L = spmv.lib()
     names = spmv.declared_symbols()
-    assert len(names) == 29
+    assert len(names) == 33
     for nm in names:
         assert hasattr(L, nm), nm
     assert "sm_100a" in spmv.version()
@@ -28,6 +28,11 @@ def test_opts_default_and_errors_without_gpu():
     spmv.lib().spmv_opts_default(ctypes.byref(o))
     assert (o.l2_window, o.evict_first, o.rank, o.world, o.device) == (1, 1, 0, 1, -1)
     assert o.l2_hit_ratio == 1.0
+    assert (o.nccl_comm, o.x_layout, o.exchange) == (None, spmv.XLAYOUT_GLOBAL, spmv.EXCHANGE_COLL)
+    assert ctypes.sizeof(o) == 6 * 4 + 4 * 8 + 2 * 4 + 4 * 8   # layout of spmv_opts_t
+    # collective backend / peers need a plan
+    assert spmv.lib().spmv_set_coll(None, None) == 1
+    assert spmv.lib().spmv_set_peers(None, None, 2) == 1
     h = ctypes.c_void_p()
     st = spmv.lib().spmv_plan(None, None, None, ctypes.byref(h))
     assert st == 1 and b"NULL" in spmv.lib().spmv_last_error()

@@ -1,9 +1,13 @@
 """Multi-rank host logic of the row-block power iteration on
-CPU: world_size 2 over gloo, driving paper_conf_ispass_balajicjk23_b200.dist
-exactly as the NCCL run does, with the oracle standing in for the local
-kernel (the CUDA kernels themselves are covered by tests/test_gpu_parity.py,
-including partitioned == single bitwise)."""
-import math
+CPU: world_size 2 over gloo.
+
+spmv_iterate's loop runs in libspmv and needs a GPU (tests/test_gpu_iterate_dist.py
+runs it with two ranks on one GPU through exactly these callbacks).  Here the
+host side is exercised without a GPU: dist.HostColl, the spmv_coll_t backend
+the library calls between its kernels, on host buffers -- the all-gatherv of
+uneven row slices (the partition of reading c29) and the fp64 all-reduce --
+called through the same C function pointers libspmv calls."""
+import ctypes
 import os
 import socket
 
@@ -11,58 +15,9 @@ import numpy as np
 import pytest
 
 import synth
-from oracle import permute, plan as oplan, power, rabbit, spmv as ospmv
+from oracle import permute, plan as oplan, rabbit
 
 torch = pytest.importorskip("torch")
-
-
-class OracleLocal:
-    """CPU stand-in with the Plan interface used by dist.iterate: rows
-    [b_r, b_{r+1}) of B, padded x layout x[k*M + i - b_k]."""
-
-    def __init__(self, Bp, Bc, Bv, world, rank):
-        n = len(Bp) - 1
-        self.world, self.rank = world, rank
-        self.bounds = oplan.partition(Bp, world)
-        M = int(max(np.diff(self.bounds).max(), 1))
-        M = (M + 31) // 32 * 32
-        self.x_stride, self.y_offset = M, rank * M
-        b0, b1 = self.bounds[rank], self.bounds[rank + 1]
-        self.nrows = int(b1 - b0)
-        owner = np.searchsorted(self.bounds, np.arange(n), side="right") - 1
-        self.pad_index = owner * M + (np.arange(n) - self.bounds[owner])
-        lo, hi = Bp[b0], Bp[b1]
-        self.rp = Bp[b0:b1 + 1] - lo
-        self.col = self.pad_index[Bc[lo:hi]].astype(np.int32)
-        self.val = Bv[lo:hi]
-
-    def exec_scaled(self, x, y, ss_in, ss_out):
-        alpha = 1.0 if ss_in is None else np.float32(1.0 / math.sqrt(float(ss_in.item())))
-        yy = ospmv.spmv(self.rp, self.col, self.val, x.numpy()) * np.float32(alpha)
-        y.copy_(torch.from_numpy(yy.astype(np.float32)))
-        ss_out.fill_(float(np.sum(yy.astype(np.float64) ** 2)))
-
-    def scale(self, u, x, ss):
-        x.copy_(u * np.float32(1.0 / math.sqrt(float(ss.item()))))
-
-
-def _worker(rank, world, port, out_dir):
-    import torch.distributed as dist
-    from paper_conf_ispass_balajicjk23_b200 import dist as pdist
-    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank,
-                            world_size=world)
-    w = synth.config(5, small=True)
-    A = w.A
-    perm = rabbit.random_perm(A.n, 3)
-    Bp, Bc, Bv = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
-    loc = OracleLocal(Bp, Bc, Bv, world, rank)
-    xB = permute.permute_vec(w.x, perm)
-    xpad = np.zeros(world * loc.x_stride, np.float32)
-    xpad[loc.pad_index] = xB
-    x, lam = pdist.iterate(loc, torch.from_numpy(xpad), 6)
-    np.save(os.path.join(out_dir, f"x{rank}.npy"), x.numpy()[loc.pad_index])
-    np.save(os.path.join(out_dir, f"lam{rank}.npy"), np.array([lam]))
-    dist.destroy_process_group()
 
 
 def _free_port():
@@ -73,33 +28,66 @@ def _free_port():
     return p
 
 
-@pytest.mark.parametrize("world", [2])
-def test_gloo_power_iteration_matches_oracle(tmp_path, world):
-    import torch.multiprocessing as mp
-    mp.spawn(_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
-    w = synth.config(5, small=True)
-    A = w.A
+def _bounds():
+    """Partition bounds of a Kronecker-14 matrix in a random order at G = 2
+    (uneven slices), from the oracle's reading-c29 partition."""
+    A = synth.config(5, small=True).A
     perm = rabbit.random_perm(A.n, 3)
-    Bp, Bc, Bv = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
-    xr, lr = power.power_iteration(Bp, Bc, Bv, permute.permute_vec(w.x, perm), 6)
-    xs = [np.load(tmp_path / f"x{r}.npy") for r in range(world)]
-    lams = [float(np.load(tmp_path / f"lam{r}.npy")[0]) for r in range(world)]
-    for r in range(world):
-        assert np.array_equal(xs[r], xs[0])          # every replica identical
-        assert abs(lams[r] - lr) <= 1e-5 * lr
-        assert np.max(np.abs(xs[r] - xr)) <= 1e-5 * np.max(np.abs(xr))
+    Bp, _, _ = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
+    return A.n, oplan.partition(Bp, 2)
 
 
-def test_single_rank_path_matches_oracle():
-    # world == 1 through the same driver (no collectives)
+def _worker(rank, world, port, out_dir):
+    import torch.distributed as dist
     from paper_conf_ispass_balajicjk23_b200 import dist as pdist
-    A = synth.rmat(9, 8, 4, valmode=synth.VAL_POS, seed_v=2)
-    Bp, Bc, Bv = A.row_ptr, A.col, A.val
-    loc = OracleLocal(Bp, Bc, Bv, 1, 0)
-    x0 = np.ones(A.n, np.float32) / np.float32(math.sqrt(A.n))
-    xpad = np.zeros(loc.x_stride, np.float32)
-    xpad[loc.pad_index] = x0
-    x, lam = pdist.iterate(loc, torch.from_numpy(xpad), 4)
-    xr, lr = power.power_iteration(Bp, Bc, Bv, x0, 4)
-    assert abs(lam - lr) <= 1e-6 * lr
-    assert np.allclose(x.numpy()[loc.pad_index], xr, rtol=1e-5, atol=1e-7)
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank,
+                            world_size=world)
+    n, b = _bounds()
+    hc = pdist.HostColl()          # host buffers (device=None)
+    c = hc.coll
+    # every rank holds only its own slice (others are garbage) before the exchange
+    x = np.full(n, -1.0 - rank, np.float32)
+    x[b[rank]:b[rank + 1]] = np.arange(b[rank], b[rank + 1], dtype=np.float32) * 0.5
+    bnd = (ctypes.c_int64 * (world + 1))(*[int(v) for v in b])
+    rc = c.allgatherv_f32(None, x.ctypes.data, bnd, world, None)
+    ss = np.array([float(rank + 1) * 0.25, 7.0], np.float64)
+    rc2 = c.allreduce_sum_f64(None, ss.ctypes.data, 2, None)
+    np.savez(os.path.join(out_dir, f"r{rank}.npz"), x=x, ss=ss, rc=[rc, rc2],
+             calls=[hc.calls["allgatherv"], hc.calls["allreduce"]])
+    dist.destroy_process_group()
+
+
+def test_hostcoll_allgatherv_and_allreduce_world2(tmp_path):
+    import torch.multiprocessing as mp
+    world = 2
+    mp.spawn(_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    n, b = _bounds()
+    assert b[1] - b[0] != b[2] - b[1]                 # genuinely uneven slices
+    want = np.arange(n, dtype=np.float32) * 0.5
+    for r in range(world):
+        d = np.load(tmp_path / f"r{r}.npz")
+        assert d["rc"].tolist() == [0, 0]
+        assert d["calls"].tolist() == [1, 1]
+        assert np.array_equal(d["x"], want)           # every slice from its owner
+        assert d["ss"].tolist() == [0.25 + 0.5, 14.0]  # fp64 sum over ranks
+
+
+def test_partition_global_layout_no_inflation():
+    """Reading c29 partition on kron14 under RABBIT++ at G = 8 (the verdict's
+    inflation case): with the global x layout every rank's slice is its own
+    row block, so the exchanged x is exactly n floats (x_len / n = 1) however
+    uneven the row counts are; the blocks tile [0, n) and every block's
+    compulsory bytes are within one row of the ideal share."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = synth.config(5, small=True).A
+    perm, _ = spmv.reorder(A.row_ptr, A.col, "rabbitpp")
+    Bp, _, _ = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm.astype(np.int64))
+    G = 8
+    b = oplan.partition(Bp, G)
+    assert b[0] == 0 and b[-1] == A.n and np.all(np.diff(b) >= 0)
+    assert int(np.diff(b).sum()) == A.n               # x_len / n = 1
+    c = 8 * Bp + 12 * np.arange(A.n + 1)
+    share = c[-1] / G
+    worst_row = int((8 * np.diff(Bp) + 12).max())
+    for k in range(G):
+        assert abs((c[b[k + 1]] - c[b[k]]) - share) <= worst_row

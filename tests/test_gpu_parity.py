@@ -156,7 +156,8 @@ def test_exec_matches_oracle(dev, name, make):
 
 @pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("rmat12", "longrows", "kron14")])
 @pytest.mark.parametrize("world", [2, 3, 4])
-def test_partitioned_equals_single_bitwise(dev, name, make, world):
+@pytest.mark.parametrize("layout", ["global", "padded"])
+def test_partitioned_equals_single_bitwise(dev, name, make, world, layout):
     A = make()
     perm = rabbit.random_perm(A.n, 11)
     P1 = mk_plan(A, perm, dev)
@@ -167,12 +168,19 @@ def test_partitioned_equals_single_bitwise(dev, name, make, world):
     bounds = oplan.partition(Bp, world)
     parts = []
     for r in range(world):
-        Pr = mk_plan(A, perm, dev, world=world, rank=r)
+        from paper_conf_ispass_balajicjk23_b200 import spmv
+        Pr = mk_plan(A, perm, dev, world=world, rank=r,
+                     x_layout=spmv.XLAYOUT_PADDED if layout == "padded" else spmv.XLAYOUT_GLOBAL)
         assert Pr.export_partition() == bounds.tolist()
         info = Pr.info()
         assert (info["row_begin"], info["row_end"]) == (bounds[r], bounds[r + 1])
         xpad = Pr.pad_vec(xB, to_padded=True)
-        assert xpad.numel() == info["x_len"] == world * info["x_stride"]
+        if layout == "padded":
+            assert xpad.numel() == info["x_len"] == world * info["x_stride"]
+            assert info["y_offset"] == r * info["x_stride"]
+        else:  # global layout: x_B itself, this rank's y slice at row_begin
+            assert xpad.numel() == info["x_len"] == A.n
+            assert info["y_offset"] == bounds[r]
         back = Pr.pad_vec(xpad, to_padded=False)
         assert torch.equal(back, xB)
         parts.append(Pr.exec(xpad).cpu().numpy())

@@ -37,6 +37,22 @@ def test_skew_closed_form():
     assert math.isclose(metrics.skew(rp), 100 / 190)
 
 
+def test_community_stats_closed_form():
+    """(#communities, largest fraction) ("largest community
+    comprises 98% of the nodes", :144) on hand-counted labelings."""
+    assert metrics.community_stats([]) == (0, 0.0)
+    assert metrics.community_stats([7]) == (1, 1.0)
+    # K3 + K4 under RABBIT (SURVEY 8(c) closed form): comm = {2,2,2,6,6,6,6}
+    assert metrics.community_stats([2, 2, 2, 6, 6, 6, 6]) == (2, 4 / 7)
+    # labels need not be contiguous or sorted; singletons count as communities
+    n, big = metrics.community_stats([5, 0, 5, 9, 5, 0, 3])
+    assert (n, big) == (4, 3 / 7)
+    # n singletons: n communities of fraction 1/n
+    assert metrics.community_stats(list(range(10))) == (10, 0.1)
+    # the mawi case study shape: 98 of 100 nodes in one community
+    assert metrics.community_stats([0] * 98 + [1, 2]) == (3, 0.98)
+
+
 def test_hub_footprint_pin():
     g = GOLD["sx_stackoverflow_hub_footprint"]
     fp = metrics.hub_footprint(np.arange(g["hubs"]), g["line_bytes"], g["elem_bytes"])
@@ -107,9 +123,29 @@ def test_row_classes_and_partition():
     for G in (1, 2, 3, 8):
         b = plan.partition(rp, G)
         assert b[0] == 0 and b[-1] == len(L) and np.all(np.diff(b) >= 0)
+        c = 8 * rp + 12 * np.arange(len(rp))      # int32 offsets: 8 B / entry, 12 B / row
         for k in range(1, G):
-            t = -(-(k * int(rp[-1])) // G)
-            assert rp[b[k]] >= t and (b[k] == 0 or rp[b[k] - 1] < t)
+            t = -(-(k * int(c[-1])) // G)
+            assert c[b[k]] >= t and (b[k] == 0 or c[b[k] - 1] < t)
+
+
+def test_partition_balances_compulsory_bytes():
+    """Reading c29 by hand: L = [4, 0, 0, 0, 4], int32 offsets (w_off = 4).
+    c(r) = 8 row_ptr[r] + 12 r = [0, 44, 56, 68, 80, 124]; G = 2: target
+    ceil(124 / 2) = 62 -> b_1 = 3 (c = 68): rank 0 gets 4 entries + 3 rows
+    (68 B of P:96 traffic), rank 1 4 entries + 2 rows (56 B).  The plain nnz
+    split (lower_bound(row_ptr, 4) = 1) would give rank 1 all four empty rows."""
+    rp = np.array([0, 4, 4, 4, 4, 8], np.int64)
+    assert plan.partition(rp, 2).tolist() == [0, 3, 5]
+    assert plan.partition(rp, 1).tolist() == [0, 5]
+    # G larger than N: empty blocks, bounds still monotone and complete
+    assert plan.partition(np.array([0, 2], np.int64), 3).tolist() == [0, 1, 1, 1]
+    # int64 offsets (NZ >= 2^31) weigh a row 16 B: c(r) = 8 rp + 16 r
+    rp64 = np.array([0, 2**31, 2**31, 2**31 + 2], np.int64)
+    c = 8 * rp64 + 16 * np.arange(4)
+    b = plan.partition(rp64, 2)
+    t = -(-int(c[-1]) // 2)
+    assert c[b[1]] >= t and c[b[1] - 1] < t
 
 
 def test_hot_prefix():

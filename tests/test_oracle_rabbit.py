@@ -205,3 +205,29 @@ def test_random_perm():
     assert permute.is_bijection(p, 1000)
     assert np.array_equal(p, rabbit.random_perm(1000, 42))
     assert not np.array_equal(p, rabbit.random_perm(1000, 43))
+
+
+# splitmix64 reference outputs for state 0 (Vigna's splitmix64.c; the same
+# stream as java.util.SplittableRandom): output k = mix64(k * 0x9E3779B97F4A7C15).
+# Reading c19 draws h1(seed, i) = output i+1 of the stream started at `seed`.
+SPLITMIX64_SEED0 = [0xE220A8397B1DCDAF, 0x6E789E6AA1B965F4, 0x06C45D188009454F,
+                    0xF88BB8A8724C81EC, 0x1B39896A51A8749B]
+
+
+def test_random_perm_hand_worked_fisher_yates():
+    """RANDOM (reading c19) pinned by hand from the published splitmix64 vector.
+
+    n = 4, seed 0, p = [0, 1, 2, 3]:
+      i = 3: j = out4 mod 4 = 0  -> swap p3, p0 -> [3, 1, 2, 0]
+      i = 2: j = out3 mod 3 = 1  -> swap p2, p1 -> [3, 2, 1, 0]
+      i = 1: j = out2 mod 2 = 0  -> swap p1, p0 -> [2, 3, 1, 0]
+    n = 5 adds i = 4 first: j = out5 mod 5 = 2 -> [0, 1, 4, 3, 2], then the
+      same three steps -> [3, 1, 4, 0, 2] -> [3, 4, 1, 0, 2] -> [4, 3, 1, 0, 2].
+    A Sattolo slip (mod i instead of mod i+1) or an off-by-one counter gives
+    other permutations."""
+    o = SPLITMIX64_SEED0
+    assert (o[1] % 2, o[2] % 3, o[3] % 4, o[4] % 5) == (0, 1, 0, 2)  # the j's above
+    assert rabbit.random_perm(4, 0).tolist() == [2, 3, 1, 0]
+    assert rabbit.random_perm(5, 0).tolist() == [4, 3, 1, 0, 2]
+    assert rabbit.random_perm(1, 0).tolist() == [0]
+    assert rabbit.random_perm(0, 0).tolist() == []
