@@ -1,24 +1,40 @@
 """Benchmark of the community-reordered CSR SpMV hot path (BASELINE.json metric).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
-                    [--config 2] [--orderings original,rabbit,rabbitpp]
+                    [--config 5] [--orderings original,rabbit,rabbitpp]
+                    [--exchange coll|peer] [--suite]
 
-N = 1: workload = BASELINE.json configs[1] (planted-community SBM, 4M rows,
-64M nnz).  Input prep (host RABBIT / RABBIT++ reorder, GPU plan + P A P^T)
-happens once and is reported separately (PAPER.md:221 amortisation).  A
-step is one spmv_exec y_B = B x_B over the whole matrix with x_B, B resident
-in HBM; L2 is flushed (512 MiB read) before every step, outside the CUDA
-events that time it, so each step pays compulsory traffic like the paper's
-ideal model.  value = ideal bytes / step time (GB/s);
-runtime / ideal = peak / value.
+Default workload, every N: BASELINE.json configs[4] -- power iteration on the
+Graph500 Kronecker scale-28 graph (268 M rows, 4.26 G nnz, int64 row
+pointers), row-block partitioned across the N GPUs, the largest
+configuration in BASELINE.json and the one its "1/2/4/8 B200" metric scales
+over.  A step is one power-iteration step of spmv_iterate (PAPER.md:221
+"SpMV iterations"; reading c22): the scaled SpMV y = B u / s over this rank's
+rows with the fixed-order sum of y^2, the all-reduce of that sum and the
+exchange of the y slices (N > 1).  K steps run as one spmv_iterate call,
+bracketed by a barrier + device synchronisation and timed with CUDA events on
+the launching stream; max over ranks.  B and x are resident in HBM; the
+matrix (37.8 GB) and x (1.07 GB) are far larger than the 126 MB L2, so no
+flush is needed between steps.
 
-N > 1 (torchrun): row-block power iteration on the same matrix, one rank per
-GPU: step = exec_scaled + NCCL all-reduce (8 B) + in-place all-gather of x;
-value = whole-job SpMV throughput (ideal bytes of the full B per step / max
-over ranks of the step time); scaling "strong".
+value = ideal bytes of one SpMV of the whole matrix (PAPER.md:96 with the
+real offset width) / step time, in GB/s, whole job; runtime / ideal =
+peak / value (peak = measured copy bandwidth).
+
+Input preparation is reported separately (PAPER.md:221 amortisation): the
+matrix is generated on the GPU (synth.config_gpu, the host generator's exact
+CSR), rank 0 reorders on the host (RABBIT / RABBIT++ with concurrent merges,
+SURVEY §8(f4)) and broadcasts the permutation, every rank builds its plan and
+B = P A P^T on its GPU.
+
+Configs 1-4 (--config k) time one plain spmv_exec per step with the L2
+flushed (a 512 MiB read and a reset of the persisting L2 lines) before every
+step, outside the events.
 
 --impl reference: the oracle (plain C fp64 CSR loop, oracle/c) timed on the
-host cores on the same workload, each step one full SpMV.
+host cores on a bounded sample of the same reordered workload.
+--suite: every config's paper ordering, one JSON line each plus the geometric
+mean of runtime / ideal (profiles/, not the driver's line).
 """
 from __future__ import annotations
 
@@ -37,6 +53,8 @@ sys.path.insert(0, ROOT)
 
 METRIC = "SpMV runtime & DRAM bytes ÷ ideal, achieved HBM GB/s, GFLOP/s at 1/2/4/8 B200"
 FALLBACK_HBM = 6650.0
+L2_BYTES = 126 * 2**20
+NCU_SUMMARY = os.path.join("profiles", "ncu_summary.json")
 
 
 def peaks():
@@ -89,15 +107,21 @@ class Clocks:
                 "samples": len(self.samples)}
 
 
-def load_workload(k: int):
-    import synth
-    t = time.perf_counter()
-    w = synth.config(k)
-    return w, time.perf_counter() - t
+def host_info():
+    """CPU model and core count of this host (lscpu), for cpu_baseline."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.startswith("Model name:"):
+                model = ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return {"model": model, "logical_cpus": os.cpu_count()}
 
 
 def ncu_traffic(workload: str, ordering: str):
-    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    p = os.path.join(ROOT, NCU_SUMMARY)
     if not os.path.exists(p):
         return None
     d = json.load(open(p))
@@ -105,28 +129,75 @@ def ncu_traffic(workload: str, ordering: str):
     return e if isinstance(e, dict) else None
 
 
-def reorder_cached(args, name, A, ordering, planted=None):
-    """spmv_reorder (host), optionally memoised on disk for development runs
-    (--perm-cache DIR); the default bench run always recomputes.  "planted" is
-    the generator's ground-truth order (SBM communities / stencil grid), a
-    reference point, not a method of the paper."""
+def ideal_bytes(n, nnz):
+    """PAPER.md:96 with the real row-offset width (reading c2)."""
+    return 2 * n * 4 + (n + 1) * (8 if nnz >= 2**31 else 4) + 2 * nnz * 4
+
+
+# ------------------------------------------------------------------ inputs
+class Inputs:
+    """The workload on this rank's device: row_ptr / col / val tensors, host x,
+    host pattern (rank 0, for the reorder), generator timing."""
+
+    def __init__(self, k, dev, need_host: bool):
+        import numpy as np
+        import torch
+
+        import synth
+        t = time.perf_counter()
+        self.k = k
+        if k in (1, 3, 5):   # RMAT / Kronecker: generated on the GPU
+            self.name, A, self.x = synth.config_gpu(k, device=dev.index or 0)
+            self.n, self.nnz = A.n, A.nnz
+            self.rp_d, self.col_d, self.val_d = A.row_ptr, A.col, A.val
+            self.host = A.to_host() if need_host else None
+            self.where = "gpu (synth_gpu, bit-identical to the host generator)"
+        else:
+            w = synth.config(k)
+            self.name, self.x, A = w.name, w.x, w.A
+            self.n, self.nnz = A.n, A.nnz
+            self.rp_d = torch.from_numpy(A.row_ptr).to(dev)
+            self.col_d = torch.from_numpy(A.col).to(dev)
+            self.val_d = torch.from_numpy(A.val).to(dev)
+            self.host = A
+            self.where = "host (synth)"
+        if self.nnz < 2**31:
+            self.rp_d = self.rp_d.to(torch.int32)
+        torch.cuda.synchronize(dev)
+        self.gen_s = time.perf_counter() - t
+        self.x = np.ascontiguousarray(self.x, np.float32)
+
+
+def reorder(args, inp, ordering):
+    """spmv_reorder on the host (rank 0); --perm-cache memoises for dev runs."""
     import numpy as np
     from paper_conf_ispass_balajicjk23_b200 import spmv
-    if ordering == "planted":
-        if planted is None:
-            raise SystemExit(f"workload {name} has no planted order")
-        return planted.astype(np.int32), spmv.ReorderStats(
-            **{f: 0 for f in spmv.ReorderStats.__dataclass_fields__})
     if args.perm_cache:
-        f = os.path.join(args.perm_cache, f"{name}_{ordering}_{args.seed}.npz")
+        f = os.path.join(args.perm_cache, f"{inp.name}_{ordering}_{args.seed}.npz")
         if os.path.exists(f):
             d = np.load(f, allow_pickle=True)
-            return d["perm"], spmv.ReorderStats(**d["stats"].item())
-    perm, st = spmv.reorder(A.row_ptr, A.col, ordering, seed=args.seed)
+            return d["perm"], d["stats"].item()
+    perm, st = spmv.reorder(inp.host.row_ptr, inp.host.col, ordering, seed=args.seed,
+                            parallel=ordering not in ("original", "random", "degsort")
+                            and not args.sequential_reorder)
+    st = dict(st.__dict__)
     if args.perm_cache:
         os.makedirs(args.perm_cache, exist_ok=True)
-        np.savez(f, perm=perm, stats=np.array(st.__dict__, dtype=object))
+        np.savez(f, perm=perm, stats=np.array(st, dtype=object))
     return perm, st
+
+
+def share_perm(perm, n, dev, world, rank):
+    """Rank 0's permutation to every rank (NCCL broadcast of the device copy)."""
+    import torch
+    import torch.distributed as dist
+    if rank == 0:
+        pd = torch.from_numpy(perm).to(dev)
+    else:
+        pd = torch.empty(n, dtype=torch.int32, device=dev)
+    if world > 1:
+        dist.broadcast(pd, src=0)
+    return pd
 
 
 # --------------------------------------------------------------------- GPU
@@ -149,116 +220,107 @@ def run_gpu(args):
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group(args.backend)
-    w, gen_s = load_workload(args.config)
-    A = w.A
+    iterate_mode = args.config == 5
+    inp = Inputs(args.config, dev, need_host=rank == 0)
     hbm, peak_src = peaks()
+    ideal = ideal_bytes(inp.n, inp.nnz)
     orderings = args.orderings.split(",")
     main = orderings[-1]
-    results = {}
-    rp_d = torch.from_numpy(A.row_ptr).to(dev)
-    col_d = torch.from_numpy(A.col).to(dev)
-    val_d = torch.from_numpy(A.val).to(dev)
-    if A.nnz < 2**31:
-        rp_d = rp_d.to(torch.int32)
-    # L2 flush by READING 512 MiB (4x L2): leaves L2 full of clean lines, so the
-    # timed step pays compulsory DRAM reads without write-backs of the flush
-    flush = torch.zeros(512 * 2**20 // 4, dtype=torch.float32, device=dev)
-    sink = torch.zeros((), dtype=torch.float32, device=dev)
+    stream = torch.cuda.Stream(device=dev)   # non-legacy: the L2 window is a stream attribute
+    torch.cuda.set_stream(stream)
+    flush = None
+    if not iterate_mode:
+        flush = torch.zeros(512 * 2**20 // 4, dtype=torch.float32, device=dev)
+        sink = torch.zeros((), dtype=torch.float32, device=dev)
+        lib = spmv.lib()
 
     def flush_l2():
+        # a 512 MiB read evicts normal lines; persisting lines (the plan's
+        # access-policy window on x_B[0:H)) need an explicit reset
         torch.sum(flush, dim=0, out=sink)
+        lib.spmv_reset_persisting_l2(None)
 
-    # a dedicated (non-legacy) stream: the L2 access-policy window of spmv_exec
-    # is a stream attribute and cannot be set on the legacy default stream
-    stream = torch.cuda.Stream()
-    torch.cuda.set_stream(stream)
-    line = None
+    comm = None
+    if world > 1 and args.backend == "nccl":
+        comm = pdist.nccl_comm_ptr(device=dev)
+    results, line, main_info = {}, None, None
     for ordering in orderings:
-        perm, st = reorder_cached(args, w.name, A, ordering, w.planted)
-        if ordering == main:
-            main_perm = perm
-        perm_d = torch.from_numpy(perm).to(dev)
-        torch.cuda.synchronize()
+        if rank == 0:
+            t = time.perf_counter()
+            perm, st = reorder(args, inp, ordering)
+            st["wall_s"] = time.perf_counter() - t
+        else:
+            perm, st = None, {}
+        if world > 1:
+            dist.barrier()
+        perm_d = share_perm(perm, inp.n, dev, world, rank)
+        torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
-        P = spmv.Plan(rp_d, col_d, val_d, perm_d, world=world, rank=rank, variant=args.variant)
-        torch.cuda.synchronize()
+        P = spmv.Plan(inp.rp_d, inp.col_d, inp.val_d, perm_d, world=world, rank=rank,
+                      variant=args.variant, nccl_comm=comm,
+                      exchange=spmv.EXCHANGE_PEER if args.exchange == "peer" else spmv.EXCHANGE_COLL)
+        torch.cuda.synchronize(dev)
         plan_s = time.perf_counter() - t0
         info = P.info()
-        x_d = torch.from_numpy(w.x).to(dev)
+        hc = pb = None
+        if world > 1 and args.backend != "nccl":
+            hc = pdist.HostColl(device=dev)
+            P.set_coll(hc.coll)
+        if world > 1 and args.exchange == "peer":
+            pb = pdist.PeerBuffers(P, dev)
+        x_d = torch.from_numpy(inp.x).to(dev)
         xB = P.permute_vec(x_d)
-        if world > 1:
-            xB = P.pad_vec(xB, to_padded=True)
-        ideal = 2 * A.n * 4 + (A.n + 1) * info["offset_bytes"] + 2 * A.nnz * 4
-        ideal_p96 = 2 * A.n * 4 + (A.n + 1 + 2 * A.nnz) * 4
-        launches = info["exec_launches"]
         is_main = ordering == main
-        fx = None
-        K = args.steps if is_main else max(10, args.steps // 4)
-        if world == 1:
-            y = torch.empty(A.n, dtype=torch.float32, device=dev)
+        K = args.steps if is_main else max(5, args.steps // 4)
+        y = torch.empty(max(info["row_end"] - info["row_begin"], 1), dtype=torch.float32, device=dev)
+        if iterate_mode:
+            xs = xB.clone()
+            launches_per_step = info["exec_launches"] + 1   # + the fixed-order norm
 
-            def step():
-                P.exec(xB, y)
+            def warm(w):
+                P.iterate(xs, w)
+
+            def timed(k):
+                P.iterate(xs, k)
         else:
-            loc = pdist.PlanLocal(P)
-            xa, xb = xB, torch.empty_like(xB)
-            ss = torch.zeros(2, dtype=torch.float64, device=dev)
-            state = {"t": 0, "xa": xa, "xb": xb, "ss_in": None}
-            M, off, nr = loc.x_stride, loc.y_offset, loc.nrows
+            launches_per_step = info["exec_launches"]
 
-            if args.exchange == "fused":  # y rows stored into every peer's x
-                fx = pdist.FusedExchange(P, dev, host_staged=args.backend != "nccl")
-                fx.x.copy_(xB)
-
-            def step():
-                t = state["t"]
-                ss_out = ss[t & 1:(t & 1) + 1]
-                if fx is not None:
-                    fx.step(state["ss_in"], ss_out)
-                    state["ss_in"] = ss_out
-                    state["t"] = t + 1
-                    return
-                P.exec_scaled(state["xa"], state["xb"][off:off + nr], state["ss_in"], ss_out)
-                if args.backend == "nccl":
-                    dist.all_reduce(ss_out)
-                    dist.all_gather_into_tensor(state["xb"], state["xb"][off:off + M])
-                else:  # gloo test path: host staging
-                    h = ss_out.cpu()
-                    dist.all_reduce(h)
-                    ss_out.copy_(h)
-                    hx = state["xb"].cpu()
-                    dist.all_gather_into_tensor(hx, hx[off:off + M].clone())
-                    state["xb"].copy_(hx)
-                state["ss_in"] = ss_out
-                state["xa"], state["xb"] = state["xb"], state["xa"]
-                state["t"] = t + 1
-            launches += 1  # exec_scaled's fixed-order norm reduction
-        for _ in range(args.warmup):
-            flush_l2()
-            step()
-        torch.cuda.synchronize()
-        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-              for _ in range(K)]
+            def warm(w):
+                for _ in range(w):
+                    flush_l2()
+                    P.exec(xB, y)
+        warm(args.warmup)
+        torch.cuda.synchronize(dev)
         clocks = Clocks(local) if is_main and rank == 0 else None
         if world > 1:
             dist.barrier()
-        torch.cuda.synchronize()
+        torch.cuda.synchronize(dev)
         if clocks:
             clocks.start()
             time.sleep(0.3)
         wall0 = time.perf_counter()
-        for i in range(K):
-            flush_l2()
-            ev[i][0].record(stream)
-            step()
-            ev[i][1].record(stream)
-        torch.cuda.synchronize()
+        if iterate_mode:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            timed(K)
+            e1.record(stream)
+            torch.cuda.synchronize(dev)
+            times = [e0.elapsed_time(e1) / K]
+        else:
+            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                  for _ in range(K)]
+            for i in range(K):
+                flush_l2()
+                ev[i][0].record(stream)
+                P.exec(xB, y)
+                ev[i][1].record(stream)
+            torch.cuda.synchronize(dev)
+            times = [a.elapsed_time(b) for a, b in ev]
         wall = time.perf_counter() - wall0
         if world > 1:
             dist.barrier()
         ck = clocks.stop() if clocks else None
-        times = [a.elapsed_time(b) for a, b in ev]
-        ms = sum(times) / K
+        ms = sum(times) / len(times)
         if world > 1:
             t = torch.tensor([ms], dtype=torch.float64, device=dev)
             if args.backend == "nccl":
@@ -268,105 +330,88 @@ def run_gpu(args):
                 dist.all_reduce(h, op=dist.ReduceOp.MAX)
                 t.copy_(h)
             ms = float(t.item())
-        # warm (no flush) back-to-back
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(K):
-            step()
-        e1.record(stream)
-        torch.cuda.synchronize()
-        warm_ms = e0.elapsed_time(e1) / K
-        graph_ms = None
-        if world == 1 and ideal < 256 * 2**20:
-            # small (L2-resident) matrices: launch overhead dominates a single
-            # exec, so also time G execs captured in one CUDA graph (warm)
-            G = 200
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=stream):
-                for _ in range(G):
-                    step()
-            g.replay()
-            torch.cuda.synchronize()
-            e0.record(stream)
-            for _ in range(5):
-                g.replay()
-            e1.record(stream)
-            torch.cuda.synchronize()
-            graph_ms = e0.elapsed_time(e1) / (5 * G)
         gbs = ideal / (ms * 1e-3) / 1e9
-        res = {"ms": ms, "ms_median": statistics.median(times), "warm_ms": warm_ms,
-               "graph_warm_ms": graph_ms,
-               "gbs_ideal_over_t": gbs, "gflops": 2 * A.nnz / (ms * 1e-3) / 1e9,
-               "runtime_over_ideal": hbm / gbs, "reorder_s": st.seconds, "plan_permute_s": plan_s,
-               "insularity": st.insularity, "insular_frac": st.insular_frac,
-               "n_communities": st.n_communities, "largest_comm_frac": st.largest_comm_frac,
-               "modularity": st.modularity, "skew": st.skew, "hubs": st.n_hubs,
-               "H": info["hot_prefix"], "tiles": info["n_tiles"], "cta_rows": info["n_cta_rows"],
-               "hub_rows": info["n_hub_rows"], "l2_window_bytes": P.info()["l2_window_bytes"],
+        res = {"ms": ms, "gbs_ideal_over_t": gbs, "gflops": 2 * inp.nnz / (ms * 1e-3) / 1e9,
+               "runtime_over_ideal": hbm / gbs, "reorder_s": st.get("seconds"),
+               "plan_permute_s": plan_s,
+               "H": info["hot_prefix"], "cta_rows": info["n_cta_rows"],
+               "mid_rows": info["n_mid_rows"], "hub_rows": info["n_hub_rows"],
+               "l2_window_bytes": P.info()["l2_window_bytes"],
                "stream_evict_first": info["stream_evict_first"]}
-        if world == 1 and not args.no_side:
-            # the paper's Table IV kernels on the same reordered matrix
-            res["spmm4"] = side_measure("spmm4", P, A, info, K, flush_l2, stream, dev, hbm)
-            res["coo"] = side_measure("coo", P, A, info, K, flush_l2, stream, dev, hbm)
-        tr = ncu_traffic(w.name, ordering)
+        if not iterate_mode:
+            res["ms_median"] = statistics.median(times)
+        for f in ("insularity", "insular_frac", "n_communities", "largest_comm_frac",
+                  "modularity", "skew", "n_hubs", "parallel", "n_deferred", "seconds_detect"):
+            if f in st:
+                res[f] = st[f]
+        if world > 1:
+            b = P.export_partition()
+            res["partition_rows"] = [b[k + 1] - b[k] for k in range(world)]
+        if world == 1 and not args.no_side and not iterate_mode:
+            res["spmm4"] = side_measure("spmm4", P, inp, info, K, flush_l2, stream, dev, hbm)
+            res["coo"] = side_measure("coo", P, inp, info, K, flush_l2, stream, dev, hbm)
+        tr = ncu_traffic(inp.name, ordering)
         if tr:
             res["dram_over_ideal_ncu"] = tr.get("dram_bytes", 0) / ideal
         results[ordering] = res
         if is_main:
-            if world == 1:
-                e2e = e2e_measure(P, A, w.x, args, dev, ideal)
+            main_info = dict(info)
+            if iterate_mode:
+                e2e = e2e_iterate(P, inp, perm_d, args, dev, ideal, world, rank)
             else:
-                state["xcur"] = (lambda: fx.x) if fx is not None else (lambda: state["xa"])
-                e2e = e2e_dist_measure(P, loc, w.x, perm, step_state=state, step=step, args=args,
-                                       dev=dev, ideal=ideal, world=world)
+                e2e = e2e_exec(P, inp, args, dev, ideal)
             line = dict(metric=METRIC, value=round(gbs, 2), unit="GB/s", n_gpus=world, steps=K,
                         warmup=args.warmup, ms_per_step=round(ms, 5), higher_is_better=True,
-                        scaling="strong", vs_baseline=None, dtype="f32",
-                        data="synthetic")
-            line["config"] = {"workload": f"{w.name} (BASELINE configs[{args.config - 1}])",
-                              "n": A.n, "nnz": A.nnz, "ordering": ordering,
-                              "parallelism": f"row-block x{world}" if world > 1 else "1 GPU",
-                              "step": "spmv_exec" if world == 1 else
-                              ("exec_scaled_bcast (fused NVLink peer stores) + all_reduce (power iteration)"
-                                       if args.exchange == "fused" else
-                                       "exec_scaled + all_reduce + all_gather (power iteration)"),
-                              "l2": "flushed before every step (512 MiB read, outside the events)",
-                              "ideal_bytes": ideal, "ideal_bytes_paper_4B_offsets": ideal_p96,
-                              "kernel_variant": ["lane", "panel"][args.variant],
-                              "wall_s_timed_region": round(wall, 4)}
+                        scaling="strong", vs_baseline=None, dtype="f32", data="synthetic")
+            line["config"] = {
+                "workload": f"{inp.name} (BASELINE configs[{args.config - 1}])",
+                "n": inp.n, "nnz": inp.nnz, "ordering": ordering,
+                "parallelism": f"row-block x{world}" if world > 1 else "1 GPU",
+                "step": ("spmv_iterate power-iteration step: exec_scaled over this rank's rows + "
+                         "fixed-order sum y^2" + (" + all-reduce + " + (
+                             "peer-store exchange (PEER)" if args.exchange == "peer" else
+                             "all-gatherv (grouped ncclBroadcast)") if world > 1 else ""))
+                if iterate_mode else "spmv_exec",
+                "l2": ("inputs larger than L2 (matrix %.1f GB, x %.2f GB vs 126 MB): no flush"
+                       % (ideal / 1e9, 4 * inp.n / 1e9)) if iterate_mode else
+                      "flushed before every step (512 MiB read + persisting-L2 reset, outside the events)",
+                "ideal_bytes": ideal,
+                "ideal_bytes_paper_4B_offsets": 2 * inp.n * 4 + (inp.n + 1 + 2 * inp.nnz) * 4,
+                "generator": inp.where,
+                "kernel_variant": ["lane", "panel"][args.variant],
+                "wall_s_timed_region": round(wall, 4)}
             line["runtime_over_ideal"] = round(hbm / gbs, 4)
-            line["gflops"] = round(2 * A.nnz / (ms * 1e-3) / 1e9, 2)
-            kern_bytes = ideal
-            line["roofline"] = {"bound": "hbm", "achieved": round(kern_bytes / (ms * 1e-3) / 1e9, 2),
-                                "peak": hbm, "unit": "GB/s",
-                                "frac": round(kern_bytes / (ms * 1e-3) / 1e9 / hbm, 4),
-                                "traffic": tr.get("dram_bytes") if tr else None,
-                                "kernel": ["k_lane", "k_panel"][args.variant] + " (+k_cta_rows/k_hub_* if present)",
-                                "peak_source": peak_src,
-                                "algorithmic_bytes_per_launch": kern_bytes}
+            line["gflops"] = round(2 * inp.nnz / (ms * 1e-3) / 1e9, 2)
+            line["roofline"] = {
+                "bound": "hbm", "achieved": round(gbs, 2), "peak": hbm, "unit": "GB/s",
+                "frac": round(gbs / hbm, 4),
+                "traffic": tr.get("dram_bytes") if tr else None,
+                "traffic_measured_in_run": False,
+                "traffic_source": NCU_SUMMARY if tr else None,
+                "kernel": "the SpMV of a step: k_lane + k_warp_rows + k_cta_rows + k_hub_chunk/"
+                          "k_hub_fix on three streams (one launch sequence per step)",
+                "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": ideal}
             line["e2e"] = e2e
-            line["gpu_launches"] = launches * K
+            line["gpu_launches"] = launches_per_step * K + (1 if iterate_mode else 0)
             line["clocks"] = ck
-            line["input_prep"] = {"generate_s": round(gen_s, 3), "reorder_s": round(st.seconds, 3),
+            line["input_prep"] = {"generate_s": round(inp.gen_s, 3),
+                                  "reorder_s": round(st.get("wall_s", 0.0), 3) if rank == 0 else None,
                                   "plan_permute_s": round(plan_s, 4)}
-        if fx is not None:
-            fx.close()
+        if pb is not None:
+            pb.close()
         P.close()
     line["orderings"] = {k: {kk: (round(vv, 5) if isinstance(vv, float) else vv)
                              for kk, vv in v.items()} for k, v in results.items()}
-    if "random" in results or "original" in results:
-        base = results.get("original") or results.get("random")
-        if base and main in results:
-            saving = base["ms"] - results[main]["ms"]
-            line["amortization_iters_vs_" + ("original" if "original" in results else "random")] = \
-                (results[main]["reorder_s"] * 1e3 / saving) if saving > 0 else None
+    base = results.get("random") or results.get("original")
+    if base and main in results and rank == 0:
+        saving = base["ms"] - results[main]["ms"]
+        rs = results[main].get("reorder_s") or 0.0
+        line["amortization_iters_vs_" + ("random" if "random" in results else "original")] = \
+            (rs * 1e3 / saving) if saving > 0 else None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        from oracle import permute as opermute
-        B = opermute.permute_csr_scipy(A.n, A.row_ptr, A.col, A.val, main_perm)
-        Bm = type("M", (), {"row_ptr": B[0], "col": B[1], "val": B[2]})()
-        line["cpu_baseline"] = cpu_baseline(Bm, opermute.permute_vec(w.x, main_perm),
-                                            ideal_bytes=line["config"]["ideal_bytes"])
+        perm, _ = reorder(args, inp, main)
+        line["cpu_baseline"] = cpu_baseline(inp, perm, budget_s=args.cpu_budget)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -374,25 +419,26 @@ def run_gpu(args):
         dist.destroy_process_group()
 
 
-def side_measure(kind, P, A, info, K, flush_l2, stream, dev, hbm):
+def side_measure(kind, P, inp, info, K, flush_l2, stream, dev, hbm):
     """Table IV kernels on the same plan, cold L2 like the
     SpMV steps, ideal traffic "updated according to the kernel":
       spmm4: 8 NZ + (N+1) w_off + 16 N (X) + 16 N (Y)
       coo:   12 NZ + 4 N (x) + 4 N (y)"""
     import torch
+    n, nnz = inp.n, inp.nnz
     if kind == "spmm4":
-        X = torch.empty((A.n, 4), dtype=torch.float32, device=dev).uniform_(-1, 1)
+        X = torch.empty((n, 4), dtype=torch.float32, device=dev).uniform_(-1, 1)
         Y = torch.empty_like(X)
-        ideal = 32 * A.n + (A.n + 1) * info["offset_bytes"] + 8 * A.nnz
-        flops = 8 * A.nnz
+        ideal = 32 * n + (n + 1) * info["offset_bytes"] + 8 * nnz
+        flops = 8 * nnz
 
         def run():
             P.exec_spmm4(X, Y)
     else:
-        X = torch.empty(A.n, dtype=torch.float32, device=dev).uniform_(-1, 1)
+        X = torch.empty(n, dtype=torch.float32, device=dev).uniform_(-1, 1)
         Y = torch.empty_like(X)
-        ideal = 8 * A.n + 12 * A.nnz
-        flops = 2 * A.nnz
+        ideal = 8 * n + 12 * nnz
+        flops = 2 * nnz
 
         def run():
             P.exec_coo(X, Y)
@@ -414,20 +460,20 @@ def side_measure(kind, P, A, info, K, flush_l2, stream, dev, hbm):
             "runtime_over_ideal": round(hbm / gbs, 4), "gflops": round(flops / (ms * 1e-3) / 1e9, 2)}
 
 
-def e2e_measure(P, A, x_host, args, dev, ideal):
+def e2e_exec(P, inp, args, dev, ideal):
     """Same metric through the public API with HOST buffers: pinned H2D of x,
     P x, exec, P^T y, D2H of y -- all inside the timed region.  Steps are
     software-pipelined over two buffer slots on three streams (H2D copy engine,
-    compute, D2H copy engine), as a serving loop would run it: step i+1's
-    upload and step i-1's download overlap step i's kernels."""
+    compute, D2H copy engine), as a serving loop would run it."""
     import torch
+    n = inp.n
     comp = torch.cuda.current_stream()
     s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
-    xh = torch.from_numpy(x_host).pin_memory()
-    yh = [torch.empty(A.n, dtype=torch.float32).pin_memory() for _ in range(2)]
-    xd = [torch.empty(A.n, dtype=torch.float32, device=dev) for _ in range(2)]
-    yd = [torch.empty(A.n, dtype=torch.float32, device=dev) for _ in range(2)]
-    xB = torch.empty(A.n, dtype=torch.float32, device=dev)
+    xh = torch.from_numpy(inp.x).pin_memory()
+    yh = [torch.empty(n, dtype=torch.float32).pin_memory() for _ in range(2)]
+    xd = [torch.empty(n, dtype=torch.float32, device=dev) for _ in range(2)]
+    yd = [torch.empty(n, dtype=torch.float32, device=dev) for _ in range(2)]
+    xB = torch.empty(n, dtype=torch.float32, device=dev)
     yB = torch.empty_like(xB)
     ev = {k: [torch.cuda.Event() for _ in range(2)] for k in ("h2d", "comp", "d2h")}
     started = [False, False]
@@ -435,13 +481,13 @@ def e2e_measure(P, A, x_host, args, dev, ideal):
     def step(i):
         b = i & 1
         if started[b]:
-            s_in.wait_event(ev["comp"][b])     # xd[b] no longer read
+            s_in.wait_event(ev["comp"][b])
         with torch.cuda.stream(s_in):
             xd[b].copy_(xh, non_blocking=True)
         ev["h2d"][b].record(s_in)
         comp.wait_event(ev["h2d"][b])
         if started[b]:
-            comp.wait_event(ev["d2h"][b])      # yd[b] already downloaded
+            comp.wait_event(ev["d2h"][b])
         P.permute_vec(xd[b], out=xB)
         P.exec(xB, yB)
         P.permute_vec(yB, inverse=True, out=yd[b])
@@ -465,7 +511,6 @@ def e2e_measure(P, A, x_host, args, dev, ideal):
     e1.record(comp)
     torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / K
-    # the downloaded y of the last step is the full public-API result
     xd[0].copy_(xh)
     P.permute_vec(xd[0], out=xB)
     P.exec(xB, yB)
@@ -473,75 +518,120 @@ def e2e_measure(P, A, x_host, args, dev, ideal):
     if not torch.equal(yd[0].cpu(), yh[(K - 1) & 1]):
         raise RuntimeError("e2e: pipelined result differs from a direct call")
     return {"value": round(ideal / (ms * 1e-3) / 1e9, 2), "unit": "GB/s", "ms_per_step": round(ms, 5),
-            "h2d_bytes_per_step": 4 * A.n, "d2h_bytes_per_step": 4 * A.n,
+            "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 4 * n,
             "path": "pinned H2D x -> spmv_permute_vec -> spmv_exec -> spmv_permute_vec^T -> D2H y "
                     "(two slots, copy engines overlapped with the kernels)"}
 
 
-def e2e_dist_measure(P, loc, x_host, perm, step_state, step, args, dev, ideal, world):
-    """N > 1: per step, pinned H2D of this rank's slice of x_B into its segment of
-    the padded x, the distributed step (exec_scaled + all-reduce + all-gather),
-    D2H of the 8-byte norm; max over ranks of the per-step time."""
+def e2e_iterate(P, inp, perm_d, args, dev, ideal, world, rank):
+    """The power iteration as a user calls it, from HOST memory: pinned H2D of
+    x_0, P x, spmv_iterate (K steps), P^T x, D2H of x_K and lambda -- all
+    inside the timed region; per-step bytes = the copies / K.  Max over
+    ranks."""
     import torch
     import torch.distributed as dist
-    b0, b1 = P.export_partition()[loc.rank], P.export_partition()[loc.rank + 1]
-    xB = P.permute_vec(torch.from_numpy(x_host).to(dev))  # setup, outside the timed region
-    xs = xB[b0:b1].cpu().pin_memory()
-    ssh = torch.empty(1, dtype=torch.float64).pin_memory()
-    off = loc.y_offset
-
-    def e2e_step():
-        step_state["xcur"]()[off:off + (b1 - b0)].copy_(xs, non_blocking=True)
-        step()
-        ssh.copy_(step_state["ss_in"], non_blocking=True)
-
-    for _ in range(args.warmup):
-        e2e_step()
-    torch.cuda.synchronize()
-    dist.barrier()
+    n, K = inp.n, args.steps
+    xh = torch.from_numpy(inp.x).pin_memory()
+    outh = torch.empty(n, dtype=torch.float32).pin_memory()
+    xd = torch.empty(n, dtype=torch.float32, device=dev)
+    xB = torch.empty(n, dtype=torch.float32, device=dev)
+    comp = torch.cuda.current_stream()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize(dev)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for _ in range(args.steps):
-        e2e_step()
-    e1.record()
-    torch.cuda.synchronize()
-    ms = e0.elapsed_time(e1) / args.steps
-    t = torch.tensor([ms], dtype=torch.float64)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX) if args.backend == "gloo" else None
-    if args.backend == "nccl":
-        td = t.to(dev)
-        dist.all_reduce(td, op=dist.ReduceOp.MAX)
-        t = td.cpu()
-    ms = float(t.item())
+    e0.record(comp)
+    xd.copy_(xh, non_blocking=True)
+    P.permute_vec(xd, out=xB)
+    lam = P.iterate(xB, K)
+    P.permute_vec(xB, inverse=True, out=xd)
+    outh.copy_(xd, non_blocking=True)
+    e1.record(comp)
+    torch.cuda.synchronize(dev)
+    ms = e0.elapsed_time(e1) / K
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        if args.backend == "nccl":
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        else:
+            h = t.cpu()
+            dist.all_reduce(h, op=dist.ReduceOp.MAX)
+            t.copy_(h)
+        ms = float(t.item())
+    if not (math.isfinite(lam) and lam > 0 and bool(torch.isfinite(outh).all())):
+        raise RuntimeError("e2e: power iteration result not finite")
     return {"value": round(ideal / (ms * 1e-3) / 1e9, 2), "unit": "GB/s", "ms_per_step": round(ms, 5),
-            "h2d_bytes_per_step": 4 * int(P.info()["n"]), "d2h_bytes_per_step": 8 * world,
-            "path": "pinned H2D of each rank's x slice -> spmv_exec_scaled -> NCCL all-reduce "
-                    "+ all-gather -> D2H of the norm (summed over ranks)"}
+            "h2d_bytes_per_step": round(4 * n / K, 1), "d2h_bytes_per_step": round((4 * n + 8) / K, 1),
+            "lambda": lam,
+            "path": "pinned H2D x_0 -> spmv_permute_vec -> spmv_iterate (K steps) -> "
+                    "spmv_permute_vec^T -> D2H x_K + lambda, copies amortised over K steps"}
 
 
 # ------------------------------------------------------------------- oracle
-def cpu_baseline(A, x, ideal_bytes, budget_s=10.0, steps=None, warmup=0):
-    """The oracle as it stands (plain C fp64 CSR loop, OpenMP over all host
-    cores) on the same workload; bounded sample of full SpMVs."""
+def oracle_sample(inp, perm, target_nnz=None):
+    """A bounded, contiguous row block of B = P A P^T built by the oracle's own
+    permutation (oracle.permute.permute_block) and x_B, for the CPU timing."""
+    import numpy as np
+
+    from oracle import permute as opermute
+    n, nnz = inp.n, inp.nnz
+    host = inp.host
+    inv = opermute.inverse(perm)
+    xB = opermute.permute_vec(inp.x, perm)
+    if target_nnz is None or target_nnz >= nnz:
+        r0, r1 = 0, n
+    else:   # a middle block of rows with about target_nnz entries of B
+        lenB = np.diff(host.row_ptr)[inv]
+        cum = np.concatenate([[0], np.cumsum(lenB)])
+        r0 = int(np.searchsorted(cum, (nnz - target_nnz) // 2))
+        r1 = int(np.searchsorted(cum, (nnz + target_nnz) // 2))
+    rp, col, val = opermute.permute_block(host.row_ptr, host.col, host.val, perm, inv, r0, r1)
+    return rp, col, val, xB, r0, r1
+
+
+def cpu_baseline(inp, perm, budget_s=10.0, steps=None, warmup=0):
+    """The oracle as it stands (plain C fp64 CSR loop, OpenMP over the host
+    cores, and the same loop on 1 core) on a bounded sample of the same
+    reordered workload, in the metric's unit (ideal bytes of the sample, P:96
+    restricted to its rows, per second).  Workloads above 2^28 entries are
+    sampled as a contiguous middle block of B's rows (~2^26 entries)."""
     from oracle import cref
-    threads = cref.threads()
-    for _ in range(warmup):
-        cref.spmv_f64(A.row_ptr, A.col, A.val, x)
-    times = []
-    t_start = time.perf_counter()
-    while True:
-        t = time.perf_counter()
-        cref.spmv_f64(A.row_ptr, A.col, A.val, x)
-        times.append(time.perf_counter() - t)
-        if steps is not None:
-            if len(times) >= steps:
+    big = inp.nnz > 2**28
+    rp, col, val, xB, r0, r1 = oracle_sample(inp, perm, target_nnz=2**26 if big else None)
+    m, rows = int(rp[-1]), r1 - r0
+    w_off = 8 if inp.nnz >= 2**31 else 4
+    sample_ideal = 8 * m + (rows + 1) * w_off + 8 * rows
+    desc = "all of B" if not big else \
+        f"rows {r0}..{r1} of B ({m} entries, {100.0 * m / inp.nnz:.2f} % of nnz)"
+
+    def timeit(threads, budget, nsteps, nwarm):
+        cref.threads(threads)
+        for _ in range(nwarm):
+            cref.spmv_f64(rp, col, val, xB)
+        times, t_start = [], time.perf_counter()
+        while True:
+            t = time.perf_counter()
+            cref.spmv_f64(rp, col, val, xB)
+            times.append(time.perf_counter() - t)
+            if nsteps is not None:
+                if len(times) >= nsteps:
+                    break
+            elif time.perf_counter() - t_start > budget:
                 break
-        elif time.perf_counter() - t_start > budget_s:
-            break
-    s = statistics.mean(times)
-    return {"value": round(ideal_bytes / s / 1e9, 3), "unit": "GB/s", "cores": threads,
-            "kind": "oracle", "ms_per_spmv": round(s * 1e3, 3),
-            "sample": f"{len(times)} full SpMVs of the workload (plain C fp64, OpenMP static nnz-balanced)"}
+        return statistics.mean(times), len(times)
+
+    ncpu = os.cpu_count() or 1
+    s_all, k_all = timeit(ncpu, budget_s, steps, warmup)
+    used = cref.threads(0)
+    s_one, k_one = timeit(1, budget_s / 2, None if steps is None else max(1, steps // 4), 0)
+    cref.threads(ncpu)
+    return {"value": round(sample_ideal / s_all / 1e9, 3), "unit": "GB/s", "cores": used,
+            "kind": "oracle", "ms_per_spmv": round(s_all * 1e3 * inp.nnz / max(m, 1), 3),
+            "sample": f"{k_all} SpMVs of {desc} (plain C fp64, OpenMP static nnz-balanced, "
+                      f"{used} threads); ms_per_spmv scaled to the whole matrix by nnz",
+            "one_core": {"value": round(sample_ideal / s_one / 1e9, 3), "unit": "GB/s", "cores": 1,
+                         "sample": f"{k_one} SpMVs of the same rows on 1 thread"},
+            "host": host_info()}
 
 
 def run_reference(args):
@@ -549,23 +639,22 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    w, _ = load_workload(args.config)
-    A = w.A
-    from paper_conf_ispass_balajicjk23_b200 import spmv
-    perm, _ = spmv.reorder(A.row_ptr, A.col, args.orderings.split(",")[-1], seed=args.seed)
-    from oracle import permute
-    Bp, Bc, Bv = permute.permute_csr_scipy(A.n, A.row_ptr, A.col, A.val, perm.astype("int64"))
-    xB = permute.permute_vec(w.x, perm)
-    ideal = 2 * A.n * 4 + (A.n + 1) * (8 if A.nnz >= 2**31 else 4) + 2 * A.nnz * 4
-    cb = cpu_baseline(type("M", (), {"row_ptr": Bp, "col": Bc, "val": Bv})(), xB, ideal,
-                      steps=args.steps, warmup=args.warmup)
-    ms = cb["ms_per_spmv"]
+    import torch
+    dev = torch.device("cuda", 0) if torch.cuda.is_available() else None
+    ordering = args.orderings.split(",")[-1]
+    if dev is None and args.config in (1, 3, 5):
+        raise SystemExit("--impl reference for this config needs the GPU generator")
+    inp = Inputs(args.config, dev, need_host=True)
+    perm, _ = reorder(args, inp, ordering)   # input preparation, outside the timed region
+    ideal = ideal_bytes(inp.n, inp.nnz)
+    cb = cpu_baseline(inp, perm, steps=args.steps, warmup=args.warmup)
     line = dict(metric=METRIC, value=cb["value"], unit="GB/s", n_gpus=world, steps=args.steps,
-                warmup=args.warmup, ms_per_step=ms, higher_is_better=True, scaling="strong",
-                vs_baseline=None, dtype="f64", data="synthetic", impl="reference",
-                config={"workload": f"{w.name} (BASELINE configs[{args.config - 1}])", "n": A.n,
-                        "nnz": A.nnz, "ordering": args.orderings.split(",")[-1],
-                        "ideal_bytes": ideal},
+                warmup=args.warmup, ms_per_step=cb["ms_per_spmv"], higher_is_better=True,
+                scaling="strong", vs_baseline=None, dtype="f64", data="synthetic", impl="reference",
+                config={"workload": f"{inp.name} (BASELINE configs[{args.config - 1}])", "n": inp.n,
+                        "nnz": inp.nnz, "ordering": ordering, "ideal_bytes": ideal,
+                        "step": "one SpMV of the sample (the oracle has no power-iteration driver of "
+                                "its own; the step is its SpMV)"},
                 cpu_baseline=cb,
                 e2e={"value": cb["value"], "unit": "GB/s", "h2d_bytes_per_step": 0,
                      "d2h_bytes_per_step": 0})
@@ -575,25 +664,33 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-based)")
-    ap.add_argument("--orderings", default="original,rabbit,rabbitpp",
-                    help="comma list; the last one is the headline line")
+    ap.add_argument("--config", type=int, default=5, help="BASELINE.json config index (1-based)")
+    ap.add_argument("--orderings", default=None,
+                    help="comma list; the last one is the headline line (default: "
+                         "original,rabbit,rabbitpp for config 5, random,original,rabbit,rabbitpp else)")
     ap.add_argument("--seed", type=int, default=20230423)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=10.0)
     ap.add_argument("--no-side", action="store_true",
                     help="skip the Table IV side measurements (SpMM-CSR-4, SpMV-COO)")
     ap.add_argument("--perm-cache", default=None, help="dev only: memoise reorder results here")
+    ap.add_argument("--sequential-reorder", action="store_true",
+                    help="RABBIT detection with the sequential (bit-exact) merge loop")
     ap.add_argument("--variant", type=int, default=0, help="short-row kernel: 0 lane, 1 panel")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="collectives for N > 1 (gloo: host-staged, test only)")
-    ap.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
-                    help="N > 1: NCCL all-gather of x, or the fused exec + NVLink peer stores")
+    ap.add_argument("--exchange", default="coll", choices=["coll", "peer"],
+                    help="N > 1: all-gatherv through the collective backend, or the SpMV's own "
+                         "peer stores (CUDA IPC over NVLink)")
     ap.add_argument("--single-device", action="store_true",
                     help="test only: put every rank on cuda:0 (with --backend gloo)")
     args = ap.parse_args()
+    if args.orderings is None:
+        args.orderings = "original,rabbit,rabbitpp" if args.config == 5 else \
+            "random,original,rabbit,rabbitpp"
     if args.warmup < 3:
         args.warmup = 3
     if args.impl == "reference":

@@ -79,6 +79,24 @@ def permute_rows(row_ptr, col, val, perm, inv, rows):
     return out
 
 
+def permute_block(row_ptr, col, val, perm, inv, r0: int, r1: int):
+    """Rows [r0, r1) of B = P A P^T as a CSR block (row_ptr rebased to 0):
+    row r of B is row inv[r] of A with columns relabelled by perm, stably
+    sorted by new column (the definition permute_csr follows), vectorised so
+    that a bounded sample of a billion-entry matrix is cheap to build."""
+    row_ptr = np.asarray(row_ptr, np.int64)
+    src = np.asarray(inv, np.int64)[r0:r1]
+    a, b = row_ptr[src], row_ptr[src + 1]
+    L = b - a
+    rp = np.concatenate([[0], np.cumsum(L)]).astype(np.int64)
+    m = int(rp[-1])
+    rowid = np.repeat(np.arange(r1 - r0, dtype=np.int64), L)
+    k = np.arange(m, dtype=np.int64) - np.repeat(rp[:-1], L) + np.repeat(a, L)
+    c = np.asarray(perm, np.int64)[np.asarray(col)[k].astype(np.int64)]
+    o = np.lexsort((np.arange(m), c, rowid))          # by row, then new column, stable
+    return rp, c[o].astype(np.int32), np.asarray(val, np.float32)[k][o]
+
+
 def permute_vec(x, perm, inverse_: bool = False) -> np.ndarray:
     """out = P x  (out[perm[i]] = x[i]);  inverse: out = P^T x (out[i] = x[perm[i]])."""
     x = np.asarray(x)

@@ -379,10 +379,22 @@ spmv_status spmv_export_coo_rows(spmv_plan_t p, int32_t* rows, void* stream) {
   API_END
 }
 
+spmv_status spmv_reset_persisting_l2(void* stream) {
+  (void)stream;
+  API_BEGIN
+  SPMV_CUDA(cudaCtxResetPersistingL2Cache());
+  API_END
+}
+
 void spmv_destroy(spmv_plan_t p) {
   if (!p) return;
   cudaSetDevice(p->device);
   cudaDeviceSynchronize();
+  if (p->l2_limit_raised) {  // the window raised the device-wide persisting limit
+    cudaCtxResetPersistingL2Cache();
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, p->l2_limit_before);
+    cudaGetLastError();
+  }
   spmv::plan_free(p);
   if (p->s) cudaStreamDestroy(p->s);
   delete p;

@@ -1056,7 +1056,13 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   if (bytes <= 0) return;
   size_t cur = 0;
   cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-  if ((int64_t)cur < bytes) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)bytes);
+  if ((int64_t)cur < bytes) {
+    if (!p->l2_limit_raised) {
+      p->l2_limit_before = cur;
+      p->l2_limit_raised = true;
+    }
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)bytes);
+  }
   cudaStreamAttrValue v{};
   v.accessPolicyWindow.base_ptr = (void*)x;
   v.accessPolicyWindow.num_bytes = (size_t)bytes;

@@ -110,6 +110,8 @@ struct spmv_plan_s {
   // state
   bool permuted = false;
   int64_t l2_window_bytes = 0;
+  bool l2_limit_raised = false;   // cudaLimitPersistingL2CacheSize raised by set_window
+  size_t l2_limit_before = 0;
   const void* win_ptr = nullptr;
   cudaStream_t win_stream[3] = {nullptr, nullptr, nullptr};
 };

@@ -39,11 +39,25 @@ void set_error(const std::string& m);
 
 namespace {
 
+bool verbose() {
+  static int v = -1;
+  if (v < 0) v = getenv("SPMV_REORDER_VERBOSE") ? 1 : 0;
+  return v == 1;
+}
+
+void phase(const char* what, std::chrono::steady_clock::time_point& t) {
+  auto now = std::chrono::steady_clock::now();
+  if (verbose())
+    fprintf(stderr, "[spmv_reorder] %-14s %8.3f s\n", what,
+            std::chrono::duration<double>(now - t).count());
+  t = now;
+}
+
 struct Sym {  // S = Bp + Bp^T in CSR, weights 1 or 2
   int64_t n = 0;
   std::vector<int64_t> ptr;
-  std::vector<int32_t> idx;
-  std::vector<uint8_t> w;
+  std::unique_ptr<int32_t[]> idx;  // uninitialised allocations: filled in parallel
+  std::unique_ptr<uint8_t[]> w;
 };
 
 void scan_inplace(std::vector<int64_t>& v) {  // exclusive, v has n+1 slots
@@ -55,48 +69,132 @@ void scan_inplace(std::vector<int64_t>& v) {  // exclusive, v has n+1 slots
   }
 }
 
+// parallel exclusive scan of cnt[0..n) into out[0..n], out[n] = total
+void scan_par(const int64_t* cnt, int64_t* out, int64_t n) {
+  const int T = omp_get_max_threads();
+  std::vector<int64_t> part(T + 1, 0);
+#pragma omp parallel num_threads(T)
+  {
+    const int t = omp_get_thread_num(), TT = omp_get_num_threads();
+    const int64_t lo = n * t / TT, hi = n * (t + 1) / TT;
+    int64_t s = 0;
+    for (int64_t i = lo; i < hi; ++i) s += cnt[i];
+    part[t + 1] = s;
+#pragma omp barrier
+#pragma omp single
+    for (int k = 1; k <= TT; ++k) part[k] += part[k - 1];
+    int64_t a = part[t];
+    for (int64_t i = lo; i < hi; ++i) {
+      const int64_t c = cnt[i];
+      out[i] = a;
+      a += c;
+    }
+  }
+  out[n] = part[T];
+}
+
+// S = Bp + Bp^T (reading c5).  Bp: per row sorted unique off-diagonal columns.
+// Bp^T without random atomics: a stable radix partition of the (column, row)
+// pairs into 2^16-column buckets (threads own contiguous row ranges, so each
+// bucket receives its pairs in ascending row order), then a stable counting
+// sort by column inside each bucket -- every transposed row comes out sorted.
+// Rows of Bp and Bp^T are then merged; an entry present in both gets weight 2.
 Sym symmetrize(int64_t n, const int64_t* rp, const int32_t* col) {
-  // Bp: per row sorted unique off-diagonal columns
+  const int64_t nnz = rp[n];
+  std::unique_ptr<int32_t[]> bidx(new int32_t[std::max<int64_t>(nnz, 1)]);
   std::vector<int64_t> bl(n + 1, 0);
-  std::vector<int32_t> bidx((size_t)rp[n]);
 #pragma omp parallel for schedule(dynamic, 1024)
   for (int64_t i = 0; i < n; ++i) {
-    int32_t* b = bidx.data() + rp[i];
+    int32_t* b = bidx.get() + rp[i];
     int64_t m = 0;
+    bool sorted = true;
     for (int64_t k = rp[i]; k < rp[i + 1]; ++k)
-      if (col[k] != i) b[m++] = col[k];
-    std::sort(b, b + m);
-    bl[i] = std::unique(b, b + m) - b;
-  }
-  // transpose: parallel counts and scatter with atomic cursors, then each
-  // transposed row sorted (the result is the same as a sequential transpose)
-  std::vector<int64_t> tcnt(n + 1, 0);
-#pragma omp parallel for schedule(dynamic, 1024)
-  for (int64_t i = 0; i < n; ++i)
-    for (int64_t k = 0; k < bl[i]; ++k)
-      __atomic_fetch_add(&tcnt[bidx[rp[i] + k]], (int64_t)1, __ATOMIC_RELAXED);
-  std::vector<int64_t> tptr(tcnt);
-  scan_inplace(tptr);
-  std::vector<int32_t> tidx((size_t)tptr[n]);
-  {
-    std::vector<int64_t> cur(tptr.begin(), tptr.end() - 1);
-#pragma omp parallel for schedule(dynamic, 1024)
-    for (int64_t i = 0; i < n; ++i)
-      for (int64_t k = 0; k < bl[i]; ++k) {
-        const int64_t pos = __atomic_fetch_add(&cur[bidx[rp[i] + k]], (int64_t)1, __ATOMIC_RELAXED);
-        tidx[pos] = (int32_t)i;
+      if (col[k] != i) {
+        if (m && col[k] <= b[m - 1]) sorted = false;
+        b[m++] = col[k];
       }
-#pragma omp parallel for schedule(dynamic, 1024)
-    for (int64_t j = 0; j < n; ++j) std::sort(tidx.begin() + tptr[j], tidx.begin() + tptr[j + 1]);
+    if (!sorted) {
+      std::sort(b, b + m);
+      m = std::unique(b, b + m) - b;
+    }
+    bl[i] = m;
   }
+  constexpr int SHIFT = 16;
+  const int64_t NB = (n >> SHIFT) + 1;
+  const int T = omp_get_max_threads();
+  // row ranges of the threads, balanced by entries
+  std::vector<int64_t> rlo(T + 1, n);
+  rlo[0] = 0;
+  for (int t = 1; t < T; ++t)
+    rlo[t] = std::lower_bound(rp, rp + n + 1, nnz * t / T) - rp;
+  for (int t = 1; t <= T; ++t) rlo[t] = std::max(rlo[t], rlo[t - 1]);
+  std::vector<int64_t> cnt((size_t)T * NB, 0);  // [t][bucket]
+#pragma omp parallel num_threads(T)
+  {
+    const int t = omp_get_thread_num();
+    int64_t* c = cnt.data() + (size_t)t * NB;
+    for (int64_t i = rlo[t]; i < rlo[t + 1]; ++i)
+      for (int64_t k = 0; k < bl[i]; ++k) c[bidx[rp[i] + k] >> SHIFT]++;
+  }
+  // bucket-major offsets: off[b][t]
+  std::vector<int64_t> off((size_t)NB * T + 1);
+  {
+    int64_t a = 0;
+    for (int64_t b = 0; b < NB; ++b)
+      for (int t = 0; t < T; ++t) {
+        off[(size_t)b * T + t] = a;
+        a += cnt[(size_t)t * NB + b];
+      }
+    off[(size_t)NB * T] = a;
+  }
+  const int64_t nt = off[(size_t)NB * T];
+  std::unique_ptr<uint64_t[]> pairs(new uint64_t[std::max<int64_t>(nt, 1)]);  // col << 32 | row
+#pragma omp parallel num_threads(T)
+  {
+    const int t = omp_get_thread_num();
+    std::vector<int64_t> cur(NB);
+    for (int64_t b = 0; b < NB; ++b) cur[b] = off[(size_t)b * T + t];
+    for (int64_t i = rlo[t]; i < rlo[t + 1]; ++i)
+      for (int64_t k = 0; k < bl[i]; ++k) {
+        const uint32_t j = (uint32_t)bidx[rp[i] + k];
+        pairs[cur[j >> SHIFT]++] = ((uint64_t)j << 32) | (uint32_t)i;
+      }
+  }
+  std::vector<int64_t> tptr(n + 1, 0);
+  std::unique_ptr<int32_t[]> tidx(new int32_t[std::max<int64_t>(nt, 1)]);
+#pragma omp parallel
+  {
+    std::vector<int64_t> cc((size_t)1 << SHIFT);
+#pragma omp for schedule(dynamic, 1)
+    for (int64_t b = 0; b < NB; ++b) {
+      const int64_t p0 = off[(size_t)b * T], p1 = off[(size_t)(b + 1) * T];
+      const int64_t j0 = b << SHIFT, j1 = std::min<int64_t>(n, (b + 1) << SHIFT);
+      std::fill(cc.begin(), cc.begin() + (j1 - j0), 0);
+      for (int64_t q = p0; q < p1; ++q) cc[(pairs[q] >> 32) - j0]++;
+      int64_t a = p0;
+      for (int64_t j = j0; j < j1; ++j) {
+        tptr[j] = a;
+        const int64_t c = cc[j - j0];
+        cc[j - j0] = a;
+        a += c;
+      }
+      for (int64_t q = p0; q < p1; ++q) {
+        const uint64_t e = pairs[q];
+        tidx[cc[(e >> 32) - j0]++] = (int32_t)(uint32_t)e;
+      }
+    }
+  }
+  tptr[n] = nt;
+  pairs.reset();
   // merge row i of Bp and Bp^T
   Sym S;
   S.n = n;
   S.ptr.assign(n + 1, 0);
+  std::vector<int64_t> len(n);
 #pragma omp parallel for schedule(dynamic, 1024)
   for (int64_t i = 0; i < n; ++i) {
-    const int32_t *a = bidx.data() + rp[i], *ae = a + bl[i];
-    const int32_t *b = tidx.data() + tptr[i], *be = tidx.data() + tptr[i + 1];
+    const int32_t *a = bidx.get() + rp[i], *ae = a + bl[i];
+    const int32_t *b = tidx.get() + tptr[i], *be = tidx.get() + tptr[i + 1];
     int64_t m = 0;
     while (a < ae || b < be) {
       if (b == be || (a < ae && *a < *b)) ++a;
@@ -104,15 +202,16 @@ Sym symmetrize(int64_t n, const int64_t* rp, const int32_t* col) {
       else { ++a; ++b; }
       ++m;
     }
-    S.ptr[i] = m;
+    len[i] = m;
   }
-  scan_inplace(S.ptr);
-  S.idx.resize((size_t)S.ptr[n]);
-  S.w.resize((size_t)S.ptr[n]);
+  scan_par(len.data(), S.ptr.data(), n);
+  const int64_t ns = S.ptr[n];
+  S.idx.reset(new int32_t[std::max<int64_t>(ns, 1)]);
+  S.w.reset(new uint8_t[std::max<int64_t>(ns, 1)]);
 #pragma omp parallel for schedule(dynamic, 1024)
   for (int64_t i = 0; i < n; ++i) {
-    const int32_t *a = bidx.data() + rp[i], *ae = a + bl[i];
-    const int32_t *b = tidx.data() + tptr[i], *be = tidx.data() + tptr[i + 1];
+    const int32_t *a = bidx.get() + rp[i], *ae = a + bl[i];
+    const int32_t *b = tidx.get() + tptr[i], *be = tidx.get() + tptr[i + 1];
     int64_t o = S.ptr[i];
     while (a < ae || b < be) {
       if (b == be || (a < ae && *a < *b)) { S.idx[o] = *a++; S.w[o++] = 1; }
@@ -321,6 +420,7 @@ struct HashAcc {  // per-thread (root -> summed weight) map, open addressing
 Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
   const int64_t n = S.n;
   constexpr int64_t PROC = -1, MLOCK = -2, MERGED = -3;
+  auto tp = std::chrono::steady_clock::now();
   std::vector<int64_t> deg(n);
 #pragma omp parallel for schedule(static)
   for (int64_t v = 0; v < n; ++v) {
@@ -358,130 +458,227 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
   std::vector<std::vector<int32_t>> tops(T), deferred(T);
   std::vector<std::vector<MergeRec>> logs(T);
   std::vector<int64_t> merges(T, 0), retries(T, 0);
+  std::vector<HashAcc> Hs(T);
+  phase("par:setup", tp);
 
-  // one sequential step on u; returns false when u must be deferred
-  auto step = [&](int32_t u, HashAcc& H, std::vector<Edge>& tl, int tid) -> bool {
+  auto expected = [&](int32_t u) {
+    size_t e = (size_t)(S.ptr[u + 1] - S.ptr[u]);
+    for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) e += agg[c].size();
+    return e;
+  };
+  // u's aggregated list: its S-row and its children's lists, neighbours
+  // mapped to their current roots, weights summed per root, u dropped
+  auto aggregate = [&](int32_t u, HashAcc& H, std::vector<Edge>& tl) {
+    H.prepare(expected(u));
+    for (int64_t k = S.ptr[u]; k < S.ptr[u + 1]; ++k) {
+      const int32_t r = find(S.idx[k]);
+      if (r != u) H.add(r, S.w[k]);
+    }
+    for (int32_t c = first_child[u]; c != -1; c = next_sib[c])
+      for (const Edge& e : agg[c]) {
+        const int32_t r = find(e.v);
+        if (r != u) H.add(r, e.w);
+      }
+    tl.clear();
+    for (uint32_t h : H.used) tl.push_back({H.key[h], H.val[h]});
+    H.clear();
+  };
+  // the same list with every thread (the tail phase, where the hubs with the
+  // largest aggregated lists come last and nothing else runs): chunks of the
+  // S-row and child lists hashed per thread, then a group-by on root % T
+  std::vector<std::vector<Edge>> parts((size_t)T * T), outs(T);
+  auto aggregate_all = [&](int32_t u, std::vector<Edge>& tl) {
+    struct Seg { int32_t c; int64_t b, e; };  // c = -1: S-row of u
+    std::vector<Seg> segs;
+    constexpr int64_t CH = 1 << 15;
+    for (int64_t b = S.ptr[u]; b < S.ptr[u + 1]; b += CH)
+      segs.push_back({-1, b, std::min<int64_t>(b + CH, S.ptr[u + 1])});
+    for (int32_t c = first_child[u]; c != -1; c = next_sib[c])
+      for (int64_t b = 0; b < (int64_t)agg[c].size(); b += CH)
+        segs.push_back({c, b, std::min<int64_t>(b + CH, (int64_t)agg[c].size())});
+    const size_t ex = expected(u);
+#pragma omp parallel num_threads(T)
+    {
+      const int t = omp_get_thread_num();
+      HashAcc& H = Hs[t];
+      H.prepare(ex);
+#pragma omp for schedule(dynamic, 1)
+      for (int64_t q = 0; q < (int64_t)segs.size(); ++q) {
+        const Seg& g = segs[q];
+        if (g.c < 0) {
+          for (int64_t k = g.b; k < g.e; ++k) {
+            const int32_t r = find(S.idx[k]);
+            if (r != u) H.add(r, S.w[k]);
+          }
+        } else {
+          const Edge* L = agg[g.c].data();
+          for (int64_t k = g.b; k < g.e; ++k) {
+            const int32_t r = find(L[k].v);
+            if (r != u) H.add(r, L[k].w);
+          }
+        }
+      }
+      for (uint32_t h : H.used) parts[(size_t)t * T + (uint32_t)H.key[h] % (uint32_t)T].push_back({H.key[h], H.val[h]});
+      H.clear();
+#pragma omp barrier
+      size_t m = 0;
+      for (int t2 = 0; t2 < T; ++t2) m += parts[(size_t)t2 * T + t].size();
+      H.prepare(m);
+      for (int t2 = 0; t2 < T; ++t2) {
+        for (const Edge& e : parts[(size_t)t2 * T + t]) H.add(e.v, e.w);
+        parts[(size_t)t2 * T + t].clear();
+      }
+      outs[t].clear();
+      for (uint32_t h : H.used) outs[t].push_back({H.key[h], H.val[h]});
+      H.clear();
+    }
+    tl.clear();
+    for (int t = 0; t < T; ++t) tl.insert(tl.end(), outs[t].begin(), outs[t].end());
+  };
+
+  // one step of the sequential reading on u.  mode 0: concurrent (returns
+  // false when u is deferred: its target is being processed, or u's
+  // aggregated list is large enough to deserve every thread later); mode 1:
+  // nothing else runs (no recheck needed); mode 2: as 1, aggregated with
+  // every thread
+  constexpr size_t BIG = (size_t)1 << 16;
+  std::vector<std::vector<int32_t>> bigs(T);
+  auto step = [&](int32_t u, HashAcc& H, std::vector<Edge>& tl, int tid, int mode) -> bool {
     int64_t tu;
     for (;;) {  // PROC-lock u (it may be the target of a short merge section)
       tu = tot[u].load(std::memory_order_acquire);
       if (tu == MLOCK) continue;
       if (tot[u].compare_exchange_weak(tu, PROC, std::memory_order_acq_rel)) break;
     }
+    if (mode == 0 && expected(u) > BIG) {
+      tot[u].store(tu, std::memory_order_release);
+      bigs[tid].push_back(u);
+      return false;
+    }
+    auto free_children = [&]() {
+      for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) std::vector<Edge>().swap(agg[c]);
+    };
     for (int attempt = 0;; ++attempt) {
-      size_t expect = (size_t)(S.ptr[u + 1] - S.ptr[u]);
-      for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) expect += agg[c].size();
-      H.prepare(expect);
-      for (int64_t k = S.ptr[u]; k < S.ptr[u + 1]; ++k) {
-        const int32_t r = find(S.idx[k]);
-        if (r != u) H.add(r, S.w[k]);
-      }
-      for (int32_t c = first_child[u]; c != -1; c = next_sib[c])
-        for (const Edge& e : agg[c]) {
-          const int32_t r = find(e.v);
-          if (r != u) H.add(r, e.w);
-        }
-      tl.clear();
+      if (mode == 2) aggregate_all(u, tl);
+      else aggregate(u, H, tl);
       int32_t best = -1;
       __int128 bestdq = 0;
-      for (uint32_t h : H.used) {
-        const int32_t r = H.key[h];
-        tl.push_back({r, H.val[h]});
-        const int64_t tr = tot[r].load(std::memory_order_acquire);
+      int64_t bestw = 0;
+      for (const Edge& e : tl) {
+        const int64_t tr = tot[e.v].load(std::memory_order_acquire);
         if (tr < 0) continue;  // being processed / locked / merged meanwhile
-        const __int128 dq = (__int128)two_m * H.val[h] - (__int128)tu * tr;
-        if (best == -1 || dq > bestdq || (dq == bestdq && r < best)) {
-          best = r;
+        const __int128 dq = (__int128)two_m * e.w - (__int128)tu * tr;
+        if (best == -1 || dq > bestdq || (dq == bestdq && e.v < best)) {
+          best = e.v;
           bestdq = dq;
+          bestw = e.w;
         }
       }
-      H.clear();
       if (best == -1 || bestdq <= 0) {
-        for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) std::vector<Edge>().swap(agg[c]);
+        free_children();
         tot[u].store(tu, std::memory_order_release);
         tops[tid].push_back(u);
         return true;
       }
-      // lock the target
-      int64_t tv = tot[best].load(std::memory_order_acquire);
-      bool locked = false, defer = false;
-      for (;;) {
-        if (tv == MLOCK) {
-          tv = tot[best].load(std::memory_order_acquire);
+      if (mode != 0) {  // exclusive: the aggregation is current, the gain exact
+        const int64_t tv = tot[best].load(std::memory_order_relaxed);
+        agg[u] = tl;
+        if (last_child[best] == -1) first_child[best] = u;
+        else next_sib[last_child[best]] = u;
+        last_child[best] = u;
+        parent[u].store(best, std::memory_order_relaxed);
+        tot[u].store(MERGED, std::memory_order_relaxed);
+        tot[best].store(tv + tu, std::memory_order_relaxed);
+        merges[tid]++;
+        if (want_log) logs[tid].push_back({u, best, (__int128)two_m * bestw - (__int128)tu * tv});
+        free_children();
+        return true;
+      }
+      // exact w(C_u, C_v) against a snapshot tv of the target's total.  tot
+      // only grows with merges into v (and turns MERGED when v itself merges),
+      // so a CAS that still finds tv proves C_v is the community w was
+      // computed against; the critical section is then just the bookkeeping.
+      int outcome = 0;  // 0: re-aggregate, 1: merged, 2: defer, 3: no gain
+      agg[u] = tl;      // published with the merge (read by v's processor later)
+      for (int k = 0; k < 16 && outcome == 0; ++k) {
+        int64_t tv = tot[best].load(std::memory_order_acquire);
+        while (tv == MLOCK) tv = tot[best].load(std::memory_order_acquire);
+        if (tv == PROC) { outcome = 2; break; }
+        if (tv == MERGED) break;
+        int64_t w = 0;
+        for (const Edge& e : tl)
+          if (find(e.v) == best) w += e.w;
+        const __int128 dq = (__int128)two_m * w - (__int128)tu * tv;
+        if (dq <= 0) { outcome = 3; break; }
+        int64_t expect = tv;
+        if (!tot[best].compare_exchange_strong(expect, MLOCK, std::memory_order_acq_rel)) {
+          retries[tid]++;
           continue;
         }
-        if (tv == PROC) { defer = true; break; }
-        if (tv == MERGED) break;  // merged meanwhile: aggregate again
-        if (tot[best].compare_exchange_weak(tv, MLOCK, std::memory_order_acq_rel)) {
-          locked = true;
-          break;
-        }
+        if (last_child[best] == -1) first_child[best] = u;
+        else next_sib[last_child[best]] = u;
+        last_child[best] = u;
+        parent[u].store(best, std::memory_order_release);
+        tot[u].store(MERGED, std::memory_order_release);
+        tot[best].store(tv + tu, std::memory_order_release);
+        merges[tid]++;
+        if (want_log) logs[tid].push_back({u, best, dq});
+        outcome = 1;
       }
-      if (defer || (!locked && attempt >= 3)) {
-        tot[u].store(tu, std::memory_order_release);
-        deferred[tid].push_back(u);
-        return false;
+      if (outcome == 1) {
+        free_children();
+        return true;
       }
-      if (!locked) {
-        retries[tid]++;
-        continue;
-      }
-      // exact w(C_u, C_v) under the lock
-      int64_t w = 0;
-      for (const Edge& e : tl)
-        if (find(e.v) == best) w += e.w;
-      const __int128 dq = (__int128)two_m * w - (__int128)tu * tv;
-      if (dq <= 0) {
-        tot[best].store(tv, std::memory_order_release);
-        if (attempt >= 3) {
-          for (int32_t c = first_child[u]; c != -1; c = next_sib[c])
-            std::vector<Edge>().swap(agg[c]);
+      std::vector<Edge>().swap(agg[u]);
+      if (outcome == 2 || attempt >= 3) {
+        if (outcome == 3) {  // the best gain vanished: u stays top level
+          free_children();
           tot[u].store(tu, std::memory_order_release);
           tops[tid].push_back(u);
           return true;
         }
-        retries[tid]++;
-        continue;
+        tot[u].store(tu, std::memory_order_release);
+        deferred[tid].push_back(u);
+        return false;
       }
-      for (int32_t c = first_child[u]; c != -1; c = next_sib[c]) std::vector<Edge>().swap(agg[c]);
-      agg[u] = tl;
-      if (last_child[best] == -1) first_child[best] = u;
-      else next_sib[last_child[best]] = u;
-      last_child[best] = u;
-      parent[u].store(best, std::memory_order_release);
-      tot[u].store(MERGED, std::memory_order_release);
-      merges[tid]++;
-      if (want_log) logs[tid].push_back({u, best, dq});
-      tot[best].store(tv + tu, std::memory_order_release);
-      return true;
+      retries[tid]++;
     }
   };
 
+  // every vertex in parallel (large aggregations postponed), then the
+  // deferred ones in processing order: the large ones with every thread
 #pragma omp parallel num_threads(T)
   {
     const int tid = omp_get_thread_num();
-    HashAcc H;
     std::vector<Edge> tl;
 #pragma omp for schedule(dynamic, 256)
-    for (int64_t oi = 0; oi < n; ++oi) step((int32_t)order[oi], H, tl, tid);
+    for (int64_t oi = 0; oi < n; ++oi) step((int32_t)order[oi], Hs[tid], tl, tid, 0);
   }
-  // deferred vertices: sequentially, in processing order
-  std::vector<int32_t> rest;
-  for (auto& d : deferred) rest.insert(rest.end(), d.begin(), d.end());
-  std::sort(rest.begin(), rest.end(), [&](int32_t a, int32_t b) { return pos[a] < pos[b]; });
+  phase("par:merges", tp);
   Rabbit R;
   R.parallel = true;
   R.two_m = two_m;
-  R.n_deferred = (int64_t)rest.size();
   {
-    HashAcc H;
+    std::vector<int32_t> rest;
+    for (auto& d : deferred) rest.insert(rest.end(), d.begin(), d.end());
+    R.n_deferred = (int64_t)rest.size();
+    for (auto& d : bigs) rest.insert(rest.end(), d.begin(), d.end());
+    std::sort(rest.begin(), rest.end(), [&](int32_t a, int32_t b) { return pos[a] < pos[b]; });
     std::vector<Edge> tl;
-    for (auto& d : deferred) d.clear();
-    for (int32_t u : rest)
-      if (!step(u, H, tl, 0)) {  // nothing runs concurrently now: cannot defer again
-        spmv::set_error("rabbit_detect_par: deferred vertex deferred again");
-        throw std::runtime_error("rabbit_detect_par");
-      }
+    double t_all = 0, t_one = 0;
+    int64_t n_all = 0;
+    for (int32_t u : rest) {
+      const bool all = expected(u) > BIG;
+      auto t0 = std::chrono::steady_clock::now();
+      step(u, Hs[0], tl, 0, all ? 2 : 1);
+      const double dt = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+      if (all) { t_all += dt; n_all++; } else t_one += dt;
+    }
+    if (verbose())
+      fprintf(stderr, "[spmv_reorder] deferred: %lld (%lld large, %.3f s), others %.3f s\n",
+              (long long)rest.size(), (long long)n_all, t_all, t_one);
   }
+  phase("par:tail", tp);
   for (int t = 0; t < T; ++t) {
     R.n_merges += merges[t];
     R.n_retries += retries[t];
@@ -494,6 +691,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
   std::sort(top.begin(), top.end(), [&](int32_t a, int32_t b) { return pos[a] < pos[b]; });
   std::vector<std::vector<Edge>>().swap(agg);
   dendrogram_ids(top, first_child, next_sib, R, n);
+  phase("par:dfs", tp);
   return R;
 }
 
@@ -539,20 +737,6 @@ uint64_t input_key(int64_t n, int64_t nnz, const int64_t* rp, const int32_t* col
   return mix64(a ^ mix64(b) ^ (uint64_t)n * 31 ^ (uint64_t)nnz);
 }
 }  // namespace
-
-static bool verbose() {
-  static int v = -1;
-  if (v < 0) v = getenv("SPMV_REORDER_VERBOSE") ? 1 : 0;
-  return v == 1;
-}
-
-static void phase(const char* what, std::chrono::steady_clock::time_point& t) {
-  auto now = std::chrono::steady_clock::now();
-  if (verbose())
-    fprintf(stderr, "[spmv_reorder] %-14s %8.3f s\n", what,
-            std::chrono::duration<double>(now - t).count());
-  t = now;
-}
 
 extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, const int32_t* col,
                                     int method, uint64_t seed, int32_t* perm_out,

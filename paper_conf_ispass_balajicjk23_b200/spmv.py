@@ -123,6 +123,7 @@ def lib() -> ctypes.CDLL:
             "spmv_export_partition": (i32, [vp, vp]),
             "spmv_export_inverse": (i32, [vp, vp, vp]),
             "spmv_destroy": (None, [vp]),
+            "spmv_reset_persisting_l2": (i32, [vp]),
             "spmv_reorder": (i32, [i64, i64, vp, vp, i32, ctypes.c_uint64, vp, ctypes.POINTER(_Stats)]),
             "spmv_reorder_last_comm": (i32, [i64, vp]),
             "spmv_reorder_last_merges": (i32, [i64, vp, vp, vp, ctypes.POINTER(ctypes.c_int64)]),

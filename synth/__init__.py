@@ -29,16 +29,27 @@ from . import gen  # noqa: F401  (reference loops)
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "libsynth.so")
 _SRC = os.path.join(_HERE, "csrc", "synth.cpp")
+_SO_GPU = os.path.join(_HERE, "libsynth_gpu.so")
+_SRC_GPU = os.path.join(_HERE, "csrc", "synth_gpu.cu")
 
 BASE_SEED = 20230423
 
 
 def build(force: bool = False) -> str:
-    """Compile libsynth.so in-tree (host C++, OpenMP)."""
+    """Compile libsynth.so (host C++, OpenMP) and libsynth_gpu.so (the RMAT /
+    Kronecker generator on the GPU, sm_100a) in-tree."""
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
         cmd = ["g++", "-O3", "-march=x86-64-v2", "-std=c++17", "-fopenmp", "-shared",
                "-fPIC", "-o", _SO, _SRC]
         subprocess.check_call(cmd)
+    if force or not os.path.exists(_SO_GPU) or \
+            os.path.getmtime(_SO_GPU) < os.path.getmtime(_SRC_GPU):
+        nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+        cmd = [nvcc, "-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a",
+               "-lineinfo", "-Xcompiler", "-fPIC", "-shared", "-o", _SO_GPU + ".tmp", _SRC_GPU,
+               "-lcudart"]
+        subprocess.check_call(cmd)
+        os.replace(_SO_GPU + ".tmp", _SO_GPU)
     return _SO
 
 
@@ -137,6 +148,85 @@ def stencil27(nx, periodic=False, relabel=True, seed_scr=0, valmode=VAL_SYM,
     return _take(m)
 
 
+class _GpuCsr(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("nnz", ctypes.c_int64),
+                ("row_ptr", ctypes.c_void_p), ("col", ctypes.c_void_p),
+                ("val", ctypes.c_void_p)]
+
+
+_lib_gpu = None
+
+
+def lib_gpu():
+    global _lib_gpu
+    if _lib_gpu is None:
+        build()
+        L = ctypes.CDLL(_SO_GPU)
+        u64, i64, i32, dbl = ctypes.c_uint64, ctypes.c_int64, ctypes.c_int, ctypes.c_double
+        L.synth_rmat_gpu.argtypes = [i32, i64, u64, dbl, dbl, dbl, i32, u64, i32, u64, i32,
+                                     ctypes.POINTER(_GpuCsr)]
+        L.synth_gpu_free.argtypes = [ctypes.POINTER(_GpuCsr)]
+        L.synth_gpu_error.restype = ctypes.c_char_p
+        _lib_gpu = L
+    return _lib_gpu
+
+
+class _DevArray:
+    """Owner of one cudaMalloc'ed array of a _GpuCsr (freed with the last view)."""
+
+    def __init__(self, owner, ptr, n, typestr):
+        self._owner = owner
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": typestr,
+                                         "data": (int(ptr) if ptr else 0, False), "version": 3}
+
+
+class _GpuOwner:
+    def __init__(self, m):
+        self.m = m
+
+    def __del__(self):
+        try:
+            lib_gpu().synth_gpu_free(ctypes.byref(self.m))
+        except Exception:
+            pass
+
+
+@dataclass
+class DeviceCsr:
+    """CSR on a CUDA device (torch tensors): row_ptr int64[n+1], col int32[nnz],
+    val float32[nnz]."""
+    n: int
+    row_ptr: object
+    col: object
+    val: object
+
+    @property
+    def nnz(self) -> int:
+        return int(self.col.numel())
+
+    def to_host(self) -> Csr:
+        return Csr(self.n, self.row_ptr.cpu().numpy(), self.col.cpu().numpy(),
+                   self.val.cpu().numpy())
+
+
+def rmat_gpu(scale, edge_factor=16, seed=1, a=0.57, b=0.19, c=0.19, scramble=False,
+             seed_scr=0, valmode=VAL_SYM, seed_v=0, device=0) -> DeviceCsr:
+    """rmat() generated on CUDA device `device` (bit-identical CSR)."""
+    import torch
+    m = _GpuCsr()
+    rc = lib_gpu().synth_rmat_gpu(scale, edge_factor, seed, a, b, c, int(scramble), seed_scr,
+                                  valmode, seed_v, int(device), ctypes.byref(m))
+    if rc:
+        raise RuntimeError(f"synth_rmat_gpu failed ({rc}): {lib_gpu().synth_gpu_error().decode()}")
+    own = _GpuOwner(m)
+    dev = torch.device("cuda", int(device))
+    t = lambda p, k, ts: torch.as_tensor(_DevArray(own, p, k, ts), device=dev)  # noqa: E731
+    nnz = int(m.nnz)
+    return DeviceCsr(int(m.n), t(m.row_ptr, m.n + 1, "<i8"),
+                     t(m.col, nnz, "<i4") if nnz else torch.zeros(0, dtype=torch.int32, device=dev),
+                     t(m.val, nnz, "<f4") if nnz else torch.zeros(0, dtype=torch.float32, device=dev))
+
+
 def vector(n, seed_x, mode=VAL_SYM) -> np.ndarray:
     out = np.empty(n, np.float32)
     lib().synth_vector(n, seed_x, mode, out.ctypes.data)
@@ -162,6 +252,26 @@ class Workload:
     x: np.ndarray
     planted: np.ndarray | None = None   # ground-truth order (SBM communities, stencil
                                         # grid), perm[old] = new; reference only
+
+
+def config_gpu(k: int, device=0, small: bool = False):
+    """The RMAT / Kronecker workloads (k = 1, 3, 5) generated on the GPU:
+    (name, DeviceCsr, x host float32) -- the same matrix as config(k)."""
+    se, sv, sx, ss = seeds(k)
+    if k == 1:
+        sc = 12 if small else 16
+        A = rmat_gpu(sc, 16, se, seed_v=sv, device=device)
+        return f"rmat{sc}", A, vector(A.n, sx)
+    if k == 3:
+        sc = 16 if small else 26
+        A = rmat_gpu(sc, 16, se, seed_v=sv, device=device)
+        return f"rmat{sc}", A, vector(A.n, sx)
+    if k == 5:
+        sc = 14 if small else 28
+        A = rmat_gpu(sc, 16, se, scramble=True, seed_scr=ss, valmode=VAL_POS, seed_v=sv,
+                     device=device)
+        return f"kron{sc}", A, np.full(A.n, np.float32(1.0 / np.sqrt(A.n)), np.float32)
+    raise ValueError(f"config {k} has no GPU generator")
 
 
 def config(k: int, small: bool = False) -> Workload:

@@ -67,3 +67,20 @@ def test_identity_perm_sorts_rows():
     rp = np.array([0, 3, 3])
     Bp, Bc, Bv = permute.permute_csr(2, rp, col, val, np.arange(2))
     assert list(Bc) == [0, 1, 1] and list(Bv) == [2, 1, 3]
+
+
+def test_permute_block_equals_definition():
+    """permute_block (the bounded-sample builder of bench.py's cpu_baseline)
+    gives exactly the rows of permute_csr, which is pinned to the dense
+    definition B[perm i, perm j] = A[i, j] above."""
+    import synth
+    from oracle import rabbit
+    A = synth.rmat(10, 8, 5, seed_v=2)
+    perm = rabbit.random_perm(A.n, 3)
+    inv = permute.inverse(perm)
+    Bp, Bc, Bv = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
+    for r0, r1 in ((0, A.n), (17, 400), (A.n - 5, A.n), (3, 3)):
+        rp, c, v = permute.permute_block(A.row_ptr, A.col, A.val, perm, inv, r0, r1)
+        assert np.array_equal(rp, Bp[r0:r1 + 1] - Bp[r0])
+        assert np.array_equal(c, Bc[Bp[r0]:Bp[r1]])
+        assert np.array_equal(v.view(np.int32), Bv[Bp[r0]:Bp[r1]].view(np.int32))
