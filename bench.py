@@ -2,7 +2,7 @@
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
                     [--config 5] [--orderings original,rabbit,rabbitpp]
-                    [--exchange coll|peer] [--suite]
+                    [--exchange coll|peer]
 
 Default workload, every N: BASELINE.json configs[4] -- power iteration on the
 Graph500 Kronecker scale-28 graph (268 M rows, 4.26 G nnz, int64 row
@@ -33,8 +33,7 @@ step, outside the events.
 
 --impl reference: the oracle (plain C fp64 CSR loop, oracle/c) timed on the
 host cores on a bounded sample of the same reordered workload.
---suite: every config's paper ordering, one JSON line each plus the geometric
-mean of runtime / ideal (profiles/, not the driver's line).
+scripts/suite.py runs every config and the geometric mean of runtime / ideal.
 """
 from __future__ import annotations
 
@@ -139,7 +138,7 @@ class Inputs:
     """The workload on this rank's device: row_ptr / col / val tensors, host x,
     host pattern (rank 0, for the reorder), generator timing."""
 
-    def __init__(self, k, dev, need_host: bool):
+    def __init__(self, k, dev, need_host: bool, small: bool = False):
         import numpy as np
         import torch
 
@@ -147,13 +146,16 @@ class Inputs:
         t = time.perf_counter()
         self.k = k
         if k in (1, 3, 5):   # RMAT / Kronecker: generated on the GPU
-            self.name, A, self.x = synth.config_gpu(k, device=dev.index or 0)
+            self.name, A, self.x = synth.config_gpu(k, device=dev.index or 0, small=small)
             self.n, self.nnz = A.n, A.nnz
             self.rp_d, self.col_d, self.val_d = A.row_ptr, A.col, A.val
-            self.host = A.to_host() if need_host else None
+            # the reorder needs the pattern only; values come to the host later
+            # (cpu_baseline), so the host never holds two copies at its peak
+            self.host = synth.Csr(A.n, A.row_ptr.cpu().numpy(), A.col.cpu().numpy(), None) \
+                if need_host else None
             self.where = "gpu (synth_gpu, bit-identical to the host generator)"
         else:
-            w = synth.config(k)
+            w = synth.config(k, small=small)
             self.name, self.x, A = w.name, w.x, w.A
             self.n, self.nnz = A.n, A.nnz
             self.rp_d = torch.from_numpy(A.row_ptr).to(dev)
@@ -221,7 +223,7 @@ def run_gpu(args):
         else:
             dist.init_process_group(args.backend)
     iterate_mode = args.config == 5
-    inp = Inputs(args.config, dev, need_host=rank == 0)
+    inp = Inputs(args.config, dev, need_host=rank == 0, small=args.small)
     hbm, peak_src = peaks()
     ideal = ideal_bytes(inp.n, inp.nnz)
     orderings = args.orderings.split(",")
@@ -576,6 +578,8 @@ def oracle_sample(inp, perm, target_nnz=None):
     from oracle import permute as opermute
     n, nnz = inp.n, inp.nnz
     host = inp.host
+    if host.val is None:
+        host.val = inp.val_d.cpu().numpy()
     inv = opermute.inverse(perm)
     xB = opermute.permute_vec(inp.x, perm)
     if target_nnz is None or target_nnz >= nnz:
@@ -644,7 +648,7 @@ def run_reference(args):
     ordering = args.orderings.split(",")[-1]
     if dev is None and args.config in (1, 3, 5):
         raise SystemExit("--impl reference for this config needs the GPU generator")
-    inp = Inputs(args.config, dev, need_host=True)
+    inp = Inputs(args.config, dev, need_host=True, small=args.small)
     perm, _ = reorder(args, inp, ordering)   # input preparation, outside the timed region
     ideal = ideal_bytes(inp.n, inp.nnz)
     cb = cpu_baseline(inp, perm, steps=args.steps, warmup=args.warmup)
@@ -685,6 +689,8 @@ def main():
     ap.add_argument("--exchange", default="coll", choices=["coll", "peer"],
                     help="N > 1: all-gatherv through the collective backend, or the SpMV's own "
                          "peer stores (CUDA IPC over NVLink)")
+    ap.add_argument("--small", action="store_true",
+                    help="test only: the same-shaped reduced instance of the config")
     ap.add_argument("--single-device", action="store_true",
                     help="test only: put every rank on cuda:0 (with --backend gloo)")
     args = ap.parse_args()

@@ -72,6 +72,8 @@ spmv_status spmv_plan(const spmv_csr_t* A, const int32_t* perm, const spmv_opts_
   if (p->opts.world < 1 || p->opts.rank < 0 || p->opts.rank >= p->opts.world)
     SPMV_FAIL(SPMV_EINVAL, "spmv_plan: need 0 <= rank < world");
   if (p->opts.world > 1024) SPMV_FAIL(SPMV_EUNSUPPORTED, "spmv_plan: world > 1024");
+  if (p->opts.hot_x > 0)
+    SPMV_FAIL(SPMV_EUNSUPPORTED, "spmv_plan: the hot-column set (opts.hot_x) was removed");
   if (!(p->opts.l2_hit_ratio >= 0.0 && p->opts.l2_hit_ratio <= 1.0))
     SPMV_FAIL(SPMV_EINVAL, "spmv_plan: l2_hit_ratio must be in [0, 1]");
   int dev = p->opts.device;
@@ -296,8 +298,6 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->stream_evict_first = spmv::lane_ef_mode(p);
   info->exec_launches = spmv::exec_launches(p, false);
   info->spmm4_launches = spmv::spmm4_launches(p);
-  info->hot_cols = p->hot_S;
-  info->hot_nnz = p->hot_nnz;
   API_END
 }
 

@@ -18,8 +18,6 @@ constexpr int WARP_MAX = 2048;      // warp-per-row class upper bound (canonical
 constexpr int CTA_MAX = 16384;      // CTA-per-row class upper bound
 constexpr int HUB_CHUNK = 16384;    // merge-path chunk of a hub row
 constexpr int CTA_THREADS = 256;    // canonical width of CTA / hub-chunk sums
-constexpr int HOT_MAX = 49152;      // hot-column set: <= 192 KB of x kept L1-resident
-constexpr int HOT_BINS = 1 << 16;   // exact column-count histogram bins
 constexpr int TILE_BUF = TILE_D + STREAM_MAX + 8;  // max entries of a tile (+ alignment slack)
 
 void set_error(const std::string& msg);

@@ -129,36 +129,9 @@ __device__ __forceinline__ double warp_sum_d(double s) {
   return s;
 }
 
-// x gather of the lane-mode kernels.  HOT == 0: plain L1-allocating __ldg.
-// HOT != 0 (hot-column set): a column coded c < 0 is hot and
-// read from the 192 KB contiguous copy xh[~c] with L1::evict_last, so the hot
-// lines stay L1-resident for the whole launch and cost no L2 request after
-// their first touch per SM; other columns are read with __ldg (HOT == 1) or
-// without allocating in L1 (HOT == 2), which keeps L1 for the hot copy.
-template <int HOT>
-__device__ __forceinline__ float gx(const float* __restrict__ x, const float* __restrict__ xh,
-                                    int c) {
-  if constexpr (HOT == 0) {
-    return __ldg(x + c);
-  } else {
-    float r;
-    if (c < 0) {
-      asm("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(r) : "l"(xh + ~c));
-    } else if constexpr (HOT == 1) {
-      r = __ldg(x + c);
-    } else {
-      asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(x + c));
-    }
-    return r;
-  }
-}
-
-__global__ void k_hot_gather(const float* __restrict__ x, const int32_t* __restrict__ hot_cols,
-                             int64_t S, float* __restrict__ xh) {
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S;
-       i += (int64_t)gridDim.x * blockDim.x)
-    xh[i] = x[hot_cols[i]];
-}
+// x gather of the lane-mode kernels: L1-allocating read-only load (community
+// order puts the columns of nearby rows on few lines)
+__device__ __forceinline__ float gx(const float* __restrict__ x, int c) { return __ldg(x + c); }
 
 // ------------------------------------------------------------ stream tiles
 // k_panel: persistent CTAs, each over a contiguous range of stream tiles (a
@@ -415,13 +388,12 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 }
 
 // ------------------------------------------------------------- long rows
-template <typename OT, bool SS, int HOT, int UNR = 4>
+template <typename OT, bool SS, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
                 float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
-                const double* __restrict__ ss_in, double* __restrict__ row_ss,
-                const float* __restrict__ xh, const YDst dst) {
+                const double* __restrict__ ss_in, double* __restrict__ row_ss, const YDst dst) {
   const int lane = threadIdx.x & 31;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float alpha = alpha_of(ss_in);
@@ -445,7 +417,7 @@ __global__ void __launch_bounds__(256)
         v[u] = pu ? __ldcs(vv + j + 32 * u) : 0.f;
       }
 #pragma unroll
-      for (int u = 0; u < UNR; ++u) xv[u] = (j + 32 * u < L) ? gx<HOT>(x, xh, c[u]) : 0.f;
+      for (int u = 0; u < UNR; ++u) xv[u] = (j + 32 * u < L) ? gx(x, c[u]) : 0.f;
 #pragma unroll
       for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
     }
@@ -459,60 +431,12 @@ __global__ void __launch_bounds__(256)
   fence_bcast<SS>(dst);
 }
 
-// k_warp_rows with the hot-column set in shared memory (hot mode 3): one
-// persistent 1024-thread CTA per SM stages xh (<= 192 KB) once; a gather of a
-// hot column (coded c < 0) is a shared-memory read, so it costs bank cycles
-// instead of an L1 wavefront per distinct line (profiles r33: the gathers of
-// power-law rows are L1-wavefront bound).  Same association as k_warp_rows.
-template <typename OT, bool SS>
-__global__ void __launch_bounds__(1024, 1)
-    k_warp_rows_smem(const OT* __restrict__ rp, const int32_t* __restrict__ col,
-                     const float* __restrict__ val, const float* __restrict__ x,
-                     float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
-                     const double* __restrict__ ss_in, double* __restrict__ row_ss,
-                     const float* __restrict__ xh, int hot_S) {
-  extern __shared__ float sx[];
-  for (int i = threadIdx.x; i < hot_S; i += blockDim.x) sx[i] = xh[i];
-  __syncthreads();
-  const int lane = threadIdx.x & 31;
-  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const float alpha = alpha_of(ss_in);
-  auto g = [&](int c) { return c < 0 ? sx[~c] : __ldg(x + c); };
-  for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < nrows; q += W) {
-    const int r = rows[q];
-    const int64_t b = (int64_t)rp[r];
-    const int L = (int)((int64_t)rp[r + 1] - b);
-    const int32_t* cc = col + b;
-    const float* vv = val + b;
-    float s = 0.f;
-    int j = lane;
-    for (; j + 96 < L; j += 128) {
-      const int c0 = __ldcs(cc + j), c1 = __ldcs(cc + j + 32), c2 = __ldcs(cc + j + 64),
-                c3 = __ldcs(cc + j + 96);
-      const float v0 = __ldcs(vv + j), v1 = __ldcs(vv + j + 32), v2 = __ldcs(vv + j + 64),
-                  v3 = __ldcs(vv + j + 96);
-      const float x0 = g(c0), x1 = g(c1), x2 = g(c2), x3 = g(c3);
-      s = __fadd_rn(s, __fmul_rn(v0, x0));
-      s = __fadd_rn(s, __fmul_rn(v1, x1));
-      s = __fadd_rn(s, __fmul_rn(v2, x2));
-      s = __fadd_rn(s, __fmul_rn(v3, x3));
-    }
-    for (; j < L; j += 32) s = __fadd_rn(s, __fmul_rn(__ldcs(vv + j), g(__ldcs(cc + j))));
-    s = warp_tree(s);
-    if (lane == 0) {
-      const float v = __fmul_rn(s, alpha);
-      y[r] = v;
-      if (SS) row_ss[q] = (double)v * (double)v;
-    }
-  }
-}
-
 // canonical W = 256 sum of entries [b, b + L) of a row
-template <int HOT, int UNR = 4>
+template <int UNR = 4>
 __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             const float* __restrict__ val,
                                             const float* __restrict__ x, int64_t b, int64_t L,
-                                            float* red, const float* __restrict__ xh) {
+                                            float* red) {
   const int tid = threadIdx.x;
   float s = 0.f;
   // UNR strided entries in flight, ragged end guarded (+0 slots, as k_warp_rows)
@@ -526,7 +450,7 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
       v[u] = pu ? __ldcs(val + b + t + 256 * u) : 0.f;
     }
 #pragma unroll
-    for (int u = 0; u < UNR; ++u) xv[u] = (t + 256 * u < L) ? gx<HOT>(x, xh, c[u]) : 0.f;
+    for (int u = 0; u < UNR; ++u) xv[u] = (t + 256 * u < L) ? gx(x, c[u]) : 0.f;
 #pragma unroll
     for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
   }
@@ -542,16 +466,16 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
   return r;  // valid in thread 0
 }
 
-template <typename OT, bool SS, int HOT, int UNR = 4>
+template <typename OT, bool SS, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_cta_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
                const int32_t* __restrict__ rows, const double* __restrict__ ss_in,
-               double* __restrict__ row_ss, const float* __restrict__ xh, const YDst dst) {
+               double* __restrict__ row_ss, const YDst dst) {
   __shared__ float red[256];
   const int r = rows[blockIdx.x];
   const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
-  const float s = cta_sum256<HOT, UNR>(col, val, x, b, L, red, xh);
+  const float s = cta_sum256<UNR>(col, val, x, b, L, red);
   if (threadIdx.x == 0) {
     const float v = __fmul_rn(s, alpha_of(ss_in));
     store_y<SS>(y, dst, r, v);
@@ -560,95 +484,20 @@ __global__ void __launch_bounds__(256)
   }
 }
 
-template <typename OT, int HOT, int UNR = 4>
+template <typename OT, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_hub_chunk(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
                 const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_idx,
-                double* __restrict__ part, const float* __restrict__ xh) {
+                double* __restrict__ part) {
   __shared__ float red[256];
   const int c = blockIdx.x;
   const int r = chunk_row[c];
   const int64_t rb = (int64_t)rp[r], L = (int64_t)rp[r + 1] - rb;
   const int64_t b = rb + (int64_t)chunk_idx[c] * HUB_CHUNK;
   const int64_t m = min((int64_t)HUB_CHUNK, rb + L - b);
-  const float s = cta_sum256<HOT, UNR>(col, val, x, b, m, red, xh);
+  const float s = cta_sum256<UNR>(col, val, x, b, m, red);
   if (threadIdx.x == 0) part[c] = (double)s;
-}
-
-// CTA rows and hub chunks with the hot-column set in shared memory (hot
-// mode 3): one persistent 1024-thread CTA per SM stages xh once; its four
-// 256-thread groups take work items (CTA rows first, then hub chunks) in a
-// fixed round robin and reduce each with the canonical W = 256 association of
-// cta_sum256 (group-local named barriers), so y is bitwise that of
-// k_cta_rows / k_hub_chunk.
-template <typename OT, bool SS>
-__global__ void __launch_bounds__(1024, 1)
-    k_long_rows_smem(const OT* __restrict__ rp, const int32_t* __restrict__ col,
-                     const float* __restrict__ val, const float* __restrict__ x,
-                     float* __restrict__ y, const int32_t* __restrict__ cta_rows, int64_t n_cta,
-                     const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_idx,
-                     int64_t n_chunks, double* __restrict__ part, const double* __restrict__ ss_in,
-                     double* __restrict__ row_ss, const float* __restrict__ xh, int hot_S) {
-  extern __shared__ float sx[];
-  __shared__ float red[4][256];
-  for (int i = threadIdx.x; i < hot_S; i += blockDim.x) sx[i] = xh[i];
-  __syncthreads();
-  const int grp = threadIdx.x >> 8, t0 = threadIdx.x & 255;
-  float* rd = red[grp];
-  const float alpha = alpha_of(ss_in);
-  auto g = [&](int c) { return c < 0 ? sx[~c] : __ldg(x + c); };
-  auto bar = [&]() { asm volatile("bar.sync %0, 256;" ::"r"(grp + 1) : "memory"); };
-  const int64_t total = n_cta + n_chunks;
-  for (int64_t it = (int64_t)blockIdx.x * 4 + grp; it < total; it += (int64_t)gridDim.x * 4) {
-    int64_t b, L;
-    int r = -1;
-    if (it < n_cta) {
-      r = cta_rows[it];
-      b = (int64_t)rp[r];
-      L = (int64_t)rp[r + 1] - b;
-    } else {
-      const int64_t c = it - n_cta;
-      const int hr = chunk_row[c];
-      const int64_t rb = (int64_t)rp[hr], RL = (int64_t)rp[hr + 1] - rb;
-      b = rb + (int64_t)chunk_idx[c] * HUB_CHUNK;
-      L = min((int64_t)HUB_CHUNK, rb + RL - b);
-    }
-    float s = 0.f;
-    int64_t t = t0;
-    for (; t + 768 < L; t += 1024) {
-      const int c0 = __ldcs(col + b + t), c1 = __ldcs(col + b + t + 256),
-                c2 = __ldcs(col + b + t + 512), c3 = __ldcs(col + b + t + 768);
-      const float v0 = __ldcs(val + b + t), v1 = __ldcs(val + b + t + 256),
-                  v2 = __ldcs(val + b + t + 512), v3 = __ldcs(val + b + t + 768);
-      const float x0 = g(c0), x1 = g(c1), x2 = g(c2), x3 = g(c3);
-      s = __fadd_rn(s, __fmul_rn(v0, x0));
-      s = __fadd_rn(s, __fmul_rn(v1, x1));
-      s = __fadd_rn(s, __fmul_rn(v2, x2));
-      s = __fadd_rn(s, __fmul_rn(v3, x3));
-    }
-    for (; t < L; t += 256) s = __fadd_rn(s, __fmul_rn(__ldcs(val + b + t), g(__ldcs(col + b + t))));
-    rd[t0] = s;
-    bar();
-#pragma unroll
-    for (int o = 128; o >= 32; o >>= 1) {
-      if (t0 < o) rd[t0] = __fadd_rn(rd[t0], rd[t0 + o]);
-      bar();
-    }
-    if (t0 < 32) {
-      const float w = warp_tree(rd[t0]);
-      if (t0 == 0) {
-        if (it < n_cta) {
-          const float v = __fmul_rn(w, alpha);
-          y[r] = v;
-          if (SS) row_ss[it] = (double)v * (double)v;
-        } else {
-          part[it - n_cta] = (double)w;
-        }
-      }
-    }
-    bar();  // rd is reused by the group's next item
-  }
 }
 
 template <bool SS>
@@ -692,17 +541,6 @@ int g_num_sms = 0;
 int num_sms(int dev) {
   if (!g_num_sms) cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
   return g_num_sms > 0 ? g_num_sms : 148;
-}
-
-// 0: no hot-column set; 1 / 2: the MID / CTA / hub kernels read hot columns
-// from the L1-resident copy (cold: __ldg / no L1 allocation);
-// 3 (default): k_warp_rows_smem keeps the hot copy in shared memory, the other
-// kernels read the plain col array.  SPMV_HOT_MODE dev knob.
-int hot_mode(const spmv_plan_s* p) {
-  if (!p->hot_S || !p->d_col_hot || p->opts.variant == 1) return 0;
-  int m = 3;
-  if (const char* e = getenv("SPMV_HOT_MODE")) m = std::min(3, std::max(1, atoi(e)));
-  return m;
 }
 
 // cudaFuncSetAttribute acts on the current device, so the max-dynamic-smem
@@ -789,12 +627,12 @@ __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
 // minBlocksPerSM = 1 lets ptxas keep both chunks and all 16 gathers of a
 // 16-entry row in flight per lane (64 registers, 4 CTAs/SM); capping registers
 // for more CTAs measured 20-40 % slower
-template <typename OT, bool SS, int EF, int HOT>
+template <typename OT, bool SS, int EF>
 __global__ void __launch_bounds__(LN_THREADS, 1)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
            int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss,
-           const float* __restrict__ xh, const YDst dst) {
+           const YDst dst) {
   __shared__ double wss[LN_WARPS];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
@@ -845,7 +683,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
           }
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
-            const float xv = gx<HOT>(x, xh, cc[i]);
+            const float xv = gx(x, cc[i]);
             res = __fadd_rn(res, (k + i >= lo && k + i < hi) ? __fmul_rn(vv[i], xv) : 0.f);
           }
         }
@@ -872,7 +710,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
   fence_bcast<SS>(dst);
 }
 
-template <typename OT, bool SS, int EF, int HOT>
+template <typename OT, bool SS, int EF>
 void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s,
                    const YDst& dst) {
   // grid-stride with ~8 CTAs per resident slot (measured better than one
@@ -882,9 +720,8 @@ void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in
   const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
   const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
-  k_lane<OT, SS, EF, HOT><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col,
-                                                        p->d_val, x, y, p->nrows, ss_in,
-                                                        p->d_blk_ss, p->d_xh, dst);
+  k_lane<OT, SS, EF><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
+                                                   p->nrows, ss_in, p->d_blk_ss, dst);
 }
 
 }  // namespace
@@ -903,74 +740,50 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   // normal, the rest evict_first) via the SPMV_LANE_EF dev knob
   int ef = lane_ef_mode(p);
   if (const char* e = getenv("SPMV_LANE_EF")) ef = std::min(2, std::max(0, atoi(e)));  // dev knob
-  if (ef == 1) launch_lane_t<OT, SS, 1, 0>(p, x, y, ss_in, s, dst);
-  else if (ef == 2) launch_lane_t<OT, SS, 2, 0>(p, x, y, ss_in, s, dst);
-  else launch_lane_t<OT, SS, 0, 0>(p, x, y, ss_in, s, dst);
+  if (ef == 1) launch_lane_t<OT, SS, 1>(p, x, y, ss_in, s, dst);
+  else if (ef == 2) launch_lane_t<OT, SS, 2>(p, x, y, ss_in, s, dst);
+  else launch_lane_t<OT, SS, 0>(p, x, y, ss_in, s, dst);
 }
 
-// Row-class kernels other than the short-row one.  HOT 1/2: every gather
-// uses the coded columns; HOT 3: only the MID rows (k_warp_rows_smem, hot copy
-// in shared memory), the CTA / hub classes read the plain columns.
-template <typename OT, bool SS, int HOT>
+// Row-class kernels other than the short-row one: MID rows (warp per row),
+// CTA rows, hub chunks + fixup, on the two plan-owned streams s1 / s2.
+template <typename OT, bool SS>
 void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s1,
                  cudaStream_t s2, bool lane_mode, const YDst& dst) {
-  constexpr int HG = HOT == 3 ? 0 : HOT;  // gather variant of the CTA / hub (and MID) kernels
   const OT* rp = (const OT*)p->d_rp;
-  const int32_t* col = HG ? p->d_col_hot : p->d_col;
+  const int32_t* col = p->d_col;
   const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
   const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
   double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
-  if (nw && HOT == 3) {
-    max_dyn_smem<k_warp_rows_smem<OT, SS>>((int)(sizeof(float) * HOT_MAX), p->device);
-    const size_t smem = sizeof(float) * (size_t)p->hot_S;
-    k_warp_rows_smem<OT, SS><<<(unsigned)num_sms(p->device), 1024, smem, s1>>>(
-        rp, p->d_col_hot, p->d_val, x, y, wr, nw, ss_in, wss, p->d_xh, (int)p->hot_S);
-  } else if (nw) {
+  if (nw) {
     const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
     int unr = 4;  // entries in flight per lane (same association for any value)
     if (const char* e = getenv("SPMV_WARP_UNR")) unr = atoi(e) == 8 ? 8 : 4;  // dev knob
     if (unr == 8)
-      k_warp_rows<OT, SS, HG, 8><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss,
-                                                    p->d_xh, dst);
+      k_warp_rows<OT, SS, 8><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, dst);
     else
-      k_warp_rows<OT, SS, HG, 4><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss,
-                                                    p->d_xh, dst);
-  }
-  const bool long_smem = HOT == 3 && (p->n_cta || p->n_chunks);
-  if (long_smem) {
-    max_dyn_smem<k_long_rows_smem<OT, SS>>((int)(sizeof(float) * HOT_MAX), p->device);
-    const size_t smem = sizeof(float) * (size_t)p->hot_S;
-    const int64_t items = p->n_cta + p->n_chunks;
-    const unsigned g = (unsigned)std::min<int64_t>((items + 3) / 4, num_sms(p->device));
-    k_long_rows_smem<OT, SS><<<g, 1024, smem, s2>>>(
-        rp, p->d_col_hot, p->d_val, x, y, p->d_cta_rows, p->n_cta, p->d_chunk_row,
-        p->d_chunk_idx, p->n_chunks, p->d_chunk_part, ss_in, p->d_cta_ss, p->d_xh,
-        (int)p->hot_S);
+      k_warp_rows<OT, SS, 4><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, dst);
   }
   int cunr = 4;  // entries in flight per thread (same association for any value)
   if (const char* e = getenv("SPMV_CTA_UNR")) cunr = atoi(e) == 8 ? 8 : 4;  // dev knob
-  if (!long_smem && p->n_cta) {
+  if (p->n_cta) {
     if (cunr == 8)
-      k_cta_rows<OT, SS, HG, 8><<<(unsigned)p->n_cta, 256, 0, s2>>>(
-          rp, col, p->d_val, x, y, p->d_cta_rows, ss_in, p->d_cta_ss, p->d_xh, dst);
+      k_cta_rows<OT, SS, 8><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
+                                                                 p->d_cta_rows, ss_in, p->d_cta_ss, dst);
     else
-      k_cta_rows<OT, SS, HG, 4><<<(unsigned)p->n_cta, 256, 0, s2>>>(
-          rp, col, p->d_val, x, y, p->d_cta_rows, ss_in, p->d_cta_ss, p->d_xh, dst);
+      k_cta_rows<OT, SS, 4><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
+                                                                 p->d_cta_rows, ss_in, p->d_cta_ss, dst);
   }
   if (p->n_chunks) {
-    if (!long_smem && cunr == 8)
-      k_hub_chunk<OT, HG, 8><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
-          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part, p->d_xh);
-    else if (!long_smem)
-      k_hub_chunk<OT, HG, 4><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
-          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part, p->d_xh);
-    const unsigned g = (unsigned)((p->n_hub + 127) / 128);
-    if (SS)
-      k_hub_fix<true><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
-                                         ss_in, y, p->d_hub_ss, dst);
+    if (cunr == 8)
+      k_hub_chunk<OT, 8><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
+          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part);
     else
-      k_hub_fix<false><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub,
-                                          p->d_chunk_part, ss_in, y, p->d_hub_ss, dst);
+      k_hub_chunk<OT, 4><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
+          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part);
+    const unsigned g = (unsigned)((p->n_hub + 127) / 128);
+    k_hub_fix<SS><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
+                                      ss_in, y, p->d_hub_ss, dst);
   }
 }
 
@@ -979,10 +792,6 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
                 cudaStream_t s, const YDst& dst) {
   const bool SS = ss_out != nullptr;
   const bool lane_mode = p->opts.variant != 1;
-  if (lane_mode && hot_mode(p)) {  // refresh the hot copy of x for this exec
-    const unsigned g = (unsigned)std::min<int64_t>((p->hot_S + 255) / 256, (int64_t)num_sms(p->device) * 4);
-    k_hot_gather<<<g, 256, 0, s>>>(x, p->d_hot_cols, p->hot_S, p->d_xh);
-  }
   const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
   // The row classes write disjoint rows of y and only read x: the warp-row
   // kernel and the CTA/hub kernels run on two plan-owned streams concurrently
@@ -1012,18 +821,8 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   }
   if (conc && !early) fork();
   {
-    const int hot = lane_mode ? hot_mode(p) : 0;
-    if (SS) {
-      if (hot == 3) launch_rows<OT, true, 3>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-      else if (hot == 2) launch_rows<OT, true, 2>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-      else if (hot == 1) launch_rows<OT, true, 1>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-      else launch_rows<OT, true, 0>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-    } else {
-      if (hot == 3) launch_rows<OT, false, 3>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-      else if (hot == 2) launch_rows<OT, false, 2>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-      else if (hot == 1) launch_rows<OT, false, 1>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-      else launch_rows<OT, false, 0>(p, x, y, ss_in, s1, s2, lane_mode, dst);
-    }
+    if (SS) launch_rows<OT, true>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+    else launch_rows<OT, false>(p, x, y, ss_in, s1, s2, lane_mode, dst);
   }
   if (conc) {
     SPMV_CUDA(cudaEventRecord(p->ev_join[0], s1));
@@ -1121,10 +920,8 @@ void exec_streams(spmv_plan_s* p) { ensure_aux(p); }
 
 int exec_launches(const spmv_plan_s* p, bool ss) {
   const bool lane_mode = p->opts.variant != 1;
-  const int hot = lane_mode ? hot_mode(p) : 0;
-  const int longk = hot == 3 ? ((p->n_cta || p->n_chunks) ? 1 : 0) + (p->n_chunks ? 1 : 0)
-                             : (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0);
-  return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0) + (hot ? 1 : 0)
+  const int longk = (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0);
+  return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0)
                     : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
          longk + (ss ? 1 : 0);
 }
@@ -1137,8 +934,8 @@ void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double*
   if (nbcast) {
     if (nbcast < 0 || nbcast > 8) SPMV_FAIL(SPMV_EINVAL, "bcast: 1..8 destination buffers");
     if (!ss_out) SPMV_FAIL(SPMV_EINVAL, "bcast needs sumsq_out (exec_scaled)");
-    if (p->opts.variant == 1 || hot_mode(p))
-      SPMV_FAIL(SPMV_EUNSUPPORTED, "bcast: lane-mode kernels without the hot-column set only");
+    if (p->opts.variant == 1)
+      SPMV_FAIL(SPMV_EUNSUPPORTED, "bcast: lane-mode kernels only (variant 0)");
     for (int k = 0; k < nbcast; ++k) {
       if (!bcast[k]) SPMV_FAIL(SPMV_EINVAL, "bcast: NULL destination");
       dst.p[k] = bcast[k] + p->y_offset;

@@ -310,46 +310,6 @@ __global__ void k_colcnt(const int32_t* colA, const int32_t* perm, int64_t nnz, 
   GRID_STRIDE(k, nnz) atomicAdd(&cnt[perm[colA[k]]], 1u);
 }
 
-// hot-column set ("hot x in L1"): histogram of column counts
-// (exact below HOT_BINS - 1, the last bin collects the rest) and their sums
-__global__ void k_cnt_hist(const uint32_t* cnt, int64_t n, unsigned long long* nb,
-                           unsigned long long* sb) {
-  GRID_STRIDE(j, n) {
-    const uint32_t c = cnt[j];
-    const uint32_t b = c < (uint32_t)(HOT_BINS - 1) ? c : (uint32_t)(HOT_BINS - 1);
-    atomicAdd(&nb[b], 1ull);
-    atomicAdd(&sb[b], (unsigned long long)c);
-  }
-}
-
-__global__ void k_hot_flag(const uint32_t* cnt, int64_t n, uint32_t t, int32_t* f) {
-  GRID_STRIDE(j, n) f[j] = cnt[j] >= t ? 1 : 0;
-}
-
-// slot_of[j] = slot of hot column j (ascending column order) or -1;
-// hot_cols[slot] = j
-__global__ void k_hot_slots(const int32_t* f, const int64_t* pos, int64_t n, int32_t* slot_of,
-                            int32_t* hot_cols) {
-  GRID_STRIDE(j, n) {
-    if (f[j]) {
-      slot_of[j] = (int32_t)pos[j];
-      hot_cols[pos[j]] = (int32_t)j;
-    } else {
-      slot_of[j] = -1;
-    }
-  }
-}
-
-// col_hot[k] = ~slot (< 0) for a hot column, else the column itself
-__global__ void k_hot_encode(const int32_t* col, int64_t nnz, const int32_t* slot_of,
-                             int32_t* col_hot) {
-  GRID_STRIDE(k, nnz) {
-    const int32_t c = col[k];
-    const int32_t sl = slot_of[c];
-    col_hot[k] = sl >= 0 ? ~sl : c;
-  }
-}
-
 __global__ void k_first_cold(const uint32_t* cnt, int64_t n, int64_t nnz,
                              unsigned long long* H) {
   // smallest j with !(colcnt_B[j] * N > NZ): warp-level min first, one atomic per warp
@@ -661,57 +621,6 @@ int64_t class_list(const OT* rp, int64_t nrows, int64_t lo, int64_t hi, int32_t*
 
 }  // namespace
 
-// Hot-column set: the HOT_MAX most-referenced columns of B by
-// count (threshold t = smallest count with #{cnt >= t} <= HOT_MAX, t >= 2),
-// used by the lane-mode SpMV kernels through a 192 KB contiguous copy of x
-// that stays L1-resident.  On when opts.hot_x > 0, or (opts.hot_x == 0, auto)
-// when world == 1, variant 0, N >= 4 HOT_MAX and the set holds >= 15 % of the
-// non-zeros (power-law inputs).
-static void choose_hot(spmv_plan_s* p, const uint32_t* cnt, int64_t n, int64_t nnz,
-                       cudaStream_t s) {
-  p->hot_S = 0;
-  int64_t mode = p->opts.hot_x;
-  if (const char* e = getenv("SPMV_HOT")) mode = atoll(e);  // dev knob (A/B)
-  // auto (0) is off: measured on C3 (profiles r33) the L1-resident copy does
-  // not shorten the L1-wavefront-bound gathers; kept for A/B (mode > 0)
-  if (mode <= 0 || p->world != 1 || p->opts.variant == 1 || n == 0 || nnz == 0) return;
-  unsigned long long* nb = dalloc<unsigned long long>(2 * HOT_BINS);
-  SPMV_CUDA(cudaMemsetAsync(nb, 0, sizeof(unsigned long long) * 2 * HOT_BINS, s));
-  k_cnt_hist<<<grid_for(n), TPB, 0, s>>>(cnt, n, nb, nb + HOT_BINS);
-  SPMV_LAUNCH_CHECK();
-  std::vector<unsigned long long> h(2 * HOT_BINS);
-  SPMV_CUDA(cudaMemcpyAsync(h.data(), nb, sizeof(unsigned long long) * 2 * HOT_BINS,
-                            cudaMemcpyDeviceToHost, s));
-  SPMV_CUDA(cudaStreamSynchronize(s));
-  dfree(nb);
-  unsigned long long cols = 0, cover = 0;
-  int b = HOT_BINS - 1;
-  for (; b >= 2; --b) {
-    if (cols + h[b] > (unsigned long long)HOT_MAX) break;
-    cols += h[b];
-    cover += h[HOT_BINS + b];
-  }
-  const uint32_t t = (uint32_t)(b + 1);  // every column with count >= t is hot
-  if (cols == 0) return;
-  if (mode == 0 && cover * 100 < (unsigned long long)nnz * 15) return;
-  int32_t* f = dalloc<int32_t>(n);
-  int64_t* pos = dalloc<int64_t>(n + 1);
-  int64_t* tmp = dalloc<int64_t>(scan_temp_len(n));
-  k_hot_flag<<<grid_for(n), TPB, 0, s>>>(cnt, n, t, f);
-  exclusive_scan<int32_t>(f, n, pos, tmp, s);
-  p->d_slot_of = dalloc<int32_t>(n);
-  p->d_hot_cols = dalloc<int32_t>((int64_t)cols);
-  p->d_xh = dalloc<float>((int64_t)cols);
-  k_hot_slots<<<grid_for(n), TPB, 0, s>>>(f, pos, n, p->d_slot_of, p->d_hot_cols);
-  SPMV_LAUNCH_CHECK();
-  SPMV_CUDA(cudaStreamSynchronize(s));
-  dfree(f);
-  dfree(pos);
-  dfree(tmp);
-  p->hot_S = (int64_t)cols;
-  p->hot_nnz = (int64_t)cover;
-}
-
 template <typename AT, typename OT>
 static void build_typed(spmv_plan_s* p, const AT* rpA) {
   cudaStream_t s = p->s;
@@ -794,7 +703,6 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   SPMV_LAUNCH_CHECK();
   p->H = (int64_t)d2h_one(dH, s);
   dfree(dH);
-  choose_hot(p, cnt, n, nnz, s);
   dfree(cnt);
   dfree(rpB);
 
@@ -942,15 +850,6 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
       dfree(K1); dfree(K2); dfree(V1); dfree(V2);
     }
   }
-  if (p->hot_S && p->nnz_local) {
-    if (!p->d_col_hot) {
-      p->d_col_hot = dalloc<int32_t>(p->nnz_local + 8);
-      SPMV_CUDA(cudaMemsetAsync(p->d_col_hot + p->nnz_local, 0, 32, s));
-    }
-    k_hot_encode<<<grid_for(p->nnz_local), TPB, 0, s>>>(p->d_col, p->nnz_local, p->d_slot_of,
-                                                        p->d_col_hot);
-    SPMV_LAUNCH_CHECK();
-  }
   if (padded(p) && p->nnz_local) {
     int64_t* d_part = dalloc<int64_t>(p->world + 1);
     SPMV_CUDA(cudaMemcpyAsync(d_part, p->part.data(), 8 * (p->world + 1), cudaMemcpyHostToDevice, s));
@@ -1097,7 +996,6 @@ void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStr
 
 void plan_free(spmv_plan_s* p) {
   coo_free(p);
-  dfree(p->d_slot_of); dfree(p->d_hot_cols); dfree(p->d_xh); dfree(p->d_col_hot);
   dfree(p->s1); dfree(p->s2); dfree(p->s3); dfree(p->big); dfree(p->boff);
   dfree(p->longrows);
   dfree(p->d_perm); dfree(p->d_inv);

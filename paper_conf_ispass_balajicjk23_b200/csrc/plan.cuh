@@ -60,13 +60,6 @@ struct spmv_plan_s {
   double* d_chunk_part = nullptr;  // [n_chunks]
   double* d_chunk_part4 = nullptr; // [4 n_chunks] spmv_exec_spmm4 (allocated on first use)
 
-  // hot-column set: the hot_S most-referenced columns; col_hot
-  // is col with hot columns coded ~slot; xh[slot] = x[hot_cols[slot]] per exec
-  int64_t hot_S = 0, hot_nnz = 0;
-  int32_t* d_slot_of = nullptr;    // [n] slot or -1
-  int32_t* d_hot_cols = nullptr;   // [hot_S]
-  float* d_xh = nullptr;           // [hot_S]
-  int32_t* d_col_hot = nullptr;    // [nnz_local + 8]
 
   // COO form of B (spmv_exec_coo; built on first use): row index per entry and
   // per-tile pieces of rows that cross a 2048-entry tile boundary

@@ -222,7 +222,7 @@ Sym symmetrize(int64_t n, const int64_t* rp, const int32_t* col) {
   return S;
 }
 
-struct Edge {
+struct __attribute__((packed)) Edge {  // 12 bytes: aggregated lists dominate host memory
   int32_t v;
   int64_t w;
 };
@@ -390,16 +390,35 @@ struct HashAcc {  // per-thread (root -> summed weight) map, open addressing
   std::vector<int64_t> val;
   std::vector<uint32_t> used;
   uint32_t mask = 0;
-  void prepare(size_t expect) {
+  static size_t cap_for(size_t expect) {
     size_t cap = 64;
     while (cap < 2 * expect) cap <<= 1;
-    if (cap > key.size()) {
-      key.assign(cap, -1);
-      val.assign(cap, 0);
-      mask = (uint32_t)(cap - 1);
+    return cap;
+  }
+  void prepare(size_t expect) {  // capacity for `expect` keys (grows further on demand)
+    const size_t cap = cap_for(expect);
+    if (cap > key.size()) rehash(cap);
+  }
+  void rehash(size_t cap) {
+    std::vector<int32_t> k2(cap, -1);
+    std::vector<int64_t> v2(cap, 0);
+    std::vector<uint32_t> u2;
+    u2.reserve(used.size());
+    const uint32_t m2 = (uint32_t)(cap - 1);
+    for (uint32_t h : used) {
+      uint32_t g = ((uint32_t)key[h] * 2654435761u) & m2;
+      while (k2[g] != -1) g = (g + 1) & m2;
+      k2[g] = key[h];
+      v2[g] = val[h];
+      u2.push_back(g);
     }
+    key.swap(k2);
+    val.swap(v2);
+    used.swap(u2);
+    mask = m2;
   }
   inline void add(int32_t r, int64_t w) {
+    if (2 * (used.size() + 1) > key.size()) rehash(cap_for(used.size() + 1) * 2);
     uint32_t h = ((uint32_t)r * 2654435761u) & mask;
     while (key[h] != -1 && key[h] != r) h = (h + 1) & mask;
     if (key[h] == -1) {
@@ -414,6 +433,12 @@ struct HashAcc {  // per-thread (root -> summed weight) map, open addressing
       val[h] = 0;
     }
     used.clear();
+  }
+  void release() {  // give a huge table back after a hub
+    std::vector<int32_t>().swap(key);
+    std::vector<int64_t>().swap(val);
+    std::vector<uint32_t>().swap(used);
+    mask = 0;
   }
 };
 
@@ -469,7 +494,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
   // u's aggregated list: its S-row and its children's lists, neighbours
   // mapped to their current roots, weights summed per root, u dropped
   auto aggregate = [&](int32_t u, HashAcc& H, std::vector<Edge>& tl) {
-    H.prepare(expected(u));
+    H.prepare(std::min<size_t>(expected(u), (size_t)1 << 20));
     for (int64_t k = S.ptr[u]; k < S.ptr[u + 1]; ++k) {
       const int32_t r = find(S.idx[k]);
       if (r != u) H.add(r, S.w[k]);
@@ -482,6 +507,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
     tl.clear();
     for (uint32_t h : H.used) tl.push_back({H.key[h], H.val[h]});
     H.clear();
+    if (H.key.size() > ((size_t)1 << 22)) H.release();
   };
   // the same list with every thread (the tail phase, where the hubs with the
   // largest aggregated lists come last and nothing else runs): chunks of the
@@ -501,7 +527,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
     {
       const int t = omp_get_thread_num();
       HashAcc& H = Hs[t];
-      H.prepare(ex);
+      H.prepare(std::min<size_t>(ex / T + 1024, (size_t)1 << 24));
 #pragma omp for schedule(dynamic, 1)
       for (int64_t q = 0; q < (int64_t)segs.size(); ++q) {
         const Seg& g = segs[q];
@@ -523,14 +549,15 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
 #pragma omp barrier
       size_t m = 0;
       for (int t2 = 0; t2 < T; ++t2) m += parts[(size_t)t2 * T + t].size();
-      H.prepare(m);
+      H.prepare(std::min<size_t>(m, (size_t)1 << 24));
       for (int t2 = 0; t2 < T; ++t2) {
         for (const Edge& e : parts[(size_t)t2 * T + t]) H.add(e.v, e.w);
-        parts[(size_t)t2 * T + t].clear();
+        std::vector<Edge>().swap(parts[(size_t)t2 * T + t]);
       }
       outs[t].clear();
       for (uint32_t h : H.used) outs[t].push_back({H.key[h], H.val[h]});
       H.clear();
+      if (H.key.size() > ((size_t)1 << 24)) H.release();
     }
     tl.clear();
     for (int t = 0; t < T; ++t) tl.insert(tl.end(), outs[t].begin(), outs[t].end());
