@@ -277,7 +277,7 @@ def run_gpu(args):
         y = torch.empty(max(info["row_end"] - info["row_begin"], 1), dtype=torch.float32, device=dev)
         if iterate_mode:
             xs = xB.clone()
-            launches_per_step = info["exec_launches"] + 1   # + the fixed-order norm
+            launches_per_step = info["exec_launches"] + 2   # + the fixed-order norm (2 kernels)
 
             def warm(w):
                 P.iterate(xs, w)

@@ -4,7 +4,17 @@
 #include <cstring>
 #include <string>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "plan.cuh"
+
+// NVTX range over one ABI call (header-only NVTX v3: a no-op unless a tool
+// such as nsys / ncu attaches), so plan / permute / exec / iterate show up as
+// named ranges on a timeline
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 namespace spmv {
 static thread_local std::string g_err;
@@ -55,6 +65,7 @@ const char* spmv_version(void) { return "spmv-b200 0.1 (sm_100a)"; }
 
 spmv_status spmv_plan(const spmv_csr_t* A, const int32_t* perm, const spmv_opts_t* opts,
                       spmv_plan_t* out) {
+  NvtxRange nvtx_("spmv_plan");
   spmv_plan_s* p = nullptr;
   API_BEGIN
   if (!A || !out) SPMV_FAIL(SPMV_EINVAL, "spmv_plan: NULL argument");
@@ -107,6 +118,7 @@ spmv_status spmv_plan(const spmv_csr_t* A, const int32_t* perm, const spmv_opts_
 }
 
 spmv_status spmv_permute(spmv_plan_t p, void* stream) {
+  NvtxRange nvtx_("spmv_permute");
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_permute: NULL plan");
   use_device(p);
@@ -116,6 +128,7 @@ spmv_status spmv_permute(spmv_plan_t p, void* stream) {
 
 spmv_status spmv_permute_vec(spmv_plan_t p, const float* in, float* out, int inverse,
                              void* stream) {
+  NvtxRange nvtx_("spmv_permute_vec");
   API_BEGIN
   if (!p || (p->n && (!in || !out))) SPMV_FAIL(SPMV_EINVAL, "spmv_permute_vec: NULL argument");
   if (p->n && in == out) SPMV_FAIL(SPMV_EINVAL, "spmv_permute_vec: in and out alias");
@@ -135,6 +148,7 @@ spmv_status spmv_pad_vec(spmv_plan_t p, const float* in, float* out, int to_padd
 }
 
 spmv_status spmv_exec(spmv_plan_t p, const float* x_B, float* y_B, void* stream) {
+  NvtxRange nvtx_("spmv_exec");
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec: NULL plan");
   if (p->nrows && (!x_B || !y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec: NULL vector");
@@ -145,6 +159,7 @@ spmv_status spmv_exec(spmv_plan_t p, const float* x_B, float* y_B, void* stream)
 
 spmv_status spmv_rabbitpp_gpu(const spmv_csr_t* A, const int32_t* perm_rabbit,
                               const int32_t* comm, int32_t* perm_out, void* stream) {
+  NvtxRange nvtx_("spmv_rabbitpp_gpu");
   API_BEGIN
   if (!A || (A->n && (!perm_rabbit || !comm || !perm_out)))
     SPMV_FAIL(SPMV_EINVAL, "spmv_rabbitpp_gpu: NULL argument");
@@ -157,6 +172,7 @@ spmv_status spmv_rabbitpp_gpu(const spmv_csr_t* A, const int32_t* perm_rabbit,
 }
 
 spmv_status spmv_exec_spmm4(spmv_plan_t p, const float* X_B, float* Y_B, void* stream) {
+  NvtxRange nvtx_("spmv_exec_spmm4");
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_spmm4: NULL plan");
   if (p->nrows && (!X_B || !Y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_spmm4: NULL matrix");
@@ -166,6 +182,7 @@ spmv_status spmv_exec_spmm4(spmv_plan_t p, const float* X_B, float* Y_B, void* s
 }
 
 spmv_status spmv_exec_coo(spmv_plan_t p, const float* x_B, float* y_B, void* stream) {
+  NvtxRange nvtx_("spmv_exec_coo");
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_coo: NULL plan");
   if (p->nrows && (!x_B || !y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_coo: NULL vector");
@@ -177,6 +194,7 @@ spmv_status spmv_exec_coo(spmv_plan_t p, const float* x_B, float* y_B, void* str
 spmv_status spmv_exec_scaled_bcast(spmv_plan_t p, const float* x_B, float* const* x_next,
                                    int n_next, const double* sumsq_in, double* sumsq_out,
                                    void* stream) {
+  NvtxRange nvtx_("spmv_exec_scaled_bcast");
   API_BEGIN
   if (!p || !x_next) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled_bcast: NULL argument");
   if (p->nrows && !x_B) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled_bcast: NULL vector");
@@ -233,6 +251,7 @@ spmv_status spmv_ipc_close(void* dev_ptr) {
 
 spmv_status spmv_exec_scaled(spmv_plan_t p, const float* x_B, float* y_B,
                              const double* sumsq_in, double* sumsq_out, void* stream) {
+  NvtxRange nvtx_("spmv_exec_scaled");
   API_BEGIN
   if (!p) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled: NULL plan");
   if (p->nrows && (!x_B || !y_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_exec_scaled: NULL vector");
@@ -243,6 +262,7 @@ spmv_status spmv_exec_scaled(spmv_plan_t p, const float* x_B, float* y_B,
 
 spmv_status spmv_iterate(spmv_plan_t p, float* x_B, int iters, double* lambda_out,
                          void* stream) {
+  NvtxRange nvtx_("spmv_iterate");
   API_BEGIN
   if (!p || (p->n && !x_B)) SPMV_FAIL(SPMV_EINVAL, "spmv_iterate: NULL argument");
   use_device(p);

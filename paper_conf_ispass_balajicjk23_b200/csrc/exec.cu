@@ -15,7 +15,8 @@
 //   k_cta_rows   one CTA per row, 2048 < L <= 16384 (256 strided partials + tree).
 //   k_hub_chunk  one CTA per 16384-entry chunk of a hub row (merge-path split);
 //   k_hub_fix    fp64 combine of the chunk sums in chunk order.
-//   k_ss_final   fixed-order fp64 sum of per-tile / per-row y^2 partials
+//   k_ss_part / k_ss_final  fixed-order fp64 sum of per-block / per-row y^2
+//                partials (fixed segments, then the segment sums in order)
 //                (power-iteration norm; deterministic).
 // No tensor cores: SpMV is not a dense contraction (AI <= 0.25 flop/B).
 #include <atomic>
@@ -515,25 +516,62 @@ __global__ void k_hub_fix(const int32_t* __restrict__ hub_rows, const int32_t* _
   fence_bcast<SS>(dst);
 }
 
-__global__ void __launch_bounds__(1024)
-    k_ss_final(const double* __restrict__ a, int64_t na, const double* __restrict__ b, int64_t nb,
-               const double* __restrict__ c, int64_t nc, const double* __restrict__ d,
-               int64_t nd, double* __restrict__ out) {
-  __shared__ double wss[32];
-  double acc = 0.0;
-  for (int64_t i = threadIdx.x; i < na; i += 1024) acc += a[i];
-  for (int64_t i = threadIdx.x; i < nb; i += 1024) acc += b[i];
-  for (int64_t i = threadIdx.x; i < nc; i += 1024) acc += c[i];
-  for (int64_t i = threadIdx.x; i < nd; i += 1024) acc += d[i];
+// Fixed-order fp64 sum of the y^2 partials (power-iteration norm).  The
+// partial arrays a | b | c | d form one virtual sequence cut into segments of
+// SS_SEG entries; CTA s sums segment s (strided per thread, then a fixed
+// tree), k_ss_final sums the segment sums in order.  The association depends
+// only on the plan's row classes, never on the grid: bitwise repeatable.
+constexpr int64_t SS_SEG = 16384;
+
+__device__ __forceinline__ double ss_at(int64_t v, const double* a, int64_t na, const double* b,
+                                        int64_t nb, const double* c, int64_t nc, const double* d) {
+  if (v < na) return a[v];
+  v -= na;
+  if (v < nb) return b[v];
+  v -= nb;
+  if (v < nc) return c[v];
+  return d[v - nc];
+}
+
+__device__ __forceinline__ double block_sum_1024(double acc, double* wss) {
   acc = warp_sum_d(acc);
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   if (lane == 0) wss[w] = acc;
   __syncthreads();
-  if (threadIdx.x == 0) {
-    double s = 0.0;
+  double s = 0.0;
+  if (threadIdx.x == 0)
     for (int i = 0; i < 32; ++i) s += wss[i];
-    *out = s;
-  }
+  return s;  // valid in thread 0
+}
+
+__global__ void __launch_bounds__(1024)
+    k_ss_part(const double* __restrict__ a, int64_t na, const double* __restrict__ b, int64_t nb,
+              const double* __restrict__ c, int64_t nc, const double* __restrict__ d, int64_t nd,
+              double* __restrict__ part) {
+  __shared__ double wss[32];
+  const int64_t tot = na + nb + nc + nd;
+  const int64_t v0 = (int64_t)blockIdx.x * SS_SEG, v1 = min(tot, v0 + SS_SEG);
+  double acc = 0.0;
+  for (int64_t v = v0 + threadIdx.x; v < v1; v += 1024) acc += ss_at(v, a, na, b, nb, c, nc, d);
+  const double sblk = block_sum_1024(acc, wss);
+  if (threadIdx.x == 0) part[blockIdx.x] = sblk;
+}
+
+__global__ void __launch_bounds__(1024)
+    k_ss_final(const double* __restrict__ part, int64_t np, double* __restrict__ out) {
+  __shared__ double wss[32];
+  double acc = 0.0;
+  for (int64_t i = threadIdx.x; i < np; i += 1024) acc += part[i];
+  const double s = block_sum_1024(acc, wss);
+  if (threadIdx.x == 0) *out = s;
+}
+
+void ss_reduce(spmv_plan_s* p, const double* a, int64_t na, const double* b, int64_t nb,
+               const double* c, int64_t nc, const double* d, int64_t nd, double* out,
+               cudaStream_t s) {
+  const int64_t np = std::max<int64_t>(1, (na + nb + nc + nd + SS_SEG - 1) / SS_SEG);
+  k_ss_part<<<(unsigned)np, 1024, 0, s>>>(a, na, b, nb, c, nc, d, nd, p->d_ss_part);
+  k_ss_final<<<1, 1024, 0, s>>>(p->d_ss_part, np, out);
 }
 
 int g_num_sms = 0;
@@ -832,12 +870,11 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   }
   if (SS) {
     if (lane_mode)
-      k_ss_final<<<1, 1024, 0, s>>>(p->d_blk_ss, (p->nrows + LN_THREADS - 1) / LN_THREADS,
-                                    p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta, p->d_hub_ss,
-                                    p->n_hub, ss_out);
+      ss_reduce(p, p->d_blk_ss, (p->nrows + LN_THREADS - 1) / LN_THREADS, p->d_mid_ss, p->n_mid,
+                p->d_cta_ss, p->n_cta, p->d_hub_ss, p->n_hub, ss_out, s);
     else
-      k_ss_final<<<1, 1024, 0, s>>>(p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss,
-                                    p->n_cta, p->d_hub_ss, p->n_hub, ss_out);
+      ss_reduce(p, p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss, p->n_cta,
+                p->d_hub_ss, p->n_hub, ss_out, s);
   }
   SPMV_LAUNCH_CHECK();
 }
@@ -923,7 +960,7 @@ int exec_launches(const spmv_plan_s* p, bool ss) {
   const int longk = (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0);
   return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0)
                     : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
-         longk + (ss ? 1 : 0);
+         longk + (ss ? 2 : 0);
 }
 
 void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,

@@ -329,7 +329,92 @@ __global__ void k_first_cold(const uint32_t* cnt, int64_t n, int64_t nnz,
 }
 
 // ------------------------------------------------------------- P A P^T data
-// warp per row for rows with L <= STREAM_MAX
+// Key (col_B << 32 | position in row) is unique inside a row, so any correct
+// sort by key is the stable sort by col_B (duplicates keep A's order).
+__device__ __forceinline__ uint64_t mkkey(int32_t c, int64_t rel) {
+  return ((uint64_t)(uint32_t)c << 32) | (uint64_t)(uint32_t)rel;
+}
+
+// bitonic sort of one key (+ value) per lane over groups of W lanes (W = 16
+// or 32; xor partners stay inside the group)
+template <int W>
+__device__ __forceinline__ void lane_bitonic(uint64_t& key, float& v, int gl) {
+#pragma unroll
+  for (int k = 2; k <= W; k <<= 1) {
+#pragma unroll
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      const uint64_t ok = __shfl_xor_sync(0xffffffffu, key, j);
+      const float ov = __shfl_xor_sync(0xffffffffu, v, j);
+      const bool take_min = ((gl & j) == 0) == ((gl & k) == 0);
+      if (take_min == (ok < key)) {
+        key = ok;
+        v = ov;
+      }
+    }
+  }
+}
+
+// Rows with L <= 32 relabelled AND sorted in registers: one read of A's row,
+// one gather of perm per entry, one write of B's row.  A warp
+// takes rows 2q and 2q+1: a half-warp each when both have L <= 16 (width-16
+// sort network), else the whole warp on each in turn (width 32).  Longer rows
+// are left to k_relabel_warp / k_relabel_cta and the shared-memory sorts.
+template <typename AT, typename OT>
+__global__ void __launch_bounds__(256)
+    k_relabel_sort_short(const AT* __restrict__ rpA, const int32_t* __restrict__ colA,
+                         const float* __restrict__ valA, const int32_t* __restrict__ perm,
+                         const int32_t* __restrict__ inv, int64_t rb, int64_t nrows,
+                         const OT* __restrict__ rpB, int32_t* __restrict__ colB,
+                         float* __restrict__ valB) {
+  const int lane = threadIdx.x & 31, half = lane >> 4, hl = lane & 15;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; 2 * q < nrows;
+       q += nw) {
+    const int64_t r = 2 * q + half;
+    int64_t d = 0, L = 0;
+    if (r < nrows) {
+      d = (int64_t)rpB[r];
+      L = (int64_t)rpB[r + 1] - d;
+    }
+    const int64_t Lo = __shfl_xor_sync(0xffffffffu, L, 16);
+    if (L <= 16 && Lo <= 16) {
+      uint64_t key = ~0ull;
+      float v = 0.f;
+      if (hl < L) {
+        const int64_t a = (int64_t)rpA[inv[rb + r]];
+        key = mkkey(perm[colA[a + hl]], hl);
+        v = valA[a + hl];
+      }
+      lane_bitonic<16>(key, v, hl);
+      if (hl < L) {
+        colB[d + hl] = (int32_t)(key >> 32);
+        valB[d + hl] = v;
+      }
+    } else {
+#pragma unroll 1
+      for (int h = 0; h < 2; ++h) {
+        const int64_t rr = 2 * q + h;
+        const int64_t Lh = __shfl_sync(0xffffffffu, L, 16 * h);
+        const int64_t dh = __shfl_sync(0xffffffffu, d, 16 * h);
+        if (Lh > 32 || rr >= nrows) continue;  // (warp-uniform)
+        uint64_t key = ~0ull;
+        float v = 0.f;
+        if (lane < Lh) {
+          const int64_t a = (int64_t)rpA[inv[rb + rr]];
+          key = mkkey(perm[colA[a + lane]], lane);
+          v = valA[a + lane];
+        }
+        lane_bitonic<32>(key, v, lane);
+        if (lane < Lh) {
+          colB[dh + lane] = (int32_t)(key >> 32);
+          valB[dh + lane] = v;
+        }
+      }
+    }
+  }
+}
+
+// warp per row for rows with 32 < L <= WARP_MAX (relabel only; sorted after)
 template <typename AT, typename OT>
 __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* valA,
                                const int32_t* perm, const int32_t* inv, int64_t rb,
@@ -339,7 +424,7 @@ __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* 
   int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t r = w; r < nrows; r += nw) {
     int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d;
-    if (L > WARP_MAX) continue;  // longer rows: k_relabel_cta
+    if (L <= SHORT_MAX || L > WARP_MAX) continue;  // k_relabel_sort_short / k_relabel_cta
     int64_t i = inv[rb + r];
     int64_t a = (int64_t)rpA[i];
     for (int64_t k = lane; k < L; k += 32) {
@@ -368,43 +453,6 @@ __global__ void k_relabel_cta(const AT* rpA, const int32_t* colA, const float* v
 }
 
 // ----------------------------------------------------------------- row sort
-// Key (col_B << 32 | position in row) is unique inside a row, so any correct
-// sort by key is the stable sort by col_B (duplicates keep A's order).
-__device__ __forceinline__ uint64_t mkkey(int32_t c, int64_t rel) {
-  return ((uint64_t)(uint32_t)c << 32) | (uint64_t)(uint32_t)rel;
-}
-
-template <typename OT>
-__global__ void k_sort_warp(const OT* rp, int64_t nrows, int32_t* col, float* val) {
-  const int lane = threadIdx.x & 31;
-  int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t r = w; r < nrows; r += nw) {
-    int64_t d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d;
-    if (L < 2 || L > 32) continue;
-    uint64_t key = lane < L ? mkkey(col[d + lane], lane) : ~0ull;
-    float v = lane < L ? val[d + lane] : 0.f;
-#pragma unroll
-    for (int k = 2; k <= 32; k <<= 1) {
-#pragma unroll
-      for (int j = k >> 1; j > 0; j >>= 1) {
-        uint64_t ok = __shfl_xor_sync(0xffffffffu, key, j);
-        float ov = __shfl_xor_sync(0xffffffffu, v, j);
-        bool take_min = ((lane & j) == 0) == ((lane & k) == 0);
-        bool other_smaller = ok < key;
-        if (take_min == other_smaller) {
-          key = ok;
-          v = ov;
-        }
-      }
-    }
-    if (lane < L) {
-      col[d + lane] = (int32_t)(key >> 32);
-      val[d + lane] = v;
-    }
-  }
-}
-
 // CTA bitonic sort of one row of length L <= P held in shared memory.
 template <int P>
 __device__ void smem_bitonic(uint64_t* keys, float* vals) {
@@ -798,6 +846,11 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   p->d_cta_ss = dalloc<double>(p->n_cta);
   p->d_hub_ss = dalloc<double>(p->n_hub);
   p->d_ss = dalloc<double>(4);
+  {  // segment sums of the norm reduction (exec.cu ss_reduce), either row scheme
+    const int64_t lane_parts = (nr + 63) / 64 + p->n_mid + p->n_cta + p->n_hub;
+    const int64_t tile_parts = p->K + p->n_warp + p->n_cta + p->n_hub;
+    p->d_ss_part = dalloc<double>(std::max(lane_parts, tile_parts) / 16384 + 2);
+  }
   SPMV_CUDA(cudaStreamSynchronize(s));
 }
 
@@ -807,13 +860,15 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
   spmv_plan_s* ps = p;
   const int64_t nr = p->nrows;
   if (nr) {
-    k_relabel_warp<AT, OT><<<grid_for(nr * 32), TPB, 0, s>>>(
+    k_relabel_sort_short<AT, OT><<<grid_for((nr + 1) / 2 * 32), 256, 0, s>>>(
         rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, nr, rp, p->d_col, p->d_val);
+    if (ps->n1 + ps->n2 + ps->n3 + ps->nbig)  // rows with L > 32 exist
+      k_relabel_warp<AT, OT><<<grid_for(nr * 32), TPB, 0, s>>>(
+          rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, nr, rp, p->d_col, p->d_val);
     if (ps->nlong)
       k_relabel_cta<AT, OT><<<(unsigned)std::min<int64_t>(ps->nlong, 148 * 8), 512, 0, s>>>(
           rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, ps->longrows, ps->nlong,
           rp, p->d_col, p->d_val);
-    k_sort_warp<OT><<<grid_for(nr * 32), TPB, 0, s>>>(rp, nr, p->d_col, p->d_val);
     SPMV_LAUNCH_CHECK();
     if (ps->n1) {
       k_sort_cta<128, OT><<<(unsigned)std::min<int64_t>(ps->n1, 148 * 64), 64, 128 * 12, s>>>(
@@ -919,6 +974,27 @@ void rabbitpp_gpu(const spmv_csr_t* A, const int32_t* perm_rabbit, const int32_t
                   int32_t* perm_out, cudaStream_t s) {
   const int64_t n = A->n, nnz = A->nnz;
   if (n == 0) return;
+  {  // the header's EINVAL promise: CSR, column range, comm range, perm bijection
+    int* fl = dalloc<int>(6);  // [0] row_ptr, [1] col, [2] perm, [4] comm
+    int32_t* inv = dalloc<int32_t>(n);
+    SPMV_CUDA(cudaMemsetAsync(fl, 0, 6 * sizeof(int), s));
+    if (A->row_ptr64) k_validate_rp<int64_t><<<grid_for(n), TPB, 0, s>>>(A->row_ptr64, n, nnz, fl);
+    else k_validate_rp<int32_t><<<grid_for(n), TPB, 0, s>>>(A->row_ptr32, n, nnz, fl);
+    if (nnz) k_validate_col<<<grid_for(nnz), TPB, 0, s>>>(A->col_idx, nnz, n, fl);
+    k_validate_col<<<grid_for(n), TPB, 0, s>>>(comm, n, n, fl + 3);  // comm[v] in [0, n) -> fl[4]
+    k_fill_i32<<<grid_for(n), TPB, 0, s>>>(inv, n, -1);
+    k_inverse<<<grid_for(n), TPB, 0, s>>>(perm_rabbit, n, inv, fl);
+    SPMV_LAUNCH_CHECK();
+    int h[6];
+    SPMV_CUDA(cudaMemcpyAsync(h, fl, sizeof(h), cudaMemcpyDeviceToHost, s));
+    SPMV_CUDA(cudaStreamSynchronize(s));
+    dfree(fl);
+    dfree(inv);
+    if (h[0]) SPMV_FAIL(SPMV_EINVAL, "spmv_rabbitpp_gpu: row_ptr is not a valid CSR row pointer");
+    if (h[1]) SPMV_FAIL(SPMV_EINVAL, "spmv_rabbitpp_gpu: column index out of range [0, n)");
+    if (h[2]) SPMV_FAIL(SPMV_EPERM, "spmv_rabbitpp_gpu: perm_rabbit is not a bijection on [0, n)");
+    if (h[4]) SPMV_FAIL(SPMV_EINVAL, "spmv_rabbitpp_gpu: community id out of range [0, n)");
+  }
   unsigned long long* cnt = dalloc<unsigned long long>(n);
   uint8_t* ins = dalloc<uint8_t>(n);
   int32_t* flags = dalloc<int32_t>(3 * n);
@@ -1005,7 +1081,7 @@ void plan_free(spmv_plan_s* p) {
   dfree(p->d_chunk_part4);
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
   dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_blk_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
-  dfree(p->d_ss); dfree(p->d_u);
+  dfree(p->d_ss); dfree(p->d_u); dfree(p->d_ss_part);
   for (int i = 0; i < 2; ++i) {
     if (p->aux[i]) { cudaStreamDestroy(p->aux[i]); p->aux[i] = nullptr; }
     if (p->ev_join[i]) { cudaEventDestroy(p->ev_join[i]); p->ev_join[i] = nullptr; }

@@ -76,6 +76,7 @@ struct spmv_plan_s {
   double* d_cta_ss = nullptr;      // [n_cta]
   double* d_hub_ss = nullptr;      // [n_hub]
   double* d_ss = nullptr;          // [4] iterate scalars
+  double* d_ss_part = nullptr;     // segment sums of the norm reduction
   float* d_u = nullptr;            // iterate ping-pong [x_len]
 
   // permute-phase sort buckets (ascending local rows)

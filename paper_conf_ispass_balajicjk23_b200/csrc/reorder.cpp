@@ -31,6 +31,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/spmv.h"
 
 namespace spmv {
@@ -254,25 +256,52 @@ std::vector<int64_t> degree_order(const std::vector<int64_t>& deg) {
 
 // pre-order DFS of the dendrogram (reading c10): roots in `top` order,
 // children in merge order
+// The trees are independent: their sizes (one counting DFS each, in
+// parallel) give every root its first ID by a prefix sum, then each tree is
+// numbered in parallel -- the same IDs as one sequential pass.
 void dendrogram_ids(const std::vector<int32_t>& top, const std::vector<int32_t>& first_child,
                     const std::vector<int32_t>& next_sib, Rabbit& R, int64_t n) {
   R.perm.assign(n, -1);
   R.comm.assign(n, -1);
-  int32_t nxt = 0;
-  std::vector<int32_t> st;
-  for (int32_t r : top) {
-    st.push_back(r);
-    while (!st.empty()) {
-      int32_t x = st.back();
-      st.pop_back();
-      R.perm[x] = nxt++;
-      R.comm[x] = r;
-      size_t mark = st.size();
-      for (int32_t c = first_child[x]; c != -1; c = next_sib[c]) st.push_back(c);
-      std::reverse(st.begin() + mark, st.end());
+  const int64_t nt = (int64_t)top.size();
+  std::vector<int64_t> size(nt + 1, 0);
+#pragma omp parallel
+  {
+    std::vector<int32_t> st;
+#pragma omp for schedule(dynamic, 1024)
+    for (int64_t t = 0; t < nt; ++t) {
+      int64_t m = 0;
+      st.push_back(top[t]);
+      while (!st.empty()) {
+        const int32_t x = st.back();
+        st.pop_back();
+        ++m;
+        for (int32_t c = first_child[x]; c != -1; c = next_sib[c]) st.push_back(c);
+      }
+      size[t] = m;
     }
   }
-  R.n_top = (int64_t)top.size();
+  scan_inplace(size);
+#pragma omp parallel
+  {
+    std::vector<int32_t> st;
+#pragma omp for schedule(dynamic, 1024)
+    for (int64_t t = 0; t < nt; ++t) {
+      const int32_t r = top[t];
+      int32_t nxt = (int32_t)size[t];
+      st.push_back(r);
+      while (!st.empty()) {
+        const int32_t x = st.back();
+        st.pop_back();
+        R.perm[x] = nxt++;
+        R.comm[x] = r;
+        const size_t mark = st.size();
+        for (int32_t c = first_child[x]; c != -1; c = next_sib[c]) st.push_back(c);
+        std::reverse(st.begin() + mark, st.end());
+      }
+    }
+  }
+  R.n_top = nt;
 }
 
 Rabbit rabbit_detect(const Sym& S, bool want_log) {
@@ -483,7 +512,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
   std::vector<std::vector<int32_t>> tops(T), deferred(T);
   std::vector<std::vector<MergeRec>> logs(T);
   std::vector<int64_t> merges(T, 0), retries(T, 0);
-  std::vector<HashAcc> Hs(T);
+  std::vector<HashAcc> Hs(T), Hsmall(T);  // small: vertices with short lists (cache-resident)
   phase("par:setup", tp);
 
   auto expected = [&](int32_t u) {
@@ -587,7 +616,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
     };
     for (int attempt = 0;; ++attempt) {
       if (mode == 2) aggregate_all(u, tl);
-      else aggregate(u, H, tl);
+      else aggregate(u, expected(u) <= 1024 ? Hsmall[tid] : H, tl);
       int32_t best = -1;
       __int128 bestdq = 0;
       int64_t bestw = 0;
@@ -768,6 +797,10 @@ uint64_t input_key(int64_t n, int64_t nnz, const int64_t* rp, const int32_t* col
 extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, const int32_t* col,
                                     int method, uint64_t seed, int32_t* perm_out,
                                     spmv_reorder_stats_t* st) {
+  nvtxRangePushA("spmv_reorder");
+  struct Pop {
+    ~Pop() { nvtxRangePop(); }
+  } pop_;
   try {
     auto t0 = std::chrono::steady_clock::now();
     const bool par = (method & SPMV_REORDER_PARALLEL) != 0;
@@ -945,6 +978,7 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
         int64_t ni = 0;
         for (int64_t v = 0; v < n; ++v) ni += ins[v];
         S0.insular_frac = n ? (double)ni / (double)n : 0.0;
+        S0.n_insular = ni;
       }
       if (method == SPMV_ORDER_RABBIT) {
         std::memcpy(perm_out, R.perm.data(), sizeof(int32_t) * n);

@@ -79,7 +79,8 @@ class _Stats(ctypes.Structure):
                 ("n_hubs", ctypes.c_int64), ("n_group0", ctypes.c_int64),
                 ("skew", ctypes.c_double), ("seconds", ctypes.c_double),
                 ("seconds_detect", ctypes.c_double), ("n_deferred", ctypes.c_int64),
-                ("parallel", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("parallel", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("n_insular", ctypes.c_int64)]
 
 
 _lib = None
@@ -380,6 +381,7 @@ class ReorderStats:
     n_deferred: int = 0
     parallel: int = 0
     reserved: int = 0
+    n_insular: int = 0
 
 
 PARALLEL, LOG = 0x100, 0x200

@@ -77,6 +77,7 @@ def test_reorder_rabbitpp_bitexact(name, A, variant, method):
     assert st.n_hubs == int(rabbit.hub_flags(A.n, A.row_ptr, A.col).sum())
     ins = rabbit.insular_flags(A.n, A.row_ptr, A.col, r.comm)
     assert math.isclose(st.insular_frac, ins.mean())
+    assert st.n_insular == int(ins.sum())
 
 
 def test_reorder_rmat16_bitexact():

@@ -270,7 +270,7 @@ def test_iterate_matches_oracle_recurrence(dev):
     P.close()
 
 
-def _full_size_check(dev, cfg, ordering, nsample=2000):
+def _full_size_check(dev, cfg, ordering, nsample=2000, parallel=False):
     """BASELINE config `cfg` at full size, in the launch configuration bench.py
     times: sampled rows' integer structure against the oracle's own
     relabelling, sampled y against the exact fsum oracle, every row against
@@ -281,7 +281,7 @@ def _full_size_check(dev, cfg, ordering, nsample=2000):
     if ordering == "original":
         perm = np.arange(A.n, dtype=np.int32)
     else:
-        perm, _ = spmv.reorder(A.row_ptr, A.col, ordering)
+        perm, _ = spmv.reorder(A.row_ptr, A.col, ordering, parallel=parallel)
     rp_dtype = torch.int32 if A.nnz < 2**31 else torch.int64
     P = mk_plan(A, perm, dev, rp_dtype=rp_dtype)
     xB = P.permute_vec(torch.from_numpy(w.x).to(dev))
@@ -411,3 +411,40 @@ def test_rabbitpp_gpu_postpass_bitexact(dev, name, make):
                               torch.from_numpy(A.col).to(dev), torch.from_numpy(pr).to(dev),
                               torch.from_numpy(comm).to(dev))
     assert np.array_equal(out32.cpu().numpy(), ppp)
+
+
+def test_rabbitpp_gpu_rejects_malformed_input(dev):
+    """spmv_rabbitpp_gpu validates before indexing with its inputs: a perm
+    that is not a bijection (EPERM), a community id or column out of range
+    (EINVAL) are refused, never used as addresses."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = synth.config(1, small=True).A
+    pr, _ = spmv.reorder(A.row_ptr, A.col, "rabbit")
+    comm = spmv.reorder_last_comm(A.n)
+    rp = torch.from_numpy(A.row_ptr).to(dev)
+    col = torch.from_numpy(A.col).to(dev)
+    bad_perm = pr.copy()
+    bad_perm[0] = bad_perm[1]
+    with pytest.raises(spmv.SpmvError) as e:
+        spmv.rabbitpp_gpu(rp, col, torch.from_numpy(bad_perm).to(dev), torch.from_numpy(comm).to(dev))
+    assert e.value.status == 2
+    bad_comm = comm.copy()
+    bad_comm[3] = A.n + 7
+    with pytest.raises(spmv.SpmvError) as e:
+        spmv.rabbitpp_gpu(rp, col, torch.from_numpy(pr).to(dev), torch.from_numpy(bad_comm).to(dev))
+    assert e.value.status == 1
+    bad_col = A.col.copy()
+    bad_col[5] = -3
+    with pytest.raises(spmv.SpmvError) as e:
+        spmv.rabbitpp_gpu(rp, torch.from_numpy(bad_col).to(dev), torch.from_numpy(pr).to(dev),
+                          torch.from_numpy(comm).to(dev))
+    assert e.value.status == 1
+
+
+def test_rmat26_rabbitpp_full_size(dev):
+    """BASELINE configs[2] (RMAT-26) at full size in RABBIT++ order (concurrent
+    RABBIT merges + the RABBIT++ post-pass): the hub-prefix persisting window,
+    the stream cache policy and every row class at scale, sampled rows' CSR
+    bit-exact and y within the tolerance, every row against the compensated C
+    oracle."""
+    _full_size_check(dev, 3, "rabbitpp", parallel=True)
