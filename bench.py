@@ -259,10 +259,20 @@ def run_gpu(args):
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
         P = spmv.Plan(inp.rp_d, inp.col_d, inp.val_d, perm_d, world=world, rank=rank,
-                      variant=args.variant, nccl_comm=comm,
+                      variant=args.variant, nccl_comm=comm, permute=False,
                       exchange=spmv.EXCHANGE_PEER if args.exchange == "peer" else spmv.EXCHANGE_COLL)
         torch.cuda.synchronize(dev)
         plan_s = time.perf_counter() - t0
+        # B = P A P^T timed on its own: algorithmic bytes
+        # 16 NZ + 20 N (read A, gather perm, write B, row pointers, inv)
+        pe0, pe1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        pe0.record(stream)
+        P.permute(stream)
+        pe1.record(stream)
+        torch.cuda.synchronize(dev)
+        permute_ms = pe0.elapsed_time(pe1)
+        nnz_loc = P.info()["nnz_local"]
+        permute_bytes = 16 * nnz_loc + 20 * (P.info()["row_end"] - P.info()["row_begin"])
         info = P.info()
         hc = pb = None
         if world > 1 and args.backend != "nccl":
@@ -335,7 +345,8 @@ def run_gpu(args):
         gbs = ideal / (ms * 1e-3) / 1e9
         res = {"ms": ms, "gbs_ideal_over_t": gbs, "gflops": 2 * inp.nnz / (ms * 1e-3) / 1e9,
                "runtime_over_ideal": hbm / gbs, "reorder_s": st.get("seconds"),
-               "plan_permute_s": plan_s,
+               "plan_s": plan_s, "permute_ms": permute_ms,
+               "permute_gbs": permute_bytes / (permute_ms * 1e-3) / 1e9,
                "H": info["hot_prefix"], "cta_rows": info["n_cta_rows"],
                "mid_rows": info["n_mid_rows"], "hub_rows": info["n_hub_rows"],
                "l2_window_bytes": P.info()["l2_window_bytes"],
@@ -399,7 +410,9 @@ def run_gpu(args):
             line["clocks"] = ck
             line["input_prep"] = {"generate_s": round(inp.gen_s, 3),
                                   "reorder_s": round(st.get("wall_s", 0.0), 3) if rank == 0 else None,
-                                  "plan_permute_s": round(plan_s, 4)}
+                                  "plan_s": round(plan_s, 4), "permute_ms": round(permute_ms, 3),
+                                  "permute_gbs": round(permute_bytes / (permute_ms * 1e-3) / 1e9, 1),
+                                  "permute_bytes_algorithmic": permute_bytes}
         if pb is not None:
             pb.close()
         P.close()

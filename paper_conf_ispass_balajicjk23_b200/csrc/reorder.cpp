@@ -597,7 +597,9 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
   // aggregated list is large enough to deserve every thread later); mode 1:
   // nothing else runs (no recheck needed); mode 2: as 1, aggregated with
   // every thread
-  constexpr size_t BIG = (size_t)1 << 16;
+  // postponed with every thread: lists of more than 1/(32 T) of all entries
+  // (smaller ones are cheaper on one thread while the others work)
+  const size_t BIG = std::max<size_t>((size_t)1 << 16, (size_t)(two_m / (32 * (int64_t)T)));
   std::vector<std::vector<int32_t>> bigs(T);
   auto step = [&](int32_t u, HashAcc& H, std::vector<Edge>& tl, int tid, int mode) -> bool {
     int64_t tu;
@@ -837,13 +839,37 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
     std::memset(&S0, 0, sizeof(S0));
     // skew: top ceil(0.1 N) row lengths / NZ
     {
-      std::vector<int64_t> L(n);
-      for (int64_t i = 0; i < n; ++i) L[i] = rp[i + 1] - rp[i];
-      int64_t top = (int64_t)std::ceil(0.1 * (double)n);
+      // exact: lengths below 2^16 by a histogram (per thread, merged), the few
+      // longer ones sorted; the top ceil(0.1 N) taken from the longest down
+      const int64_t top = (int64_t)std::ceil(0.1 * (double)n);
       if (top > 0 && n > 0) {
-        std::nth_element(L.begin(), L.begin() + (top - 1), L.end(), std::greater<int64_t>());
-        int64_t s = 0;
-        for (int64_t i = 0; i < top; ++i) s += L[i];
+        constexpr int64_t HB = 1 << 16;
+        std::vector<int64_t> hist(HB, 0);
+        std::vector<int64_t> longl;
+#pragma omp parallel
+        {
+          std::vector<int64_t> h(HB, 0);
+          std::vector<int64_t> lg;
+#pragma omp for schedule(static) nowait
+          for (int64_t i = 0; i < n; ++i) {
+            const int64_t L = rp[i + 1] - rp[i];
+            if (L < HB) h[L]++;
+            else lg.push_back(L);
+          }
+#pragma omp critical
+          {
+            for (int64_t b = 0; b < HB; ++b) hist[b] += h[b];
+            longl.insert(longl.end(), lg.begin(), lg.end());
+          }
+        }
+        std::sort(longl.begin(), longl.end(), std::greater<int64_t>());
+        int64_t left = top, s = 0;
+        for (size_t q = 0; q < longl.size() && left > 0; ++q, --left) s += longl[q];
+        for (int64_t b = HB - 1; b >= 0 && left > 0; --b) {
+          const int64_t take = std::min(left, hist[b]);
+          s += take * b;
+          left -= take;
+        }
         S0.skew = nnz ? (double)s / (double)nnz : 0.0;
       }
     }
@@ -893,8 +919,11 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
         // community sizes
         {
           std::vector<int64_t> sz(n, 0);
-          for (int64_t v = 0; v < n; ++v) sz[R.comm[v]]++;
+          const Rabbit& Rr = R;
+#pragma omp parallel for schedule(static)
+          for (int64_t v = 0; v < n; ++v) __atomic_fetch_add(&sz[Rr.comm[v]], (int64_t)1, __ATOMIC_RELAXED);
           int64_t mx = 0;
+#pragma omp parallel for reduction(max : mx) schedule(static)
           for (int64_t v = 0; v < n; ++v) mx = std::max(mx, sz[v]);
           g_cache.largest = n ? (double)mx / (double)n : 0.0;
         }
@@ -919,14 +948,25 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
             vtot[v] = t;
             insp[v] = ins;
           }
-          std::vector<__int128> inc(n, 0), totc(n, 0);
+          // per-community sums fit int64 (each <= 2m); Q' itself needs int128
+          std::vector<int64_t> inc(n, 0), totc(n, 0);
+#pragma omp parallel for schedule(static)
           for (int64_t v = 0; v < n; ++v) {
-            inc[R.comm[v]] += vin[v];
-            totc[R.comm[v]] += vtot[v];
+            __atomic_fetch_add(&inc[Rr.comm[v]], vin[v], __ATOMIC_RELAXED);
+            __atomic_fetch_add(&totc[Rr.comm[v]], vtot[v], __ATOMIC_RELAXED);
+          }
+          const int T = omp_get_max_threads();
+          std::vector<__int128> qt(T, 0);
+#pragma omp parallel num_threads(T)
+          {
+            __int128 a = 0;
+#pragma omp for schedule(static)
+            for (int64_t c = 0; c < n; ++c)
+              if (totc[c] || inc[c]) a += (__int128)R.two_m * inc[c] - (__int128)totc[c] * totc[c];
+            qt[omp_get_thread_num()] = a;
           }
           __int128 q = 0;
-          for (int64_t c = 0; c < n; ++c)
-            if (totc[c] || inc[c]) q += (__int128)R.two_m * inc[c] - totc[c] * totc[c];
+          for (int t = 0; t < T; ++t) q += qt[t];
           g_cache.qnum = (double)q;
           g_cache.q = R.two_m ? (double)q / ((double)R.two_m * (double)R.two_m) : 0.0;
         }
@@ -939,7 +979,7 @@ extern "C" spmv_status spmv_reorder(int64_t n, int64_t nnz, const int64_t* rp, c
 #pragma omp for schedule(dynamic, 4096)
             for (int64_t i = 0; i < n; ++i) {
               tmp.assign(col + rp[i], col + rp[i + 1]);
-              std::sort(tmp.begin(), tmp.end());
+              if (!std::is_sorted(tmp.begin(), tmp.end())) std::sort(tmp.begin(), tmp.end());
               tmp.erase(std::unique(tmp.begin(), tmp.end()), tmp.end());
               for (int32_t j : tmp)
                 if (j != i) {
