@@ -241,16 +241,46 @@ struct Rabbit {
   std::vector<MergeRec> log;  // filled when requested (SPMV_REORDER_LOG)
 };
 
-// ascending (deg, id) order of the vertices (reading c7): stable counting sort
+// ascending (deg, id) order of the vertices (reading c7): a stable counting
+// sort, in parallel -- threads own contiguous id ranges, per-thread histograms
+// of degrees below 2^16 are scanned degree-major, so ids stay ascending inside
+// each degree; the few larger degrees are sorted by (deg, id) and go last
 std::vector<int64_t> degree_order(const std::vector<int64_t>& deg) {
   const int64_t n = (int64_t)deg.size();
-  int64_t maxd = 0;
-  for (int64_t v = 0; v < n; ++v) maxd = std::max(maxd, deg[v]);
+  constexpr int64_t DB = 1 << 16;
+  const int T = omp_get_max_threads();
   std::vector<int64_t> order(n);
-  std::vector<int64_t> c(maxd + 2, 0);
-  for (int64_t v = 0; v < n; ++v) c[deg[v] + 1]++;
-  for (int64_t d = 0; d <= maxd; ++d) c[d + 1] += c[d];
-  for (int64_t v = 0; v < n; ++v) order[c[deg[v]]++] = v;
+  std::vector<int64_t> h((size_t)T * DB, 0);  // [t][d]
+  std::vector<std::vector<int64_t>> big(T);
+#pragma omp parallel num_threads(T)
+  {
+    const int t = omp_get_thread_num();
+    const int64_t lo = n * t / T, hi = n * (t + 1) / T;
+    int64_t* ht = h.data() + (size_t)t * DB;
+    for (int64_t v = lo; v < hi; ++v) {
+      if (deg[v] < DB) ht[deg[v]]++;
+      else big[t].push_back(v);
+    }
+#pragma omp barrier
+#pragma omp single
+    {
+      int64_t a = 0;
+      for (int64_t d = 0; d < DB; ++d)
+        for (int k = 0; k < T; ++k) {
+          const int64_t c = h[(size_t)k * DB + d];
+          h[(size_t)k * DB + d] = a;
+          a += c;
+        }
+      std::vector<int64_t> bg;
+      for (auto& b : big) bg.insert(bg.end(), b.begin(), b.end());
+      std::sort(bg.begin(), bg.end(), [&](int64_t x, int64_t y) {
+        return deg[x] != deg[y] ? deg[x] < deg[y] : x < y;
+      });
+      for (int64_t v : bg) order[a++] = v;
+    }
+    for (int64_t v = lo; v < hi; ++v)
+      if (deg[v] < DB) order[ht[deg[v]]++] = v;
+  }
   return order;
 }
 
@@ -509,7 +539,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
     }
   };
   const int T = omp_get_max_threads();
-  std::vector<std::vector<int32_t>> tops(T), deferred(T);
+  std::vector<std::vector<int32_t>> deferred(T);
   std::vector<std::vector<MergeRec>> logs(T);
   std::vector<int64_t> merges(T, 0), retries(T, 0);
   std::vector<HashAcc> Hs(T), Hsmall(T);  // small: vertices with short lists (cache-resident)
@@ -635,7 +665,6 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
       if (best == -1 || bestdq <= 0) {
         free_children();
         tot[u].store(tu, std::memory_order_release);
-        tops[tid].push_back(u);
         return true;
       }
       if (mode != 0) {  // exclusive: the aggregation is current, the gain exact
@@ -692,8 +721,7 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
         if (outcome == 3) {  // the best gain vanished: u stays top level
           free_children();
           tot[u].store(tu, std::memory_order_release);
-          tops[tid].push_back(u);
-          return true;
+            return true;
         }
         tot[u].store(tu, std::memory_order_release);
         deferred[tid].push_back(u);
@@ -743,10 +771,32 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
   }
   if (want_log)
     for (auto& l : logs) R.log.insert(R.log.end(), l.begin(), l.end());
-  // top level in processing order (the sequential reading's append order)
+  // top level = the vertices still roots, in processing order (the
+  // sequential reading's append order): a parallel compaction of `order`
   std::vector<int32_t> top;
-  for (auto& t : tops) top.insert(top.end(), t.begin(), t.end());
-  std::sort(top.begin(), top.end(), [&](int32_t a, int32_t b) { return pos[a] < pos[b]; });
+  {
+    const int TT = omp_get_max_threads();
+    std::vector<int64_t> cnt(TT + 1, 0);
+#pragma omp parallel num_threads(TT)
+    {
+      const int t = omp_get_thread_num();
+      const int64_t lo = n * t / TT, hi = n * (t + 1) / TT;
+      int64_t c = 0;
+      for (int64_t i = lo; i < hi; ++i) c += tot[order[i]].load(std::memory_order_relaxed) != MERGED;
+      cnt[t + 1] = c;
+#pragma omp barrier
+#pragma omp single
+      {
+        for (int k = 1; k <= TT; ++k) cnt[k] += cnt[k - 1];
+        top.resize(cnt[TT]);
+      }
+      int64_t o = cnt[t];
+      for (int64_t i = lo; i < hi; ++i)
+        if (tot[order[i]].load(std::memory_order_relaxed) != MERGED) top[o++] = (int32_t)order[i];
+    }
+  }
+#pragma omp parallel for schedule(dynamic, 65536)
+  for (int64_t v = 0; v < n; ++v) std::vector<Edge>().swap(agg[v]);
   std::vector<std::vector<Edge>>().swap(agg);
   dendrogram_ids(top, first_child, next_sib, R, n);
   phase("par:dfs", tp);
