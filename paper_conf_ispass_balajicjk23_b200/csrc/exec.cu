@@ -134,6 +134,44 @@ __device__ __forceinline__ double warp_sum_d(double s) {
 // order puts the columns of nearby rows on few lines)
 __device__ __forceinline__ float gx(const float* __restrict__ x, int c) { return __ldg(x + c); }
 
+// Streamed col / val entries of the MID / CTA / hub kernels.  SM 0: ld.cs
+// (L1 and L2 evict-first); SM 1: no L1 allocation, so the L1 keeps gathered x
+// lines only; SM 2: no L1 allocation and L2 evict_first.
+// (SM 2 takes an L2::evict_first cache policy from createpolicy: the static
+// qualifier exists only for 256-bit loads.)
+template <int SM>
+__device__ __forceinline__ int32_t lds(const int32_t* p, uint64_t pol) {
+  if constexpr (SM == 0) {
+    return __ldcs(p);
+  } else {
+    int32_t r;
+    if constexpr (SM == 1)
+      asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(r) : "l"(p));
+    else
+      asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+  }
+}
+template <int SM>
+__device__ __forceinline__ float lds(const float* p, uint64_t pol) {
+  if constexpr (SM == 0) {
+    return __ldcs(p);
+  } else {
+    float r;
+    if constexpr (SM == 1)
+      asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(p));
+    else
+      asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r) : "l"(p), "l"(pol));
+    return r;
+  }
+}
+template <int SM>
+__device__ __forceinline__ uint64_t stream_policy() {
+  uint64_t pol = 0;
+  if constexpr (SM == 2) asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+
 // ------------------------------------------------------------ stream tiles
 // k_panel: persistent CTAs, each over a contiguous range of stream tiles (a
 // panel of consecutive rows), two CTAs of 16 warps per SM.  Thread 0 keeps the
@@ -389,7 +427,7 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 }
 
 // ------------------------------------------------------------- long rows
-template <typename OT, bool SS, int UNR = 4>
+template <typename OT, bool SS, int SM, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
@@ -398,6 +436,7 @@ __global__ void __launch_bounds__(256)
   const int lane = threadIdx.x & 31;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float alpha = alpha_of(ss_in);
+  const uint64_t pol = stream_policy<SM>();
   for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < nrows; q += W) {
     const int r = rows[q];
     const int64_t b = (int64_t)rp[r];
@@ -414,8 +453,8 @@ __global__ void __launch_bounds__(256)
 #pragma unroll
       for (int u = 0; u < UNR; ++u) {
         const bool pu = j + 32 * u < L;
-        c[u] = pu ? __ldcs(cc + j + 32 * u) : 0;
-        v[u] = pu ? __ldcs(vv + j + 32 * u) : 0.f;
+        c[u] = pu ? lds<SM>(cc + j + 32 * u, pol) : 0;
+        v[u] = pu ? lds<SM>(vv + j + 32 * u, pol) : 0.f;
       }
 #pragma unroll
       for (int u = 0; u < UNR; ++u) xv[u] = (j + 32 * u < L) ? gx(x, c[u]) : 0.f;
@@ -433,12 +472,13 @@ __global__ void __launch_bounds__(256)
 }
 
 // canonical W = 256 sum of entries [b, b + L) of a row
-template <int UNR = 4>
+template <int SM, int UNR = 4>
 __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             const float* __restrict__ val,
                                             const float* __restrict__ x, int64_t b, int64_t L,
                                             float* red) {
   const int tid = threadIdx.x;
+  const uint64_t pol = stream_policy<SM>();
   float s = 0.f;
   // UNR strided entries in flight, ragged end guarded (+0 slots, as k_warp_rows)
   for (int64_t t = tid; t < L; t += 256 * UNR) {
@@ -447,8 +487,8 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
 #pragma unroll
     for (int u = 0; u < UNR; ++u) {
       const bool pu = t + 256 * u < L;
-      c[u] = pu ? __ldcs(col + b + t + 256 * u) : 0;
-      v[u] = pu ? __ldcs(val + b + t + 256 * u) : 0.f;
+      c[u] = pu ? lds<SM>(col + b + t + 256 * u, pol) : 0;
+      v[u] = pu ? lds<SM>(val + b + t + 256 * u, pol) : 0.f;
     }
 #pragma unroll
     for (int u = 0; u < UNR; ++u) xv[u] = (t + 256 * u < L) ? gx(x, c[u]) : 0.f;
@@ -467,7 +507,7 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
   return r;  // valid in thread 0
 }
 
-template <typename OT, bool SS, int UNR = 4>
+template <typename OT, bool SS, int SM, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_cta_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
@@ -476,7 +516,7 @@ __global__ void __launch_bounds__(256)
   __shared__ float red[256];
   const int r = rows[blockIdx.x];
   const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
-  const float s = cta_sum256<UNR>(col, val, x, b, L, red);
+  const float s = cta_sum256<SM, UNR>(col, val, x, b, L, red);
   if (threadIdx.x == 0) {
     const float v = __fmul_rn(s, alpha_of(ss_in));
     store_y<SS>(y, dst, r, v);
@@ -485,7 +525,7 @@ __global__ void __launch_bounds__(256)
   }
 }
 
-template <typename OT, int UNR = 4>
+template <typename OT, int SM, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_hub_chunk(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
@@ -497,7 +537,7 @@ __global__ void __launch_bounds__(256)
   const int64_t rb = (int64_t)rp[r], L = (int64_t)rp[r + 1] - rb;
   const int64_t b = rb + (int64_t)chunk_idx[c] * HUB_CHUNK;
   const int64_t m = min((int64_t)HUB_CHUNK, rb + L - b);
-  const float s = cta_sum256<UNR>(col, val, x, b, m, red);
+  const float s = cta_sum256<SM, UNR>(col, val, x, b, m, red);
   if (threadIdx.x == 0) part[c] = (double)s;
 }
 
@@ -623,6 +663,7 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 // sliding shared-memory x window, one barrier per block and evict_first
 // stream hints ran 1.25x slower than this plain form on SBM 4M/64M.
 constexpr int LN_THREADS = 256;
+constexpr int MID_STREAM_DEFAULT = 0;  // stream-load mode of the MID / CTA / hub kernels (lds)
 constexpr int LN_WARPS = LN_THREADS / 32;
 constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 
@@ -785,9 +826,9 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
 
 // Row-class kernels other than the short-row one: MID rows (warp per row),
 // CTA rows, hub chunks + fixup, on the two plan-owned streams s1 / s2.
-template <typename OT, bool SS>
-void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s1,
-                 cudaStream_t s2, bool lane_mode, const YDst& dst) {
+template <typename OT, bool SS, int SM>
+void launch_rows_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s1,
+                   cudaStream_t s2, bool lane_mode, const YDst& dst) {
   const OT* rp = (const OT*)p->d_rp;
   const int32_t* col = p->d_col;
   const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
@@ -795,34 +836,28 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
   if (nw) {
     const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
-    int unr = 4;  // entries in flight per lane (same association for any value)
-    if (const char* e = getenv("SPMV_WARP_UNR")) unr = atoi(e) == 8 ? 8 : 4;  // dev knob
-    if (unr == 8)
-      k_warp_rows<OT, SS, 8><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, dst);
-    else
-      k_warp_rows<OT, SS, 4><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, dst);
+    k_warp_rows<OT, SS, SM><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, dst);
   }
-  int cunr = 4;  // entries in flight per thread (same association for any value)
-  if (const char* e = getenv("SPMV_CTA_UNR")) cunr = atoi(e) == 8 ? 8 : 4;  // dev knob
-  if (p->n_cta) {
-    if (cunr == 8)
-      k_cta_rows<OT, SS, 8><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
-                                                                 p->d_cta_rows, ss_in, p->d_cta_ss, dst);
-    else
-      k_cta_rows<OT, SS, 4><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
-                                                                 p->d_cta_rows, ss_in, p->d_cta_ss, dst);
-  }
+  if (p->n_cta)
+    k_cta_rows<OT, SS, SM><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
+                                                              p->d_cta_rows, ss_in, p->d_cta_ss, dst);
   if (p->n_chunks) {
-    if (cunr == 8)
-      k_hub_chunk<OT, 8><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
-          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part);
-    else
-      k_hub_chunk<OT, 4><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
-          rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part);
+    k_hub_chunk<OT, SM><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
+        rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part);
     const unsigned g = (unsigned)((p->n_hub + 127) / 128);
     k_hub_fix<SS><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
                                       ss_in, y, p->d_hub_ss, dst);
   }
+}
+
+template <typename OT, bool SS>
+void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, cudaStream_t s1,
+                 cudaStream_t s2, bool lane_mode, const YDst& dst) {
+  int sm = MID_STREAM_DEFAULT;
+  if (const char* e = getenv("SPMV_MID_STREAM")) sm = std::min(2, std::max(0, atoi(e)));  // dev knob
+  if (sm == 1) launch_rows_t<OT, SS, 1>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+  else if (sm == 2) launch_rows_t<OT, SS, 2>(p, x, y, ss_in, s1, s2, lane_mode, dst);
+  else launch_rows_t<OT, SS, 0>(p, x, y, ss_in, s1, s2, lane_mode, dst);
 }
 
 template <typename OT>
@@ -889,6 +924,13 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   if (const char* e = getenv("SPMV_WIN_COLS")) want = std::min<int64_t>(p->x_len, atoll(e));  // dev knob
   int64_t bytes = std::min<int64_t>(want * 4, (int64_t)maxwin);
   bytes = std::min<int64_t>(bytes, (int64_t)maxpers);
+  double hit = p->opts.l2_hit_ratio;
+  if (const char* e = getenv("SPMV_WIN_FRAC")) {  // dev knob: window <= this fraction of L2
+    int l2 = 0;
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, p->device);
+    bytes = std::min<int64_t>(bytes, (int64_t)(atof(e) * l2));
+  }
+  if (const char* e = getenv("SPMV_WIN_HIT")) hit = std::min(1.0, std::max(0.0, atof(e)));  // dev knob
   if (bytes <= 0) return;
   size_t cur = 0;
   cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
@@ -902,7 +944,7 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   cudaStreamAttrValue v{};
   v.accessPolicyWindow.base_ptr = (void*)x;
   v.accessPolicyWindow.num_bytes = (size_t)bytes;
-  v.accessPolicyWindow.hitRatio = (float)p->opts.l2_hit_ratio;
+  v.accessPolicyWindow.hitRatio = (float)hit;
   v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
   v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
   if (cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v) != cudaSuccess) {

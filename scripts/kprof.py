@@ -1,7 +1,7 @@
 """Dev tool (under gpurun): one plan of config K in ordering O, timed execs.
 
     python scripts/kprof.py --config 5 --ordering rabbitpp [--steps 10] [--iterate]
-                            [--ncu 1] [--env SPMV_WARP_UNR=8 ...]
+                            [--ncu 1] [--env SPMV_MID_STREAM=1 ...]
 
 Generation on the GPU for RMAT / Kronecker configs, the reorder memoised in
 /tmp/permcache (survives within one gpurun call), cold execs (512 MiB read +

@@ -1,10 +1,12 @@
-"""Entries in flight per lane of the warp-per-row and CTA-per-row kernels
-(SPMV_WARP_UNR / SPMV_CTA_UNR dev knobs, 4 or 8).  Each lane sums its strided
-entries j, j + W, j + 2W, ... in that order whatever the unroll, and a guarded
-slot past the row adds +0, so y is bitwise the same for every setting
-(include/spmv.h canonical order) and within 1e-5 * sum|a x| of the oracle.
-Row lengths sit on both sides of every 32*4, 32*8, 256*4, 256*8 boundary and of
-the class bounds (32 / 2048 / 16384, hub chunking above)."""
+"""Stream-load modes of the warp-per-row, CTA-per-row and hub-chunk kernels
+(SPMV_MID_STREAM dev knob: ld.cs; no L1 allocation; no L1 allocation + L2
+evict_first policy).  They change where col / val are cached, never the
+values or the association (each lane sums its strided entries j, j + W, ...
+in that order, four in flight, a guarded slot past the row adding +0), so y
+is bitwise the same for every mode (include/spmv.h canonical order) and
+within 1e-5 * sum|a x| of the oracle.  Row lengths sit on both sides of every
+32*4 and 256*4 boundary and of the class bounds (32 / 2048 / 16384, hub
+chunking above)."""
 import numpy as np
 import pytest
 
@@ -43,7 +45,7 @@ ALL = CASES + [("boundaries", _boundaries)]
 
 
 @pytest.mark.parametrize("name,make", ALL)
-def test_unroll_bitwise_and_oracle(dev, name, make, monkeypatch):
+def test_stream_modes_bitwise_and_oracle(dev, name, make, monkeypatch):
     A = make()
     perm = rabbit.random_perm(A.n, 5) if A.nnz and name != "boundaries" else None
     P = mk_plan(A, perm, dev)
@@ -54,13 +56,12 @@ def test_unroll_bitwise_and_oracle(dev, name, make, monkeypatch):
     ref = ospmv.spmv(Bp, Bc, Bv, xB)
     scale = ospmv.abs_rowsum(Bp, Bc, Bv, xB)
     ys = []
-    for wu, cu in (("4", "4"), ("8", "4"), ("4", "8"), ("8", "8")):
-        monkeypatch.setenv("SPMV_WARP_UNR", wu)
-        monkeypatch.setenv("SPMV_CTA_UNR", cu)
+    for mode in ("0", "1", "2"):
+        monkeypatch.setenv("SPMV_MID_STREAM", mode)
         y = P.exec(xd).cpu().numpy()
         err = np.abs(y.astype(np.float64) - ref.astype(np.float64))
         bad = ~(err <= TOL * scale + 1e-37)
-        assert not bad.any(), f"{name} {wu}/{cu}: {int(bad.sum())} rows bad"
+        assert not bad.any(), f"{name} mode {mode}: {int(bad.sum())} rows bad"
         ys.append(y.view(np.int32).copy())
     for y in ys[1:]:
         assert np.array_equal(ys[0], y)
