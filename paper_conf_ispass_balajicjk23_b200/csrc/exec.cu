@@ -427,6 +427,38 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 }
 
 // ------------------------------------------------------------- long rows
+// canonical W = 32 sum of row r (32 strided partials + xor tree), valid in
+// every lane.  UNR strided entries in flight per lane, the ragged end
+// guarded: a slot past the row adds +0, which leaves s unchanged (s starts at
+// +0 and is never -0), so the association is exactly j, j+32, j+64, ...
+template <typename OT, int SM, int UNR = 4>
+__device__ __forceinline__ float warp_row_sum(const OT* __restrict__ rp,
+                                              const int32_t* __restrict__ col,
+                                              const float* __restrict__ val,
+                                              const float* __restrict__ x, int r, int lane,
+                                              uint64_t pol) {
+  const int64_t b = (int64_t)rp[r];
+  const int L = (int)((int64_t)rp[r + 1] - b);
+  const int32_t* cc = col + b;
+  const float* vv = val + b;
+  float s = 0.f;
+  for (int j = lane; j < L; j += 32 * UNR) {
+    int c[UNR];
+    float v[UNR], xv[UNR];
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) {
+      const bool pu = j + 32 * u < L;
+      c[u] = pu ? lds<SM>(cc + j + 32 * u, pol) : 0;
+      v[u] = pu ? lds<SM>(vv + j + 32 * u, pol) : 0.f;
+    }
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) xv[u] = (j + 32 * u < L) ? gx(x, c[u]) : 0.f;
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
+  }
+  return warp_tree(s);
+}
+
 template <typename OT, bool SS, int SM, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
@@ -439,29 +471,7 @@ __global__ void __launch_bounds__(256)
   const uint64_t pol = stream_policy<SM>();
   for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < nrows; q += W) {
     const int r = rows[q];
-    const int64_t b = (int64_t)rp[r];
-    const int L = (int)((int64_t)rp[r + 1] - b);
-    const int32_t* cc = col + b;
-    const float* vv = val + b;
-    float s = 0.f;
-    // UNR strided entries in flight per lane, the ragged end guarded: a slot
-    // past the row adds +0, which leaves s unchanged (s starts at +0 and is
-    // never -0), so the association is exactly j, j+32, j+64, ... for any UNR
-    for (int j = lane; j < L; j += 32 * UNR) {
-      int c[UNR];
-      float v[UNR], xv[UNR];
-#pragma unroll
-      for (int u = 0; u < UNR; ++u) {
-        const bool pu = j + 32 * u < L;
-        c[u] = pu ? lds<SM>(cc + j + 32 * u, pol) : 0;
-        v[u] = pu ? lds<SM>(vv + j + 32 * u, pol) : 0.f;
-      }
-#pragma unroll
-      for (int u = 0; u < UNR; ++u) xv[u] = (j + 32 * u < L) ? gx(x, c[u]) : 0.f;
-#pragma unroll
-      for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
-    }
-    s = warp_tree(s);
+    const float s = warp_row_sum<OT, SM, UNR>(rp, col, val, x, r, lane, pol);
     if (lane == 0) {
       const float v = __fmul_rn(s, alpha);
       store_y<SS>(y, dst, r, v);
@@ -703,6 +713,56 @@ __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
         : "l"(p));
 }
 
+// sequential (canonical W = 1) sum of a row of L <= SHORT_MAX entries
+// starting at a, streamed in 8-entry, 32-byte-aligned chunks.  Every slot of
+// a chunk holds a valid column of some row (or the zero tail padding), so its
+// x read is always safe; a slot outside [a, a + L) contributes the product +0
+// (selected, not computed: a neighbouring row's Inf / NaN value never reaches
+// this row, Alg. 1), which leaves the sum unchanged (it starts at +0 and is
+// never -0).
+template <typename OT, int EF>
+__device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
+                                              const float* __restrict__ val,
+                                              const float* __restrict__ x, OT a, int L) {
+  float res = 0.f;
+  const int32_t* cp = col + (a & ~(OT)7);
+  const float* vp = val + (a & ~(OT)7);
+  const int lo = (int)(a & 7), hi = lo + L;
+#pragma unroll 2
+  for (int k = 0; k < hi; k += 8) {
+    int cc[8];
+    float vv[8];
+    if (EF == 2 && k == 0) {  // (warp-uniform: every lane starts at k = 0)
+      ld_v8_stream<0>(cp + k, cc);
+      ld_v8_stream<0>(vp + k, vv);
+    } else {
+      ld_v8_stream<EF == 0 ? 0 : 1>(cp + k, cc);
+      ld_v8_stream<EF == 0 ? 0 : 1>(vp + k, vv);
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const float xv = gx(x, cc[i]);
+      res = __fadd_rn(res, (k + i >= lo && k + i < hi) ? __fmul_rn(vv[i], xv) : 0.f);
+    }
+  }
+  return res;
+}
+
+// fixed-order per-block sum of y^2 over a 256-thread block (independent of
+// the grid): warp xor sums, then the 8 warp sums in order; written by thread 0
+__device__ __forceinline__ void block_ss256(double ssacc, double* wss, double* out) {
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  ssacc = warp_sum_d(ssacc);
+  if (lane == 0) wss[warp] = ssacc;
+  __syncthreads();
+  if (tid == 0) {
+    double t = 0.0;
+    for (int w = 0; w < 8; ++w) t += wss[w];
+    *out = t;
+  }
+  __syncthreads();
+}
+
 // minBlocksPerSM = 1 lets ptxas keep both chunks and all 16 gathers of a
 // 16-entry row in flight per lane (64 registers, 4 CTAs/SM); capping registers
 // for more CTAs measured 20-40 % slower
@@ -746,26 +806,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
         // contributes the product +0 (selected, not computed: a neighbouring
         // row's Inf / NaN value never reaches this row, Alg. 1), which leaves
         // res unchanged (it starts at +0 and is never -0).
-        const int32_t* cp = col + (a & ~(OT)7);
-        const float* vp = val + (a & ~(OT)7);
-        const int lo = (int)(a & 7), hi = lo + L;
-#pragma unroll 2
-        for (int k = 0; k < hi; k += 8) {
-          int cc[8];
-          float vv[8];
-          if (EF == 2 && k == 0) {  // (warp-uniform: every lane starts at k = 0)
-            ld_v8_stream<0>(cp + k, cc);
-            ld_v8_stream<0>(vp + k, vv);
-          } else {
-            ld_v8_stream<EF == 0 ? 0 : 1>(cp + k, cc);
-            ld_v8_stream<EF == 0 ? 0 : 1>(vp + k, vv);
-          }
-#pragma unroll
-          for (int i = 0; i < 8; ++i) {
-            const float xv = gx(x, cc[i]);
-            res = __fadd_rn(res, (k + i >= lo && k + i < hi) ? __fmul_rn(vv[i], xv) : 0.f);
-          }
-        }
+        res = lane_row_sum<OT, EF>(col, val, x, a, L);
       }
     }
     double ssacc = 0.0;
@@ -774,16 +815,62 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
       store_y<SS>(y, dst, r, o);
       if (SS) ssacc = (double)o * (double)o;
     }
-    if (SS) {  // fixed-order per-block sum of y^2 (independent of the grid)
-      ssacc = warp_sum_d(ssacc);
-      if (lane == 0) wss[warp] = ssacc;
-      __syncthreads();
-      if (tid == 0) {
-        double t = 0.0;
-        for (int w = 0; w < LN_WARPS; ++w) t += wss[w];
-        blk_ss[blk] = t;
+    if (SS) block_ss256(ssacc, wss, blk_ss + blk);
+  }
+  fence_bcast<SS>(dst);
+}
+
+// Small plans (no hub rows, few entries): every row class in ONE launch, no
+// fork / join -- CTA i < B_lane computes the 256-row lane block i, the next
+// B_mid CTAs eight MID rows each (warp per row), the last n_cta CTAs one CTA
+// row each.  Same per-row association as the separate kernels (bitwise equal
+// y); launch and fork/join latency dominate such plans (RMAT-16: 8 MB).
+template <typename OT, bool SS, int EF, int SM>
+__global__ void __launch_bounds__(LN_THREADS)
+    k_small(const OT* __restrict__ rp, const int32_t* __restrict__ col,
+            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
+            int64_t nrows, const int32_t* __restrict__ mid_rows, int64_t n_mid,
+            const int32_t* __restrict__ cta_rows, int64_t B_lane, int64_t B_mid,
+            const double* __restrict__ ss_in, double* __restrict__ blk_ss,
+            double* __restrict__ mid_ss, double* __restrict__ cta_ss, const YDst dst) {
+  __shared__ double wss[LN_WARPS];
+  __shared__ float red[256];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const float alpha = alpha_of(ss_in);
+  const int64_t blk = blockIdx.x;
+  if (blk < B_lane) {  // block-uniform branches
+    const int64_t r = blk * LN_THREADS + tid;
+    double ssacc = 0.0;
+    if (r < nrows) {
+      const OT a = rp[r];
+      const int L = (int)(rp[r + 1] - a);
+      if (L <= SHORT_MAX) {
+        const float o = __fmul_rn(lane_row_sum<OT, EF>(col, val, x, a, L), alpha);
+        store_y<SS>(y, dst, r, o);
+        if (SS) ssacc = (double)o * (double)o;
       }
-      __syncthreads();
+    }
+    if (SS) block_ss256(ssacc, wss, blk_ss + blk);
+  } else if (blk < B_lane + B_mid) {
+    const int64_t q = (blk - B_lane) * 8 + warp;
+    if (q < n_mid) {
+      const int r = mid_rows[q];
+      const float s = warp_row_sum<OT, SM>(rp, col, val, x, r, lane, stream_policy<SM>());
+      if (lane == 0) {
+        const float v = __fmul_rn(s, alpha);
+        store_y<SS>(y, dst, r, v);
+        if (SS) mid_ss[q] = (double)v * (double)v;
+      }
+    }
+  } else {
+    const int64_t i = blk - B_lane - B_mid;
+    const int r = cta_rows[i];
+    const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
+    const float s = cta_sum256<SM>(col, val, x, b, L, red);
+    if (tid == 0) {
+      const float v = __fmul_rn(s, alpha);
+      store_y<SS>(y, dst, r, v);
+      if (SS) cta_ss[i] = (double)v * (double)v;
     }
   }
   fence_bcast<SS>(dst);
@@ -860,6 +947,16 @@ void launch_rows(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   else launch_rows_t<OT, SS, 0>(p, x, y, ss_in, s1, s2, lane_mode, dst);
 }
 
+// plans run by k_small: lane variant, no hub rows (their fp64 fixup is a
+// second kernel), MID or CTA rows present (else k_lane is one launch anyway),
+// at most SMALL_NNZ entries (launch / fork-join bound); SPMV_SMALL=0/1 dev knob
+constexpr int64_t SMALL_NNZ = int64_t(1) << 24;
+bool small_plan(const spmv_plan_s* p) {
+  if (p->n_chunks || !(p->n_mid || p->n_cta)) return false;
+  if (const char* e = getenv("SPMV_SMALL")) return atoi(e) != 0;
+  return p->nnz_local <= SMALL_NNZ;
+}
+
 template <typename OT>
 void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double* ss_out,
                 cudaStream_t s, const YDst& dst) {
@@ -871,6 +968,28 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   // with the short-row kernel (fork/join by events; CUDA-graph capturable).
   // The fork is recorded before (early, default) or after the short-row
   // launch (SPMV_FORK_EARLY=0: the other classes start when it has finished).
+  if (lane_mode && small_plan(p)) {  // one launch for every row class
+    const int64_t B_lane = (p->nrows + LN_THREADS - 1) / LN_THREADS, B_mid = (p->n_mid + 7) / 8;
+    const unsigned g = (unsigned)(B_lane + B_mid + p->n_cta);
+    const OT* rp = (const OT*)p->d_rp;
+    constexpr int SM = MID_STREAM_DEFAULT;
+#define SPMV_SMALL_ARGS                                                                      \
+  rp, p->d_col, p->d_val, x, y, p->nrows, p->d_mid_rows, p->n_mid, p->d_cta_rows, B_lane, B_mid, \
+      ss_in, p->d_blk_ss, p->d_mid_ss, p->d_cta_ss, dst
+    const bool ef = lane_ef_mode(p) == 1;
+    if (SS) {
+      if (ef) k_small<OT, true, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      else k_small<OT, true, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      ss_reduce(p, p->d_blk_ss, B_lane, p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta, p->d_hub_ss,
+                0, ss_out, s);
+    } else {
+      if (ef) k_small<OT, false, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      else k_small<OT, false, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+    }
+#undef SPMV_SMALL_ARGS
+    SPMV_LAUNCH_CHECK();
+    return;
+  }
   cudaStream_t s1 = s, s2 = s;
   const bool conc = p->conc && (nw > 0 || p->n_cta > 0 || p->n_chunks > 0);
   bool early = true;
@@ -1000,6 +1119,7 @@ void exec_streams(spmv_plan_s* p) { ensure_aux(p); }
 int exec_launches(const spmv_plan_s* p, bool ss) {
   const bool lane_mode = p->opts.variant != 1;
   const int longk = (p->n_cta ? 1 : 0) + (p->n_chunks ? 2 : 0);
+  if (lane_mode && small_plan(p)) return 1 + (ss ? 2 : 0);
   return (lane_mode ? (p->nrows ? 1 : 0) + (p->n_mid ? 1 : 0)
                     : (p->K ? 1 : 0) + (p->n_warp ? 1 : 0)) +
          longk + (ss ? 2 : 0);

@@ -448,3 +448,32 @@ def test_rmat26_rabbitpp_full_size(dev):
     bit-exact and y within the tolerance, every row against the compensated C
     oracle."""
     _full_size_check(dev, 3, "rabbitpp", parallel=True)
+
+
+@pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("rmat12", "kron14", "stencil24")])
+def test_small_plan_single_launch_bitwise(dev, name, make, monkeypatch):
+    """Small plans (no hub rows, <= 2^24 entries) run every row class in one
+    k_small launch: y and the scaled step's sum of y^2 bitwise equal to the
+    separate per-class kernels, one launch (+2 for the norm) instead of up to
+    three plus fork / join."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = make()
+    perm = spmv.reorder(A.row_ptr, A.col, "rabbitpp")[0]
+    P = mk_plan(A, perm, dev)
+    i = P.info()
+    xB = P.permute_vec(torch.from_numpy(synth.vector(A.n, 6)).to(dev))
+    out = {}
+    for mode in ("0", "1"):
+        monkeypatch.setenv("SPMV_SMALL", mode)
+        y = P.exec(xB)
+        z = torch.empty_like(y)
+        ss = torch.zeros(1, dtype=torch.float64, device=dev)
+        P.exec_scaled(xB, z, None, ss)
+        out[mode] = (y.clone(), z.clone(), ss.clone(), P.info()["exec_launches"])
+    assert torch.equal(out["0"][0].view(torch.int32), out["1"][0].view(torch.int32))
+    assert torch.equal(out["0"][1].view(torch.int32), out["1"][1].view(torch.int32))
+    assert torch.equal(out["0"][2], out["1"][2])
+    if i["n_mid_rows"] or i["n_cta_rows"]:
+        assert out["1"][3] == 1
+    monkeypatch.delenv("SPMV_SMALL")
+    P.close()
