@@ -674,6 +674,7 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 // stream hints ran 1.25x slower than this plain form on SBM 4M/64M.
 constexpr int LN_THREADS = 256;
 constexpr int MID_STREAM_DEFAULT = 0;  // stream-load mode of the MID / CTA / hub kernels (lds)
+constexpr bool LANE_COOP_DEFAULT = false;  // k_lane_coop for plans with shared chunks
 constexpr int LN_WARPS = LN_THREADS / 32;
 constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 
@@ -820,6 +821,77 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
   fence_bcast<SS>(dst);
 }
 
+// Warp-cooperative short rows (plans whose 8-entry chunks are shared by
+// neighbouring rows, i.e. stream_evict_first == 0: meshes, power-law graphs).
+// A warp's 32 consecutive rows occupy one contiguous entry range; the warp
+// streams it once, 256-bit chunks with L2::evict_first spread over the lanes
+// (every sector read by exactly one lane, so evict-first costs no refetch and
+// the gathered x keeps the L2), forms the products v * x[c] into a warp-private
+// shared buffer, and each lane then sums its own row from the buffer left to
+// right -- the canonical W = 1 association, bitwise k_lane's result.  A warp
+// holding a row with L > SHORT_MAX (computed by the MID / CTA / hub kernels)
+// takes k_lane's per-lane path instead, so no long row is streamed twice.
+constexpr int COOP_BUF = 32 * SHORT_MAX + 16;  // products of one warp (32 rows <= 32 entries)
+
+template <typename OT, bool SS>
+__global__ void __launch_bounds__(LN_THREADS)
+    k_lane_coop(const OT* __restrict__ rp, const int32_t* __restrict__ col,
+                const float* __restrict__ val, const float* __restrict__ x,
+                float* __restrict__ y, int64_t nrows, const double* __restrict__ ss_in,
+                double* __restrict__ blk_ss, const YDst dst) {
+  __shared__ __align__(32) float prod[LN_WARPS][COOP_BUF];
+  __shared__ double wss[LN_WARPS];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
+  const float alpha = alpha_of(ss_in);
+  float* pw = prod[warp];
+  for (int64_t blk = blockIdx.x; blk < NB; blk += gridDim.x) {
+    const int64_t r = blk * LN_THREADS + tid;
+    const bool valid = r < nrows;
+    const OT a = valid ? rp[r] : (OT)0;
+    const OT e = valid ? rp[r + 1] : (OT)0;
+    const int L = (int)(e - a);
+    float res = 0.f;
+    const bool mine = valid && L <= SHORT_MAX;
+    if (__any_sync(0xffffffffu, valid && L > SHORT_MAX)) {
+      if (mine) res = lane_row_sum<OT, 0>(col, val, x, a, L);
+    } else {
+      // the warp's entries [base, end): first row's start, last valid row's end
+      const int last = __popc(__ballot_sync(0xffffffffu, valid)) - 1;
+      const OT base = __shfl_sync(0xffffffffu, a, 0);
+      const OT end = __shfl_sync(0xffffffffu, e, last < 0 ? 0 : last);
+      const OT cb = base & ~(OT)7;
+      const int nch = (int)((end - cb + 7) >> 3);
+      for (int k = lane; k < nch; k += 32) {
+        int cc[8];
+        float vv[8];
+        ld_v8_stream<1>(col + cb + 8 * k, cc);
+        ld_v8_stream<1>(val + cb + 8 * k, vv);
+        float pr[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) pr[i] = __fmul_rn(vv[i], gx(x, cc[i]));
+        float4* d = reinterpret_cast<float4*>(pw + 8 * k);
+        d[0] = make_float4(pr[0], pr[1], pr[2], pr[3]);
+        d[1] = make_float4(pr[4], pr[5], pr[6], pr[7]);
+      }
+      __syncwarp();
+      if (mine) {
+        const float* q = pw + (int)(a - cb);
+        for (int i = 0; i < L; ++i) res = __fadd_rn(res, q[i]);
+      }
+      __syncwarp();
+    }
+    double ssacc = 0.0;
+    if (mine) {
+      const float o = __fmul_rn(res, alpha);
+      store_y<SS>(y, dst, r, o);
+      if (SS) ssacc = (double)o * (double)o;
+    }
+    if (SS) block_ss256(ssacc, wss, blk_ss + blk);
+  }
+  fence_bcast<SS>(dst);
+}
+
 // Small plans (no hub rows, few entries): every row class in ONE launch, no
 // fork / join -- CTA i < B_lane computes the 256-row lane block i, the next
 // B_mid CTAs eight MID rows each (warp per row), the last n_cta CTAs one CTA
@@ -906,6 +978,18 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   // normal, the rest evict_first) via the SPMV_LANE_EF dev knob
   int ef = lane_ef_mode(p);
   if (const char* e = getenv("SPMV_LANE_EF")) ef = std::min(2, std::max(0, atoi(e)));  // dev knob
+  bool coop = ef == 0 && LANE_COOP_DEFAULT;
+  if (const char* e = getenv("SPMV_LANE_COOP")) coop = ef == 0 && atoi(e) != 0;  // dev knob
+  if (coop) {
+    int per_sm = LN_CTAS_PER_SM;
+    if (const char* e = getenv("SPMV_LANE_CTAS")) per_sm = std::max(1, atoi(e));  // dev knob
+    const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
+    const unsigned grid =
+        (unsigned)std::max<int64_t>(1, std::min(NB, (int64_t)num_sms(p->device) * per_sm));
+    k_lane_coop<OT, SS><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
+                                                     p->nrows, ss_in, p->d_blk_ss, dst);
+    return;
+  }
   if (ef == 1) launch_lane_t<OT, SS, 1>(p, x, y, ss_in, s, dst);
   else if (ef == 2) launch_lane_t<OT, SS, 2>(p, x, y, ss_in, s, dst);
   else launch_lane_t<OT, SS, 0>(p, x, y, ss_in, s, dst);
