@@ -17,6 +17,7 @@
 #include <dlfcn.h>
 
 #include <cmath>
+#include <cstdlib>
 #include <mutex>
 
 #include "plan.cuh"
@@ -138,10 +139,16 @@ void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s
   if (iters < 1) SPMV_FAIL(SPMV_EINVAL, "iters must be >= 1");
   if (!p->permuted) SPMV_FAIL(SPMV_ESTATE, "spmv_iterate before spmv_permute");
   const int G = p->world;
+  // SPMV_FORCE_COLL=1 (test knob): run the collectives even for world == 1
+  // (an all-reduce / all-gatherv over one rank is the identity), so the NCCL
+  // path is exercised on a one-GPU box
+  bool force = false;
+  if (const char* e = getenv("SPMV_FORCE_COLL")) force = atoi(e) != 0;
+  const bool coll = G > 1 || force;
   const bool peer = G > 1 && p->opts.exchange == SPMV_EXCHANGE_PEER;
   NcclCtx nctx{p->opts.nccl_comm, p->rank};
   spmv_coll_t c{};
-  if (G > 1) {
+  if (coll) {
     if (p->has_coll) {
       c = p->coll;
     } else {
@@ -185,7 +192,7 @@ void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s
     } else {
       exec(p, a, b + p->y_offset, sin, sout, s);
     }
-    if (G > 1) {
+    if (coll) {
       if (c.allreduce_sum_f64(c.ctx, sout, 1, s))
         SPMV_FAIL(SPMV_ENCCL, std::string("spmv_iterate: all-reduce failed: ") + get_error());
       if (!peer && c.allgatherv_f32(c.ctx, b, xb.data(), G, s))
