@@ -318,6 +318,7 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->stream_evict_first = spmv::lane_ef_mode(p);
   info->exec_launches = spmv::exec_launches(p, false);
   info->spmm4_launches = spmv::spmm4_launches(p);
+  info->hot_prefix_nnz = p->H_nnz;
   API_END
 }
 

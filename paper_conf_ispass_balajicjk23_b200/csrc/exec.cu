@@ -1117,6 +1117,15 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   SPMV_LAUNCH_CHECK();
 }
 
+// The persisting window on x_B[0:H) pays only when the prefix is HOT: its
+// columns read at least WIN_HOT times as often as an average column (the hub
+// group of a power-law graph under RABBIT++; not the 98.7 % "hubs" of a
+// stencil, r57: 7.11 ms with the window vs 6.68 without).  Its size is capped
+// at half the L2: the whole prefix pinned (83 MB on Kronecker-28) starves the
+// rest of the step (r56/r57: 24.5 -> 21.0 ms).
+constexpr double WIN_HOT = 2.0;
+constexpr double WIN_L2_FRAC = 0.5;
+
 void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   if (p->win_ptr == (const void*)x && p->win_stream[slot] == s) return;
   int maxwin = 0, maxpers = 0;
@@ -1128,10 +1137,12 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   int64_t bytes = std::min<int64_t>(want * 4, (int64_t)maxwin);
   bytes = std::min<int64_t>(bytes, (int64_t)maxpers);
   double hit = p->opts.l2_hit_ratio;
-  if (const char* e = getenv("SPMV_WIN_FRAC")) {  // dev knob: window <= this fraction of L2
+  {
+    double frac = WIN_L2_FRAC;
+    if (const char* e = getenv("SPMV_WIN_FRAC")) frac = atof(e);  // dev knob
     int l2 = 0;
     cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, p->device);
-    bytes = std::min<int64_t>(bytes, (int64_t)(atof(e) * l2));
+    if (l2 > 0) bytes = std::min<int64_t>(bytes, (int64_t)(frac * l2));
   }
   if (const char* e = getenv("SPMV_WIN_HIT")) hit = std::min(1.0, std::max(0.0, atof(e)));  // dev knob
   if (bytes <= 0) return;
@@ -1162,8 +1173,16 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   p->l2_window_bytes = bytes;
 }
 
+
+bool window_pays(const spmv_plan_s* p) {
+  if (p->H <= 0 || p->n <= 0 || p->nnz <= 0) return false;
+  if (const char* e = getenv("SPMV_WIN_FORCE")) return atoi(e) != 0;  // dev knob
+  const double hot = (double)p->H_nnz / (double)p->H, avg = (double)p->nnz / (double)p->n;
+  return hot >= WIN_HOT * avg;
+}
+
 void set_window(spmv_plan_s* p, const float* x, cudaStream_t s) {
-  if (!p->opts.l2_window || p->H <= 0 || s == nullptr) return;
+  if (!p->opts.l2_window || !window_pays(p) || s == nullptr) return;
   set_window_one(p, x, s, 0);
   if (p->conc) {
     set_window_one(p, x, p->aux[0], 1);

@@ -310,6 +310,14 @@ __global__ void k_colcnt(const int32_t* colA, const int32_t* perm, int64_t nnz, 
   GRID_STRIDE(k, nnz) atomicAdd(&cnt[perm[colA[k]]], 1u);
 }
 
+__global__ void k_sum_u32(const uint32_t* a, int64_t n, unsigned long long* out) {
+  unsigned long long acc = 0;
+  GRID_STRIDE(i, n) acc += a[i];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if ((threadIdx.x & 31) == 0 && acc) atomicAdd(out, acc);
+}
+
 __global__ void k_first_cold(const uint32_t* cnt, int64_t n, int64_t nnz,
                              unsigned long long* H) {
   // smallest j with !(colcnt_B[j] * N > NZ): warp-level min first, one atomic per warp
@@ -751,6 +759,18 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   SPMV_LAUNCH_CHECK();
   p->H = (int64_t)d2h_one(dH, s);
   dfree(dH);
+  // entries of B whose column lies in the hot prefix [0, H): the window of
+  // exec is worth its L2 only if those columns are read much more often than
+  // the average column
+  p->H_nnz = 0;
+  if (p->H > 0) {
+    unsigned long long* dsum = dalloc<unsigned long long>(1);
+    SPMV_CUDA(cudaMemsetAsync(dsum, 0, 8, s));
+    k_sum_u32<<<grid_for(p->H), TPB, 0, s>>>(cnt, p->H, dsum);
+    SPMV_LAUNCH_CHECK();
+    p->H_nnz = (int64_t)d2h_one(dsum, s);
+    dfree(dsum);
+  }
   dfree(cnt);
   dfree(rpB);
 

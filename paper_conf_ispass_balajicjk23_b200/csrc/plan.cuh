@@ -44,6 +44,7 @@ struct spmv_plan_s {
 
   // bins
   int64_t K = 0, n_cta = 0, n_hub = 0, n_chunks = 0, H = 0, max_hub_len = 0;
+  int64_t H_nnz = 0;  // entries of B whose column is in the hot prefix [0, H)
   int32_t* d_tiles = nullptr;      // [K+1]
   TileDesc* d_desc = nullptr;      // [K]
   int64_t n_warp = 0;

@@ -68,7 +68,8 @@ class _Info(ctypes.Structure):
         "n_tiles", "n_warp_rows", "n_cta_rows", "n_hub_rows", "n_hub_chunks", "n_mid_rows",
         "hot_prefix", "ideal_bytes")] + \
         [(n, ctypes.c_int32) for n in ("offset_bytes", "world", "rank", "permuted",
-                                       "l2_window_bytes", "stream_evict_first", "exec_launches", "spmm4_launches")]
+                                       "l2_window_bytes", "stream_evict_first", "exec_launches", "spmm4_launches")] + \
+        [("hot_prefix_nnz", ctypes.c_int64)]
 
 
 class _Stats(ctypes.Structure):

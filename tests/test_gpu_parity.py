@@ -477,3 +477,30 @@ def test_small_plan_single_launch_bitwise(dev, name, make, monkeypatch):
         assert out["1"][3] == 1
     monkeypatch.delenv("SPMV_SMALL")
     P.close()
+
+
+@pytest.mark.parametrize("name,make", [c for c in CASES if c[0] in ("kron14", "stencil24", "sbm16x1024")])
+def test_hot_prefix_window_gate(dev, name, make):
+    """H and the entries it covers are exact (oracle plan.hot_prefix); exec
+    pins x_B[0:H) in L2 only when those columns are read >= 2x as often as the
+    average column (power-law hub groups yes, a stencil's near-average "hubs"
+    no), at most half the L2."""
+    from paper_conf_ispass_balajicjk23_b200 import spmv
+    A = make()
+    perm = spmv.reorder(A.row_ptr, A.col, "rabbitpp")[0]
+    Bp, Bc, _ = permute.permute_csr(A.n, A.row_ptr, A.col, A.val, perm)
+    H = oplan.hot_prefix(A.n, Bc)
+    hot_nnz = int((Bc < H).sum())
+    P = mk_plan(A, perm, dev)
+    i = P.info()
+    assert i["hot_prefix"] == H and i["hot_prefix_nnz"] == hot_nnz
+    s = torch.cuda.Stream(device=dev)
+    xB = torch.zeros(A.n, device=dev)
+    P.exec(xB, stream=s)
+    torch.cuda.synchronize()
+    pays = H > 0 and hot_nnz * A.n >= 2 * A.nnz * H
+    win = P.info()["l2_window_bytes"]
+    assert (win > 0) == pays, (name, H, hot_nnz, win)
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    assert win <= l2 // 2
+    P.close()
