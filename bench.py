@@ -611,10 +611,10 @@ def cpu_baseline(inp, perm, budget_s=10.0, steps=None, warmup=0):
     cores, and the same loop on 1 core) on a bounded sample of the same
     reordered workload, in the metric's unit (ideal bytes of the sample, P:96
     restricted to its rows, per second).  Workloads above 2^28 entries are
-    sampled as a contiguous middle block of B's rows (~2^26 entries)."""
+    sampled as a contiguous middle block of B's rows (~2^24 entries)."""
     from oracle import cref
     big = inp.nnz > 2**28
-    rp, col, val, xB, r0, r1 = oracle_sample(inp, perm, target_nnz=2**26 if big else None)
+    rp, col, val, xB, r0, r1 = oracle_sample(inp, perm, target_nnz=2**24 if big else None)
     m, rows = int(rp[-1]), r1 - r0
     w_off = 8 if inp.nnz >= 2**31 else 4
     sample_ideal = 8 * m + (rows + 1) * w_off + 8 * rows
@@ -687,7 +687,8 @@ def main():
     ap.add_argument("--config", type=int, default=5, help="BASELINE.json config index (1-based)")
     ap.add_argument("--orderings", default=None,
                     help="comma list; the last one is the headline line (default: "
-                         "original,rabbit,rabbitpp for config 5, random,original,rabbit,rabbitpp else)")
+                         "original,rabbit,hubsort,rabbitpp for config 5, "
+                         "random,original,rabbit,rabbitpp else)")
     ap.add_argument("--seed", type=int, default=20230423)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)
@@ -708,7 +709,7 @@ def main():
                     help="test only: put every rank on cuda:0 (with --backend gloo)")
     args = ap.parse_args()
     if args.orderings is None:
-        args.orderings = "original,rabbit,rabbitpp" if args.config == 5 else \
+        args.orderings = "original,rabbit,hubsort,rabbitpp" if args.config == 5 else \
             "random,original,rabbit,rabbitpp"
     if args.warmup < 3:
         args.warmup = 3

@@ -16,9 +16,11 @@
 // second, possibly different, NCCL.
 #include <dlfcn.h>
 
+#include <chrono>
 #include <cmath>
 #include <cstdlib>
 #include <mutex>
+#include <thread>
 
 #include "plan.cuh"
 
@@ -56,8 +58,10 @@ struct Nccl {
   int (*group_start)() = nullptr;
   int (*group_end)() = nullptr;
   const char* (*error_string)(int) = nullptr;
+  int (*async_error)(void*, int*) = nullptr;  // ncclCommGetAsyncError
   bool ok = false;
 };
+constexpr int kNcclInProgress = 7;  // ncclInProgress
 constexpr int kNcclFloat32 = 7, kNcclFloat64 = 8, kNcclSum = 0;
 
 const Nccl& nccl() {
@@ -74,6 +78,7 @@ const Nccl& nccl() {
     N.group_start = (decltype(N.group_start))dlsym(h, "ncclGroupStart");
     N.group_end = (decltype(N.group_end))dlsym(h, "ncclGroupEnd");
     N.error_string = (decltype(N.error_string))dlsym(h, "ncclGetErrorString");
+    N.async_error = (decltype(N.async_error))dlsym(h, "ncclCommGetAsyncError");
     N.ok = N.all_reduce && N.broadcast && N.all_gather && N.group_start && N.group_end;
   });
   return N;
@@ -118,6 +123,29 @@ int nccl_allgatherv(void* ctx, float* x, const int64_t* b, int world, void* stre
   const int r2 = N.group_end();
   if (r || r2) nccl_fail(r ? r : r2, "grouped ncclBroadcast");
   return r ? r : r2;
+}
+
+// Wait for the step loop with NCCL's asynchronous error state polled: a
+// failed or aborted peer turns into SPMV_ENCCL instead of a hang, and so does
+// a loop that has not finished after SPMV_NCCL_TIMEOUT_S seconds (600).
+void wait_nccl(void* comm, cudaStream_t s) {
+  const Nccl& N = nccl();
+  double limit = 600.0;
+  if (const char* e = getenv("SPMV_NCCL_TIMEOUT_S")) limit = atof(e);
+  const auto t0 = std::chrono::steady_clock::now();
+  for (;;) {
+    const cudaError_t q = cudaStreamQuery(s);
+    if (q == cudaSuccess) return;
+    if (q != cudaErrorNotReady) SPMV_CUDA(q);
+    int st = 0;
+    if (N.async_error && N.async_error(comm, &st) == 0 && st != 0 && st != kNcclInProgress) {
+      nccl_fail(st, "NCCL asynchronous error");
+      throw Err{SPMV_ENCCL};
+    }
+    if (std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() > limit)
+      SPMV_FAIL(SPMV_ENCCL, "spmv_iterate: collectives did not complete within SPMV_NCCL_TIMEOUT_S");
+    std::this_thread::sleep_for(std::chrono::microseconds(200));
+  }
 }
 
 }  // namespace
@@ -206,6 +234,7 @@ void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s
       std::swap(a, b);
     }
   }
+  if (coll && !p->has_coll) wait_nccl(p->opts.nccl_comm, s);
   iterate_finish(a, x, xl, sin, lambda, s);
 }
 

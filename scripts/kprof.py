@@ -32,6 +32,7 @@ ap.add_argument("--iterate", action="store_true", help="time spmv_iterate steps 
 ap.add_argument("--ncu", type=int, default=0)
 ap.add_argument("--env", nargs="*", default=[])
 ap.add_argument("--sequential-reorder", action="store_true")
+ap.add_argument("--no-reset", action="store_true", help="flush without the persisting-L2 reset")
 a = ap.parse_args()
 for kv in a.env:
     k, v = kv.split("=", 1)
@@ -60,6 +61,8 @@ f = f"/tmp/permcache/{name}_{a.ordering}{'_seq' if a.sequential_reorder else ''}
 t0 = time.time()
 if a.ordering == "original":
     perm = np.arange(n, dtype=np.int32)
+elif a.ordering == "planted":
+    perm = np.ascontiguousarray(w.planted, np.int32)
 elif os.path.exists(f):
     perm = np.load(f)
 else:
@@ -79,7 +82,8 @@ sink = torch.zeros((), device=dev)
 
 def fl():
     torch.sum(flush, dim=0, out=sink)
-    spmv.lib().spmv_reset_persisting_l2(None)
+    if not a.no_reset:
+        spmv.lib().spmv_reset_persisting_l2(None)
 
 
 P.exec(xB, y)
@@ -126,7 +130,8 @@ if a.iterate:
     it_ms = e0.elapsed_time(e1) / a.steps
 h = hashlib.sha1(y.cpu().numpy().tobytes()).hexdigest()[:16]
 hbm = json.load(open("MEASURED_PEAKS.json"))["hbm_gbs"] if os.path.exists("MEASURED_PEAKS.json") else 6548.8
-print(json.dumps({"workload": name, "ordering": a.ordering, "env": a.env, "n": n, "nnz": nnz,
+print(json.dumps({"workload": name, "ordering": a.ordering, "env": a.env + (["no-reset"] if a.no_reset else []),
+                  "n": n, "nnz": nnz,
                   "cold_ms": round(cold_ms, 4), "warm_ms": round(warm_ms, 4), "iterate_ms": it_ms,
                   "x_ideal_cold": round(cold_ms * 1e-3 * hbm * 1e9 / ideal, 3),
                   "gen_s": round(gen_s, 2), "reorder_s": round(reorder_s, 1),
