@@ -862,6 +862,7 @@ __global__ void __launch_bounds__(LN_THREADS)
       const OT end = __shfl_sync(0xffffffffu, e, last < 0 ? 0 : last);
       const OT cb = base & ~(OT)7;
       const int nch = (int)((end - cb + 7) >> 3);
+#pragma unroll 4
       for (int k = lane; k < nch; k += 32) {
         int cc[8];
         float vv[8];
