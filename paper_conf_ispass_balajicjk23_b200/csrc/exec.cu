@@ -674,7 +674,6 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 // stream hints ran 1.25x slower than this plain form on SBM 4M/64M.
 constexpr int LN_THREADS = 256;
 constexpr int MID_STREAM_DEFAULT = 0;  // stream-load mode of the MID / CTA / hub kernels (lds)
-constexpr bool LANE_COOP_DEFAULT = false;  // k_lane_coop for plans with shared chunks
 constexpr int LN_WARPS = LN_THREADS / 32;
 constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 
@@ -749,19 +748,13 @@ __device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
   return res;
 }
 
-// fixed-order per-block sum of y^2 over a 256-thread block (independent of
-// the grid): warp xor sums, then the 8 warp sums in order; written by thread 0
-__device__ __forceinline__ void block_ss256(double ssacc, double* wss, double* out) {
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+// fixed-order sum of y^2 of one warp's 32 rows (xor tree), stored as partial
+// (blk, warp) -- no CTA barrier in the lane kernels; the partials of a
+// 256-row block are then eight consecutive entries of the plan's partial
+// array, summed with everything else by ss_reduce in a grid-independent order
+__device__ __forceinline__ void warp_ss(double ssacc, double* out) {
   ssacc = warp_sum_d(ssacc);
-  if (lane == 0) wss[warp] = ssacc;
-  __syncthreads();
-  if (tid == 0) {
-    double t = 0.0;
-    for (int w = 0; w < 8; ++w) t += wss[w];
-    *out = t;
-  }
-  __syncthreads();
+  if ((threadIdx.x & 31) == 0) out[threadIdx.x >> 5] = ssacc;
 }
 
 // minBlocksPerSM = 1 lets ptxas keep both chunks and all 16 gathers of a
@@ -773,8 +766,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
            int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss,
            const YDst dst) {
-  __shared__ double wss[LN_WARPS];
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int tid = threadIdx.x;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
   const float alpha = alpha_of(ss_in);
   // row pointers are loaded one block iteration ahead
@@ -816,79 +808,7 @@ __global__ void __launch_bounds__(LN_THREADS, 1)
       store_y<SS>(y, dst, r, o);
       if (SS) ssacc = (double)o * (double)o;
     }
-    if (SS) block_ss256(ssacc, wss, blk_ss + blk);
-  }
-  fence_bcast<SS>(dst);
-}
-
-// Warp-cooperative short rows (plans whose 8-entry chunks are shared by
-// neighbouring rows, i.e. stream_evict_first == 0: meshes, power-law graphs).
-// A warp's 32 consecutive rows occupy one contiguous entry range; the warp
-// streams it once, 256-bit chunks with L2::evict_first spread over the lanes
-// (every sector read by exactly one lane, so evict-first costs no refetch and
-// the gathered x keeps the L2), forms the products v * x[c] into a warp-private
-// shared buffer, and each lane then sums its own row from the buffer left to
-// right -- the canonical W = 1 association, bitwise k_lane's result.  A warp
-// holding a row with L > SHORT_MAX (computed by the MID / CTA / hub kernels)
-// takes k_lane's per-lane path instead, so no long row is streamed twice.
-constexpr int COOP_BUF = 32 * SHORT_MAX + 16;  // products of one warp (32 rows <= 32 entries)
-
-template <typename OT, bool SS>
-__global__ void __launch_bounds__(LN_THREADS)
-    k_lane_coop(const OT* __restrict__ rp, const int32_t* __restrict__ col,
-                const float* __restrict__ val, const float* __restrict__ x,
-                float* __restrict__ y, int64_t nrows, const double* __restrict__ ss_in,
-                double* __restrict__ blk_ss, const YDst dst) {
-  __shared__ __align__(32) float prod[LN_WARPS][COOP_BUF];
-  __shared__ double wss[LN_WARPS];
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
-  const float alpha = alpha_of(ss_in);
-  float* pw = prod[warp];
-  for (int64_t blk = blockIdx.x; blk < NB; blk += gridDim.x) {
-    const int64_t r = blk * LN_THREADS + tid;
-    const bool valid = r < nrows;
-    const OT a = valid ? rp[r] : (OT)0;
-    const OT e = valid ? rp[r + 1] : (OT)0;
-    const int L = (int)(e - a);
-    float res = 0.f;
-    const bool mine = valid && L <= SHORT_MAX;
-    if (__any_sync(0xffffffffu, valid && L > SHORT_MAX)) {
-      if (mine) res = lane_row_sum<OT, 0>(col, val, x, a, L);
-    } else {
-      // the warp's entries [base, end): first row's start, last valid row's end
-      const int last = __popc(__ballot_sync(0xffffffffu, valid)) - 1;
-      const OT base = __shfl_sync(0xffffffffu, a, 0);
-      const OT end = __shfl_sync(0xffffffffu, e, last < 0 ? 0 : last);
-      const OT cb = base & ~(OT)7;
-      const int nch = (int)((end - cb + 7) >> 3);
-#pragma unroll 4
-      for (int k = lane; k < nch; k += 32) {
-        int cc[8];
-        float vv[8];
-        ld_v8_stream<1>(col + cb + 8 * k, cc);
-        ld_v8_stream<1>(val + cb + 8 * k, vv);
-        float pr[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) pr[i] = __fmul_rn(vv[i], gx(x, cc[i]));
-        float4* d = reinterpret_cast<float4*>(pw + 8 * k);
-        d[0] = make_float4(pr[0], pr[1], pr[2], pr[3]);
-        d[1] = make_float4(pr[4], pr[5], pr[6], pr[7]);
-      }
-      __syncwarp();
-      if (mine) {
-        const float* q = pw + (int)(a - cb);
-        for (int i = 0; i < L; ++i) res = __fadd_rn(res, q[i]);
-      }
-      __syncwarp();
-    }
-    double ssacc = 0.0;
-    if (mine) {
-      const float o = __fmul_rn(res, alpha);
-      store_y<SS>(y, dst, r, o);
-      if (SS) ssacc = (double)o * (double)o;
-    }
-    if (SS) block_ss256(ssacc, wss, blk_ss + blk);
+    if (SS) warp_ss(ssacc, blk_ss + blk * LN_WARPS);
   }
   fence_bcast<SS>(dst);
 }
@@ -906,7 +826,6 @@ __global__ void __launch_bounds__(LN_THREADS)
             const int32_t* __restrict__ cta_rows, int64_t B_lane, int64_t B_mid,
             const double* __restrict__ ss_in, double* __restrict__ blk_ss,
             double* __restrict__ mid_ss, double* __restrict__ cta_ss, const YDst dst) {
-  __shared__ double wss[LN_WARPS];
   __shared__ float red[256];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const float alpha = alpha_of(ss_in);
@@ -923,7 +842,7 @@ __global__ void __launch_bounds__(LN_THREADS)
         if (SS) ssacc = (double)o * (double)o;
       }
     }
-    if (SS) block_ss256(ssacc, wss, blk_ss + blk);
+    if (SS) warp_ss(ssacc, blk_ss + blk * LN_WARPS);
   } else if (blk < B_lane + B_mid) {
     const int64_t q = (blk - B_lane) * 8 + warp;
     if (q < n_mid) {
@@ -979,18 +898,6 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   // normal, the rest evict_first) via the SPMV_LANE_EF dev knob
   int ef = lane_ef_mode(p);
   if (const char* e = getenv("SPMV_LANE_EF")) ef = std::min(2, std::max(0, atoi(e)));  // dev knob
-  bool coop = ef == 0 && LANE_COOP_DEFAULT;
-  if (const char* e = getenv("SPMV_LANE_COOP")) coop = ef == 0 && atoi(e) != 0;  // dev knob
-  if (coop) {
-    int per_sm = LN_CTAS_PER_SM;
-    if (const char* e = getenv("SPMV_LANE_CTAS")) per_sm = std::max(1, atoi(e));  // dev knob
-    const int64_t NB = (p->nrows + LN_THREADS - 1) / LN_THREADS;
-    const unsigned grid =
-        (unsigned)std::max<int64_t>(1, std::min(NB, (int64_t)num_sms(p->device) * per_sm));
-    k_lane_coop<OT, SS><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
-                                                     p->nrows, ss_in, p->d_blk_ss, dst);
-    return;
-  }
   if (ef == 1) launch_lane_t<OT, SS, 1>(p, x, y, ss_in, s, dst);
   else if (ef == 2) launch_lane_t<OT, SS, 2>(p, x, y, ss_in, s, dst);
   else launch_lane_t<OT, SS, 0>(p, x, y, ss_in, s, dst);
@@ -1065,8 +972,8 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
     if (SS) {
       if (ef) k_small<OT, true, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
       else k_small<OT, true, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
-      ss_reduce(p, p->d_blk_ss, B_lane, p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta, p->d_hub_ss,
-                0, ss_out, s);
+      ss_reduce(p, p->d_blk_ss, B_lane * LN_WARPS, p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta,
+                p->d_hub_ss, 0, ss_out, s);
     } else {
       if (ef) k_small<OT, false, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
       else k_small<OT, false, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
@@ -1109,8 +1016,8 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   }
   if (SS) {
     if (lane_mode)
-      ss_reduce(p, p->d_blk_ss, (p->nrows + LN_THREADS - 1) / LN_THREADS, p->d_mid_ss, p->n_mid,
-                p->d_cta_ss, p->n_cta, p->d_hub_ss, p->n_hub, ss_out, s);
+      ss_reduce(p, p->d_blk_ss, (p->nrows + LN_THREADS - 1) / LN_THREADS * LN_WARPS, p->d_mid_ss,
+                p->n_mid, p->d_cta_ss, p->n_cta, p->d_hub_ss, p->n_hub, ss_out, s);
     else
       ss_reduce(p, p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss, p->n_cta,
                 p->d_hub_ss, p->n_hub, ss_out, s);

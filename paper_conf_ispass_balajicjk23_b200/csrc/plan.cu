@@ -860,14 +860,14 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   // exec scratch
   p->d_chunk_part = dalloc<double>(p->n_chunks);
   p->d_tile_ss = dalloc<double>(p->K);
-  p->d_blk_ss = dalloc<double>((nr + 63) / 64);  // >= blocks of k_lane (>= 64 rows each)
+  p->d_blk_ss = dalloc<double>((nr + 255) / 256 * 8 + 8);  // one per warp of each 256-row block
   p->d_warp_ss = dalloc<double>(p->n_warp);
   p->d_mid_ss = dalloc<double>(p->n_mid);
   p->d_cta_ss = dalloc<double>(p->n_cta);
   p->d_hub_ss = dalloc<double>(p->n_hub);
   p->d_ss = dalloc<double>(4);
   {  // segment sums of the norm reduction (exec.cu ss_reduce), either row scheme
-    const int64_t lane_parts = (nr + 63) / 64 + p->n_mid + p->n_cta + p->n_hub;
+    const int64_t lane_parts = (nr + 255) / 256 * 8 + p->n_mid + p->n_cta + p->n_hub;
     const int64_t tile_parts = p->K + p->n_warp + p->n_cta + p->n_hub;
     p->d_ss_part = dalloc<double>(std::max(lane_parts, tile_parts) / 16384 + 2);
   }

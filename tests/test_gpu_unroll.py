@@ -6,8 +6,7 @@ in that order, four in flight, a guarded slot past the row adding +0), so y
 is bitwise the same for every mode (include/spmv.h canonical order) and
 within 1e-5 * sum|a x| of the oracle.  Row lengths sit on both sides of every
 32*4 and 256*4 boundary and of the class bounds (32 / 2048 / 16384, hub
-chunking above).  The warp-cooperative short-row kernel (SPMV_LANE_COOP)
-sums the same products in the same order from shared memory: bitwise too."""
+chunking above)."""
 import numpy as np
 import pytest
 
@@ -57,14 +56,13 @@ def test_stream_modes_bitwise_and_oracle(dev, name, make, monkeypatch):
     ref = ospmv.spmv(Bp, Bc, Bv, xB)
     scale = ospmv.abs_rowsum(Bp, Bc, Bv, xB)
     ys = []
-    for mode, coop in (("0", "0"), ("1", "0"), ("2", "0"), ("0", "1")):
+    for mode in ("0", "1", "2"):
         monkeypatch.setenv("SPMV_MID_STREAM", mode)
-        monkeypatch.setenv("SPMV_LANE_COOP", coop)   # k_lane_coop (plans with shared chunks)
         monkeypatch.setenv("SPMV_SMALL", "0")        # the per-class kernels, not k_small
         y = P.exec(xd).cpu().numpy()
         err = np.abs(y.astype(np.float64) - ref.astype(np.float64))
         bad = ~(err <= TOL * scale + 1e-37)
-        assert not bad.any(), f"{name} mode {mode} coop {coop}: {int(bad.sum())} rows bad"
+        assert not bad.any(), f"{name} mode {mode}: {int(bad.sum())} rows bad"
         ys.append(y.view(np.int32).copy())
     for y in ys[1:]:
         assert np.array_equal(ys[0], y)
