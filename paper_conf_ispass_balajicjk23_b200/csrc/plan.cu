@@ -72,6 +72,18 @@ __global__ void k_inverse(const int32_t* perm, int64_t n, int32_t* inv, int* fla
   }
 }
 
+// start of B's local row j in A: srcA[perm[i] - rb] = row_ptr_A[i] for the
+// rows this rank holds (one coalesced read of row_ptr_A, no inv -> row_ptr_A
+// dependent chain in the relabel kernels)
+template <typename T>
+__global__ void k_srcA(const T* rpA, const int32_t* perm, int64_t n, int64_t rb, int64_t re,
+                       int64_t* srcA) {
+  GRID_STRIDE(i, n) {
+    const int64_t j = perm[i];
+    if (j >= rb && j < re) srcA[j - rb] = (int64_t)rpA[i];
+  }
+}
+
 template <typename T>
 __global__ void k_lenB(const T* rpA, const int32_t* perm, int64_t n, int64_t* lenB) {
   GRID_STRIDE(i, n) lenB[perm[i]] = (int64_t)rpA[i + 1] - (int64_t)rpA[i];
@@ -371,7 +383,7 @@ template <typename AT, typename OT>
 __global__ void __launch_bounds__(256)
     k_relabel_sort_short(const AT* __restrict__ rpA, const int32_t* __restrict__ colA,
                          const float* __restrict__ valA, const int32_t* __restrict__ perm,
-                         const int32_t* __restrict__ inv, int64_t rb, int64_t nrows,
+                         const int64_t* __restrict__ srcA, int64_t nrows,
                          const OT* __restrict__ rpB, int32_t* __restrict__ colB,
                          float* __restrict__ valB) {
   const int lane = threadIdx.x & 31, half = lane >> 4, hl = lane & 15;
@@ -389,7 +401,7 @@ __global__ void __launch_bounds__(256)
       uint64_t key = ~0ull;
       float v = 0.f;
       if (hl < L) {
-        const int64_t a = (int64_t)rpA[inv[rb + r]];
+        const int64_t a = srcA[r];
         key = mkkey(perm[colA[a + hl]], hl);
         v = valA[a + hl];
       }
@@ -408,7 +420,7 @@ __global__ void __launch_bounds__(256)
         uint64_t key = ~0ull;
         float v = 0.f;
         if (lane < Lh) {
-          const int64_t a = (int64_t)rpA[inv[rb + rr]];
+          const int64_t a = srcA[rr];
           key = mkkey(perm[colA[a + lane]], lane);
           v = valA[a + lane];
         }
@@ -425,7 +437,7 @@ __global__ void __launch_bounds__(256)
 // warp per row for rows with 32 < L <= WARP_MAX (relabel only; sorted after)
 template <typename AT, typename OT>
 __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* valA,
-                               const int32_t* perm, const int32_t* inv, int64_t rb,
+                               const int32_t* perm, const int64_t* srcA,
                                int64_t nrows, const OT* rpB, int32_t* colB, float* valB) {
   const int lane = threadIdx.x & 31;
   int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -433,8 +445,7 @@ __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* 
   for (int64_t r = w; r < nrows; r += nw) {
     int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d;
     if (L <= SHORT_MAX || L > WARP_MAX) continue;  // k_relabel_sort_short / k_relabel_cta
-    int64_t i = inv[rb + r];
-    int64_t a = (int64_t)rpA[i];
+    int64_t a = srcA[r];
     for (int64_t k = lane; k < L; k += 32) {
       colB[d + k] = perm[colA[a + k]];
       valB[d + k] = valA[a + k];
@@ -445,14 +456,13 @@ __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* 
 // CTA per long row (list)
 template <typename AT, typename OT>
 __global__ void k_relabel_cta(const AT* rpA, const int32_t* colA, const float* valA,
-                              const int32_t* perm, const int32_t* inv, int64_t rb,
+                              const int32_t* perm, const int64_t* srcA,
                               const int32_t* rows, int64_t nrows_list, const OT* rpB,
                               int32_t* colB, float* valB) {
   for (int64_t t = blockIdx.x; t < nrows_list; t += gridDim.x) {
     int64_t r = rows[t];
     int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d;
-    int64_t i = inv[rb + r];
-    int64_t a = (int64_t)rpA[i];
+    int64_t a = srcA[r];
     for (int64_t k = threadIdx.x; k < L; k += blockDim.x) {
       colB[d + k] = perm[colA[a + k]];
       valB[d + k] = valA[a + k];
@@ -461,14 +471,16 @@ __global__ void k_relabel_cta(const AT* rpA, const int32_t* colA, const float* v
 }
 
 // ----------------------------------------------------------------- row sort
-// CTA bitonic sort of one row of length L <= P held in shared memory.
+// CTA bitonic sort of one row of length L <= pe held in shared memory, pe =
+// the next power of two >= L (>= 64), <= P: the network is sized to the row,
+// not to the class bound (a 130-entry row sorts 256 keys, not 1024).
 template <int P>
-__device__ void smem_bitonic(uint64_t* keys, float* vals) {
+__device__ void smem_bitonic(uint64_t* keys, float* vals, int pe) {
 #pragma unroll 1
-  for (int k = 2; k <= P; k <<= 1) {
+  for (int k = 2; k <= pe; k <<= 1) {
 #pragma unroll 1
     for (int j = k >> 1; j > 0; j >>= 1) {
-      for (int i = threadIdx.x; i < P; i += blockDim.x) {
+      for (int i = threadIdx.x; i < pe; i += blockDim.x) {
         int ixj = i ^ j;
         if (ixj > i) {
           uint64_t a = keys[i], b = keys[ixj];
@@ -496,12 +508,14 @@ __global__ void k_sort_cta(const OT* rp, const int32_t* rows, int64_t nlist, int
   for (int64_t t = blockIdx.x; t < nlist; t += gridDim.x) {
     int64_t r = rows[t];
     int64_t d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d;
-    for (int i = threadIdx.x; i < P; i += blockDim.x) {
+    int pe = 64;
+    while (pe < L) pe <<= 1;
+    for (int i = threadIdx.x; i < pe; i += blockDim.x) {
       keys[i] = i < L ? mkkey(col[d + i], i) : ~0ull;
       vals[i] = i < L ? val[d + i] : 0.f;
     }
     __syncthreads();
-    smem_bitonic<P>(keys, vals);
+    smem_bitonic<P>(keys, vals, pe);
     for (int i = threadIdx.x; i < L; i += blockDim.x) {
       col[d + i] = (int32_t)(keys[i] >> 32);
       val[d + i] = vals[i];
@@ -541,7 +555,7 @@ __global__ void k_big_chunk_sort(const int64_t* boff, int64_t nb, uint64_t* K, f
     vals[i] = i < m ? V[o + c0 + i] : 0.f;
   }
   __syncthreads();
-  smem_bitonic<BIG_CHUNK>(keys, vals);
+  smem_bitonic<BIG_CHUNK>(keys, vals, BIG_CHUNK);
   for (int i = threadIdx.x; i < m; i += blockDim.x) {
     K[o + c0 + i] = keys[i];
     V[o + c0 + i] = vals[i];
@@ -746,6 +760,8 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   OT* rp = dalloc<OT>(nr + 1);
   p->d_rp = rp;
   k_local_rp<OT><<<grid_for(nr + 1), TPB, 0, s>>>(rpB, p->row_begin, nr, rp);
+  p->d_srcA = dalloc<int64_t>(nr);
+  if (n) k_srcA<AT><<<grid_for(n), TPB, 0, s>>>(rpA, p->d_perm, n, p->row_begin, p->row_end, p->d_srcA);
   SPMV_LAUNCH_CHECK();
 
   // hot prefix H over the full B
@@ -881,13 +897,13 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
   const int64_t nr = p->nrows;
   if (nr) {
     k_relabel_sort_short<AT, OT><<<grid_for((nr + 1) / 2 * 32), 256, 0, s>>>(
-        rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, nr, rp, p->d_col, p->d_val);
+        rpA, p->A_col, p->A_val, p->d_perm, p->d_srcA, nr, rp, p->d_col, p->d_val);
     if (ps->n1 + ps->n2 + ps->n3 + ps->nbig)  // rows with L > 32 exist
       k_relabel_warp<AT, OT><<<grid_for(nr * 32), TPB, 0, s>>>(
-          rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, nr, rp, p->d_col, p->d_val);
+          rpA, p->A_col, p->A_val, p->d_perm, p->d_srcA, nr, rp, p->d_col, p->d_val);
     if (ps->nlong)
       k_relabel_cta<AT, OT><<<(unsigned)std::min<int64_t>(ps->nlong, 148 * 8), 512, 0, s>>>(
-          rpA, p->A_col, p->A_val, p->d_perm, p->d_inv, p->row_begin, ps->longrows, ps->nlong,
+          rpA, p->A_col, p->A_val, p->d_perm, p->d_srcA, ps->longrows, ps->nlong,
           rp, p->d_col, p->d_val);
     SPMV_LAUNCH_CHECK();
     if (ps->n1) {
@@ -1094,7 +1110,7 @@ void plan_free(spmv_plan_s* p) {
   coo_free(p);
   dfree(p->s1); dfree(p->s2); dfree(p->s3); dfree(p->big); dfree(p->boff);
   dfree(p->longrows);
-  dfree(p->d_perm); dfree(p->d_inv);
+  dfree(p->d_perm); dfree(p->d_inv); dfree(p->d_srcA);
   if (p->d_rp) { cudaFree(p->d_rp); p->d_rp = nullptr; }
   dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows); dfree(p->d_desc);
   dfree(p->d_warp_rows); dfree(p->d_warp_ss); dfree(p->d_mid_rows); dfree(p->d_mid_ss);

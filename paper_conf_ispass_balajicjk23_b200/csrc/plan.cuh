@@ -30,6 +30,7 @@ struct spmv_plan_s {
   // owned: permutation
   int32_t* d_perm = nullptr;  // perm[old] = new (identity if none given)
   int32_t* d_inv = nullptr;   // inv[new] = old
+  int64_t* d_srcA = nullptr;  // [nrows] start in A of each local row of B
 
   // partition
   int world = 1, rank = 0;

@@ -795,9 +795,11 @@ Rabbit rabbit_detect_par(const Sym& S, bool want_log) {
         if (tot[order[i]].load(std::memory_order_relaxed) != MERGED) top[o++] = (int32_t)order[i];
     }
   }
+  phase("par:top", tp);
 #pragma omp parallel for schedule(dynamic, 65536)
   for (int64_t v = 0; v < n; ++v) std::vector<Edge>().swap(agg[v]);
   std::vector<std::vector<Edge>>().swap(agg);
+  phase("par:free", tp);
   dendrogram_ids(top, first_child, next_sib, R, n);
   phase("par:dfs", tp);
   return R;
