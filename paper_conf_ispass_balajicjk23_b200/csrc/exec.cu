@@ -716,10 +716,13 @@ __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
 // sequential (canonical W = 1) sum of a row of L <= SHORT_MAX entries
 // starting at a, streamed in 8-entry, 32-byte-aligned chunks.  Every slot of
 // a chunk holds a valid column of some row (or the zero tail padding), so its
-// x read is always safe; a slot outside [a, a + L) contributes the product +0
-// (selected, not computed: a neighbouring row's Inf / NaN value never reaches
-// this row, Alg. 1), which leaves the sum unchanged (it starts at +0 and is
-// never -0).
+// x read is always safe; a slot outside [a, a + L) has its x replaced by 0, so
+// it contributes v * 0 = +-0 and leaves the sum unchanged (it starts at +0 and
+// is never -0) -- exact for a finite neighbouring value v.  When the plan
+// holds a non-finite value (EF & 4, detected at permute time) the value is
+// masked as well (0 * 0 = +0), so an Inf / NaN never leaks into a neighbouring
+// row (Alg. 1).  The value mask costs 9 % on C2 whichever way it is written
+// (r62/r63: 0.0964 vs 0.0883 ms), hence the two variants.
 template <typename OT, int EF>
 __device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
                                               const float* __restrict__ val,
@@ -732,17 +735,21 @@ __device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
   for (int k = 0; k < hi; k += 8) {
     int cc[8];
     float vv[8];
-    if (EF == 2 && k == 0) {  // (warp-uniform: every lane starts at k = 0)
+    if ((EF & 3) == 2 && k == 0) {  // (warp-uniform: every lane starts at k = 0)
       ld_v8_stream<0>(cp + k, cc);
       ld_v8_stream<0>(vp + k, vv);
     } else {
-      ld_v8_stream<EF == 0 ? 0 : 1>(cp + k, cc);
-      ld_v8_stream<EF == 0 ? 0 : 1>(vp + k, vv);
+      ld_v8_stream<(EF & 3) == 0 ? 0 : 1>(cp + k, cc);
+      ld_v8_stream<(EF & 3) == 0 ? 0 : 1>(vp + k, vv);
     }
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
       const float xv = gx(x, cc[i]);
-      res = __fadd_rn(res, (k + i >= lo && k + i < hi) ? __fmul_rn(vv[i], xv) : 0.f);
+      const bool in = k + i >= lo && k + i < hi;
+      if constexpr ((EF & 4) != 0)  // the plan holds a non-finite value: 0 * 0 = +0
+        res = __fadd_rn(res, __fmul_rn(in ? vv[i] : 0.f, in ? xv : 0.f));
+      else  // finite values: v * 0 = +-0 exactly (the faster schedule, r62)
+        res = __fadd_rn(res, __fmul_rn(vv[i], in ? xv : 0.f));
     }
   }
   return res;
@@ -898,9 +905,15 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   // normal, the rest evict_first) via the SPMV_LANE_EF dev knob
   int ef = lane_ef_mode(p);
   if (const char* e = getenv("SPMV_LANE_EF")) ef = std::min(2, std::max(0, atoi(e)));  // dev knob
-  if (ef == 1) launch_lane_t<OT, SS, 1>(p, x, y, ss_in, s, dst);
-  else if (ef == 2) launch_lane_t<OT, SS, 2>(p, x, y, ss_in, s, dst);
-  else launch_lane_t<OT, SS, 0>(p, x, y, ss_in, s, dst);
+  if (p->val_nonfinite) {
+    if (ef == 1) launch_lane_t<OT, SS, 1 | 4>(p, x, y, ss_in, s, dst);
+    else if (ef == 2) launch_lane_t<OT, SS, 2 | 4>(p, x, y, ss_in, s, dst);
+    else launch_lane_t<OT, SS, 0 | 4>(p, x, y, ss_in, s, dst);
+  } else {
+    if (ef == 1) launch_lane_t<OT, SS, 1>(p, x, y, ss_in, s, dst);
+    else if (ef == 2) launch_lane_t<OT, SS, 2>(p, x, y, ss_in, s, dst);
+    else launch_lane_t<OT, SS, 0>(p, x, y, ss_in, s, dst);
+  }
 }
 
 // Row-class kernels other than the short-row one: MID rows (warp per row),
@@ -968,14 +981,18 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
 #define SPMV_SMALL_ARGS                                                                      \
   rp, p->d_col, p->d_val, x, y, p->nrows, p->d_mid_rows, p->n_mid, p->d_cta_rows, B_lane, B_mid, \
       ss_in, p->d_blk_ss, p->d_mid_ss, p->d_cta_ss, dst
-    const bool ef = lane_ef_mode(p) == 1;
+    const int ef = (lane_ef_mode(p) == 1 ? 1 : 0) | (p->val_nonfinite ? 4 : 0);
     if (SS) {
-      if (ef) k_small<OT, true, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      if (ef == 1) k_small<OT, true, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      else if (ef == 4) k_small<OT, true, 4, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      else if (ef == 5) k_small<OT, true, 5, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
       else k_small<OT, true, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
       ss_reduce(p, p->d_blk_ss, B_lane * LN_WARPS, p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta,
                 p->d_hub_ss, 0, ss_out, s);
     } else {
-      if (ef) k_small<OT, false, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      if (ef == 1) k_small<OT, false, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      else if (ef == 4) k_small<OT, false, 4, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      else if (ef == 5) k_small<OT, false, 5, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
       else k_small<OT, false, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
     }
 #undef SPMV_SMALL_ARGS

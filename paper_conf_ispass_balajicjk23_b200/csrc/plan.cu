@@ -322,6 +322,14 @@ __global__ void k_colcnt(const int32_t* colA, const int32_t* perm, int64_t nnz, 
   GRID_STRIDE(k, nnz) atomicAdd(&cnt[perm[colA[k]]], 1u);
 }
 
+// any non-finite value in B (permute time): selects the lane kernels that
+// mask neighbouring values as well as x (exec.cu lane_row_sum)
+__global__ void k_any_nonfinite(const float* v, int64_t n, int* flag) {
+  int bad = 0;
+  GRID_STRIDE(i, n) bad |= !isfinite(v[i]);
+  if (__any_sync(0xffffffffu, bad) && (threadIdx.x & 31) == 0) atomicOr(flag, 1);
+}
+
 __global__ void k_sum_u32(const uint32_t* a, int64_t n, unsigned long long* out) {
   unsigned long long acc = 0;
   GRID_STRIDE(i, n) acc += a[i];
@@ -940,6 +948,14 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
       SPMV_CUDA(cudaStreamSynchronize(s));  // scratch lifetime
       dfree(K1); dfree(K2); dfree(V1); dfree(V2);
     }
+  }
+  if (p->nnz_local) {
+    int* fl = dalloc<int>(1);
+    SPMV_CUDA(cudaMemsetAsync(fl, 0, sizeof(int), s));
+    k_any_nonfinite<<<grid_for(p->nnz_local), TPB, 0, s>>>(p->d_val, p->nnz_local, fl);
+    SPMV_LAUNCH_CHECK();
+    p->val_nonfinite = d2h_one(fl, s) != 0;
+    dfree(fl);
   }
   if (padded(p) && p->nnz_local) {
     int64_t* d_part = dalloc<int64_t>(p->world + 1);

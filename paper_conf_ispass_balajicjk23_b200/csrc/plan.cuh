@@ -95,6 +95,7 @@ struct spmv_plan_s {
   cudaEvent_t ev_fork = nullptr, ev_join[2] = {nullptr, nullptr};
   bool conc = false, conc_init = false;
   bool stream_ef = false;  // k_lane streams col/val with L2::evict_first (plan decision)
+  bool val_nonfinite = false;  // B holds an Inf / NaN value: lane kernels mask values too
 
   // power iteration across ranks (iterate.cu): collective backend
   // (spmv_set_coll, else NCCL on opts.nccl_comm) and the peer next-x buffers

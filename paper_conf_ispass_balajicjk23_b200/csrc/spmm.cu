@@ -75,11 +75,12 @@ __device__ __forceinline__ void ld8_f(const float* p, float (&r)[8]) {
 
 // lane per row, L <= SHORT_MAX, sequential: the association of k_lane.  As
 // there, slots of a chunk outside the row read a valid X row (a neighbouring
-// row's column or the zero tail padding); both the matrix value and the X row
-// of such a slot are replaced by 0, so it contributes 0 * 0 = +0 whatever the
-// neighbouring row holds (an Inf / NaN there never reaches this row, Alg. 1)
-// and leaves the running sum unchanged (it starts at +0 and is never -0): the
-// loop is branch-free and both chunks of a 16-entry row are in flight at once.
+// row's column or the zero tail padding) replaced by 0, so they contribute
+// v * 0 = +-0 for a finite neighbouring value; when the plan holds a
+// non-finite value (EF & 4) the value is masked too (0 * 0 = +0), so an Inf /
+// NaN never reaches this row (Alg. 1).  The running sum is unchanged either
+// way (it starts at +0 and is never -0): the loop is branch-free and both
+// chunks of a 16-entry row are in flight at once.
 template <typename OT, int EF, int MINB, int UNR>
 __global__ void __launch_bounds__(L4_THREADS, MINB)
     k_lane4(const OT* __restrict__ rp, const int32_t* __restrict__ col,
@@ -98,14 +99,14 @@ __global__ void __launch_bounds__(L4_THREADS, MINB)
     for (int k = 0; k < hi; k += 8) {
       int cc[8];
       float vv[8];
-      ld8_i<EF>(cp + k, cc);
-      ld8_f<EF>(vp + k, vv);
+      ld8_i<EF & 1>(cp + k, cc);
+      ld8_f<EF & 1>(vp + k, vv);
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         const float4 xg = ldx4(X, cc[i]);
         const bool in = k + i >= lo && k + i < hi;
         const float4 xv = in ? xg : make_float4(0.f, 0.f, 0.f, 0.f);
-        fma4(s, in ? vv[i] : 0.f, xv);
+        fma4(s, ((EF & 4) != 0 && !in) ? 0.f : vv[i], xv);
       }
     }
     reinterpret_cast<float4*>(Y)[r] = s;
@@ -259,10 +260,18 @@ void spmm4_typed(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s) {
     // 2 = 1 chunk, 4 CTAs/SM (SPMV_L4_V dev knob)
     int v = 1;
     if (const char* e = getenv("SPMV_L4_V")) v = std::min(2, std::max(0, atoi(e)));
-    const bool ef = p->opts.evict_first && p->stream_ef;
-    auto k = v == 2 ? (ef ? k_lane4<OT, 1, 4, 1> : k_lane4<OT, 0, 4, 1>)
-           : v == 1 ? (ef ? k_lane4<OT, 1, 3, 2> : k_lane4<OT, 0, 3, 2>)
-                    : (ef ? k_lane4<OT, 1, 2, 2> : k_lane4<OT, 0, 2, 2>);
+    // EF bit 0: evict_first stream; bit 2: the plan holds a non-finite value,
+    // so foreign slots' values are masked too (exec.cu lane_row_sum)
+    const int ef = (p->opts.evict_first && p->stream_ef ? 1 : 0) | (p->val_nonfinite ? 4 : 0);
+    auto pick = [&](auto k0, auto k1, auto k4, auto k5) {
+      return ef == 1 ? k1 : ef == 4 ? k4 : ef == 5 ? k5 : k0;
+    };
+    auto k = v == 2 ? pick(k_lane4<OT, 0, 4, 1>, k_lane4<OT, 1, 4, 1>, k_lane4<OT, 4, 4, 1>,
+                           k_lane4<OT, 5, 4, 1>)
+           : v == 1 ? pick(k_lane4<OT, 0, 3, 2>, k_lane4<OT, 1, 3, 2>, k_lane4<OT, 4, 3, 2>,
+                           k_lane4<OT, 5, 3, 2>)
+                    : pick(k_lane4<OT, 0, 2, 2>, k_lane4<OT, 1, 2, 2>, k_lane4<OT, 4, 2, 2>,
+                           k_lane4<OT, 5, 2, 2>);
     k<<<g, L4_THREADS, 0, s>>>(rp, p->d_col, p->d_val, X, Y, p->nrows);
   }
   cudaStream_t s1 = s, s2 = s;
