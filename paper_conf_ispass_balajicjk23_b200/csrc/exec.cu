@@ -431,14 +431,11 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 // every lane.  UNR strided entries in flight per lane, the ragged end
 // guarded: a slot past the row adds +0, which leaves s unchanged (s starts at
 // +0 and is never -0), so the association is exactly j, j+32, j+64, ...
-template <typename OT, int SM, int UNR = 4>
-__device__ __forceinline__ float warp_row_sum(const OT* __restrict__ rp,
-                                              const int32_t* __restrict__ col,
-                                              const float* __restrict__ val,
-                                              const float* __restrict__ x, int r, int lane,
-                                              uint64_t pol) {
-  const int64_t b = (int64_t)rp[r];
-  const int L = (int)((int64_t)rp[r + 1] - b);
+template <int SM, int UNR = 4>
+__device__ __forceinline__ float warp_row_sum_bl(const int32_t* __restrict__ col,
+                                                 const float* __restrict__ val,
+                                                 const float* __restrict__ x, int64_t b, int L,
+                                                 int lane, uint64_t pol) {
   const int32_t* cc = col + b;
   const float* vv = val + b;
   float s = 0.f;
@@ -459,6 +456,16 @@ __device__ __forceinline__ float warp_row_sum(const OT* __restrict__ rp,
   return warp_tree(s);
 }
 
+template <typename OT, int SM, int UNR = 4>
+__device__ __forceinline__ float warp_row_sum(const OT* __restrict__ rp,
+                                              const int32_t* __restrict__ col,
+                                              const float* __restrict__ val,
+                                              const float* __restrict__ x, int r, int lane,
+                                              uint64_t pol) {
+  const int64_t b = (int64_t)rp[r];
+  return warp_row_sum_bl<SM, UNR>(col, val, x, b, (int)((int64_t)rp[r + 1] - b), lane, pol);
+}
+
 template <typename OT, bool SS, int SM, int UNR = 4>
 __global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
@@ -469,9 +476,26 @@ __global__ void __launch_bounds__(256)
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float alpha = alpha_of(ss_in);
   const uint64_t pol = stream_policy<SM>();
-  for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < nrows; q += W) {
-    const int r = rows[q];
-    const float s = warp_row_sum<OT, SM, UNR>(rp, col, val, x, r, lane, pol);
+  // the next row's id and extent are loaded one iteration ahead, so its
+  // rows[] -> row_ptr chain overlaps the current row's gathers
+  int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  int rn = 0;
+  int64_t bn = 0, en = 0;
+  if (q < nrows) {
+    rn = rows[q];
+    bn = (int64_t)rp[rn];
+    en = (int64_t)rp[rn + 1];
+  }
+  for (; q < nrows; q += W) {
+    const int r = rn;
+    const int64_t b = bn;
+    const int L = (int)(en - bn);
+    if (q + W < nrows) {
+      rn = rows[q + W];
+      bn = (int64_t)rp[rn];
+      en = (int64_t)rp[rn + 1];
+    }
+    const float s = warp_row_sum_bl<SM, UNR>(col, val, x, b, L, lane, pol);
     if (lane == 0) {
       const float v = __fmul_rn(s, alpha);
       store_y<SS>(y, dst, r, v);
