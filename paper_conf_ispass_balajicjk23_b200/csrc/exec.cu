@@ -476,26 +476,9 @@ __global__ void __launch_bounds__(256)
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float alpha = alpha_of(ss_in);
   const uint64_t pol = stream_policy<SM>();
-  // the next row's id and extent are loaded one iteration ahead, so its
-  // rows[] -> row_ptr chain overlaps the current row's gathers
-  int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  int rn = 0;
-  int64_t bn = 0, en = 0;
-  if (q < nrows) {
-    rn = rows[q];
-    bn = (int64_t)rp[rn];
-    en = (int64_t)rp[rn + 1];
-  }
-  for (; q < nrows; q += W) {
-    const int r = rn;
-    const int64_t b = bn;
-    const int L = (int)(en - bn);
-    if (q + W < nrows) {
-      rn = rows[q + W];
-      bn = (int64_t)rp[rn];
-      en = (int64_t)rp[rn + 1];
-    }
-    const float s = warp_row_sum_bl<SM, UNR>(col, val, x, b, L, lane, pol);
+  for (int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; q < nrows; q += W) {
+    const int r = rows[q];
+    const float s = warp_row_sum<OT, SM, UNR>(rp, col, val, x, r, lane, pol);
     if (lane == 0) {
       const float v = __fmul_rn(s, alpha);
       store_y<SS>(y, dst, r, v);

@@ -119,6 +119,17 @@ e1.record()
 torch.cuda.synchronize()
 warm_ms = e0.elapsed_time(e1) / a.steps
 it_ms = None
+sc_ms = None
+if a.iterate:  # exec_scaled back to back with FIXED x / y (the norm's cost without alternation)
+    ss = torch.zeros(2, dtype=torch.float64, device=dev)
+    P.exec_scaled(xB, y, None, ss[:1])
+    e0, e1 = ev(), ev()
+    e0.record()
+    for _ in range(a.steps):
+        P.exec_scaled(xB, y, ss[:1], ss[1:])
+    e1.record()
+    torch.cuda.synchronize()
+    sc_ms = e0.elapsed_time(e1) / a.steps
 if a.iterate:
     xs = xB.clone()
     P.iterate(xs, 3)
@@ -132,7 +143,7 @@ h = hashlib.sha1(y.cpu().numpy().tobytes()).hexdigest()[:16]
 hbm = json.load(open("MEASURED_PEAKS.json"))["hbm_gbs"] if os.path.exists("MEASURED_PEAKS.json") else 6548.8
 print(json.dumps({"workload": name, "ordering": a.ordering, "env": a.env + (["no-reset"] if a.no_reset else []),
                   "n": n, "nnz": nnz,
-                  "cold_ms": round(cold_ms, 4), "warm_ms": round(warm_ms, 4), "iterate_ms": it_ms,
+                  "cold_ms": round(cold_ms, 4), "warm_ms": round(warm_ms, 4), "iterate_ms": it_ms, "scaled_fixed_ms": sc_ms,
                   "x_ideal_cold": round(cold_ms * 1e-3 * hbm * 1e9 / ideal, 3),
                   "gen_s": round(gen_s, 2), "reorder_s": round(reorder_s, 1),
                   "mid_rows": info["n_mid_rows"], "cta_rows": info["n_cta_rows"],
