@@ -774,8 +774,11 @@ __device__ __forceinline__ void warp_ss(double ssacc, double* out) {
 // minBlocksPerSM = 1 lets ptxas keep both chunks and all 16 gathers of a
 // 16-entry row in flight per lane (64 registers, 4 CTAs/SM); capping registers
 // for more CTAs measured 20-40 % slower
+// SS (the power-iteration step) needs 72 registers unbounded, which drops to
+// 3 CTAs per SM and costs 22 % (r66: 4.45 vs 3.64 ms on C5): both variants
+// are held to 64 registers, 4 CTAs per SM
 template <typename OT, bool SS, int EF>
-__global__ void __launch_bounds__(LN_THREADS, 1)
+__global__ void __launch_bounds__(LN_THREADS, SS ? 4 : 1)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
            int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss,
@@ -1076,6 +1079,9 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
     cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, p->device);
     if (l2 > 0) bytes = std::min<int64_t>(bytes, (int64_t)(frac * l2));
   }
+  // spmv_iterate reads x from two buffers in turn: both windows must fit the
+  // persisting carve-out at once, or each step evicts the other's lines
+  if (p->win_alternating) bytes = std::min<int64_t>(bytes, (int64_t)maxpers / 2);
   if (const char* e = getenv("SPMV_WIN_HIT")) hit = std::min(1.0, std::max(0.0, atof(e)));  // dev knob
   if (bytes <= 0) return;
   size_t cur = 0;

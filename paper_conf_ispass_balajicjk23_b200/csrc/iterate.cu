@@ -213,6 +213,11 @@ void iterate(spmv_plan_s* p, float* x, int iters, double* lambda, cudaStream_t s
   }
   const double* sin = nullptr;
   int cur = 0;
+  struct Alt {  // window sizing for two alternating x buffers, for this call only
+    spmv_plan_s* p;
+    explicit Alt(spmv_plan_s* q) : p(q) { p->win_alternating = true; p->win_ptr = nullptr; }
+    ~Alt() { p->win_alternating = false; p->win_ptr = nullptr; }
+  } alt_(p);
   for (int t = 0; t < iters; ++t) {
     double* sout = p->d_ss + (t & 1);
     if (peer) {

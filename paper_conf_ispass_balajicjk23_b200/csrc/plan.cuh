@@ -107,6 +107,7 @@ struct spmv_plan_s {
   // state
   bool permuted = false;
   int64_t l2_window_bytes = 0;
+  bool win_alternating = false;  // set by spmv_iterate: x alternates between two buffers
   bool l2_limit_raised = false;   // cudaLimitPersistingL2CacheSize raised by set_window
   size_t l2_limit_before = 0;
   const void* win_ptr = nullptr;
