@@ -319,6 +319,9 @@ spmv_status spmv_plan_info(spmv_plan_t p, spmv_plan_info_t* info) {
   info->exec_launches = spmv::exec_launches(p, false);
   info->spmm4_launches = spmv::spmm4_launches(p);
   info->hot_prefix_nnz = p->H_nnz;
+  info->lane_nnz = p->lane_nnz;
+  info->lane_waste_slots = p->lane_waste;
+  info->lane_pred_gather = spmv::lane_pred_mode(p);
   API_END
 }
 

@@ -427,33 +427,83 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 }
 
 // ------------------------------------------------------------- long rows
+#ifndef SPMV_WARP_PIPE  // A/B build knobs of the warp-per-row sum
+#define SPMV_WARP_PIPE 1
+#endif
+#ifndef SPMV_WARP_MINB
+#define SPMV_WARP_MINB 8
+#endif
+// Strided partial sum of the entries t0, t0 + S, t0 + 2S, ... < L of a row
+// (S = 32: a lane of the warp-per-row sum; S = 256: a thread of the CTA sum),
+// UNR entries in flight, software-pipelined: the col / val of the next UNR
+// entries are loaded before the x gathers of the current ones are consumed, so
+// an iteration costs one memory round trip (the gathers), not two (stream,
+// then gather).  The ragged end is guarded: a slot past the row has v = x = 0
+// and adds +0, which leaves s unchanged (s starts at +0 and is never -0), so
+// the association is exactly t0, t0 + S, t0 + 2S, ... for every UNR.
+template <int SM, int S, int UNR, bool PIPE = true>
+__device__ __forceinline__ float strided_sum(const int32_t* __restrict__ cc,
+                                             const float* __restrict__ vv,
+                                             const float* __restrict__ x, int64_t t0, int64_t L,
+                                             uint64_t pol) {
+  float s = 0.f;
+  if constexpr (!PIPE) {  // stream, then gather, per iteration (same association)
+    for (int64_t t = t0; t < L; t += S * UNR) {
+      int c[UNR];
+      float v[UNR], xv[UNR];
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) {
+        const bool pu = t + S * u < L;
+        c[u] = pu ? lds<SM>(cc + t + S * u, pol) : 0;
+        v[u] = pu ? lds<SM>(vv + t + S * u, pol) : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) xv[u] = (t + S * u < L) ? gx(x, c[u]) : 0.f;
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
+    }
+    return s;
+  }
+  int c[UNR];
+  float v[UNR];
+#pragma unroll
+  for (int u = 0; u < UNR; ++u) {
+    const bool pu = t0 + S * u < L;
+    c[u] = pu ? lds<SM>(cc + t0 + S * u, pol) : 0;
+    v[u] = pu ? lds<SM>(vv + t0 + S * u, pol) : 0.f;
+  }
+  for (int64_t t = t0; t < L; t += S * UNR) {
+    float xv[UNR];
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) xv[u] = (t + S * u < L) ? gx(x, c[u]) : 0.f;
+    const int64_t tn = t + S * UNR;
+    int cn[UNR];
+    float vn[UNR];
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) {
+      const bool pu = tn + S * u < L;
+      cn[u] = pu ? lds<SM>(cc + tn + S * u, pol) : 0;
+      vn[u] = pu ? lds<SM>(vv + tn + S * u, pol) : 0.f;
+    }
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
+#pragma unroll
+    for (int u = 0; u < UNR; ++u) {
+      c[u] = cn[u];
+      v[u] = vn[u];
+    }
+  }
+  return s;
+}
+
 // canonical W = 32 sum of row r (32 strided partials + xor tree), valid in
-// every lane.  UNR strided entries in flight per lane, the ragged end
-// guarded: a slot past the row adds +0, which leaves s unchanged (s starts at
-// +0 and is never -0), so the association is exactly j, j+32, j+64, ...
+// every lane
 template <int SM, int UNR = 4>
 __device__ __forceinline__ float warp_row_sum_bl(const int32_t* __restrict__ col,
                                                  const float* __restrict__ val,
                                                  const float* __restrict__ x, int64_t b, int L,
                                                  int lane, uint64_t pol) {
-  const int32_t* cc = col + b;
-  const float* vv = val + b;
-  float s = 0.f;
-  for (int j = lane; j < L; j += 32 * UNR) {
-    int c[UNR];
-    float v[UNR], xv[UNR];
-#pragma unroll
-    for (int u = 0; u < UNR; ++u) {
-      const bool pu = j + 32 * u < L;
-      c[u] = pu ? lds<SM>(cc + j + 32 * u, pol) : 0;
-      v[u] = pu ? lds<SM>(vv + j + 32 * u, pol) : 0.f;
-    }
-#pragma unroll
-    for (int u = 0; u < UNR; ++u) xv[u] = (j + 32 * u < L) ? gx(x, c[u]) : 0.f;
-#pragma unroll
-    for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
-  }
-  return warp_tree(s);
+  return warp_tree(strided_sum<SM, 32, UNR, SPMV_WARP_PIPE>(col + b, val + b, x, lane, L, pol));
 }
 
 template <typename OT, int SM, int UNR = 4>
@@ -466,8 +516,10 @@ __device__ __forceinline__ float warp_row_sum(const OT* __restrict__ rp,
   return warp_row_sum_bl<SM, UNR>(col, val, x, b, (int)((int64_t)rp[r + 1] - b), lane, pol);
 }
 
+// 8 CTAs (64 warps) per SM: held to 32 registers (the SS / int64 variant took
+// 34, which the 8-register allocation granularity rounds to 6 CTAs per SM)
 template <typename OT, bool SS, int SM, int UNR = 4>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(256, SPMV_WARP_MINB)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
                 float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
@@ -496,22 +548,7 @@ __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             float* red) {
   const int tid = threadIdx.x;
   const uint64_t pol = stream_policy<SM>();
-  float s = 0.f;
-  // UNR strided entries in flight, ragged end guarded (+0 slots, as k_warp_rows)
-  for (int64_t t = tid; t < L; t += 256 * UNR) {
-    int c[UNR];
-    float v[UNR], xv[UNR];
-#pragma unroll
-    for (int u = 0; u < UNR; ++u) {
-      const bool pu = t + 256 * u < L;
-      c[u] = pu ? lds<SM>(col + b + t + 256 * u, pol) : 0;
-      v[u] = pu ? lds<SM>(val + b + t + 256 * u, pol) : 0.f;
-    }
-#pragma unroll
-    for (int u = 0; u < UNR; ++u) xv[u] = (t + 256 * u < L) ? gx(x, c[u]) : 0.f;
-#pragma unroll
-    for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
-  }
+  const float s = strided_sum<SM, 256, UNR>(col + b, val + b, x, tid, L, pol);
   red[tid] = s;
   __syncthreads();
 #pragma unroll
@@ -679,6 +716,9 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 // Design note (profiles/r01_summary.md, r26): a persistent variant with a
 // sliding shared-memory x window, one barrier per block and evict_first
 // stream hints ran 1.25x slower than this plain form on SBM 4M/64M.
+#ifndef SPMV_SMALL_UNR  // A/B: entries in flight per thread in k_small's MID / CTA rows
+#define SPMV_SMALL_UNR 4
+#endif
 constexpr int LN_THREADS = 256;
 constexpr int MID_STREAM_DEFAULT = 0;  // stream-load mode of the MID / CTA / hub kernels (lds)
 constexpr int LN_WARPS = LN_THREADS / 32;
@@ -729,7 +769,9 @@ __device__ __forceinline__ void ld_v8_stream(const float* p, float (&r)[8]) {
 // holds a non-finite value (EF & 4, detected at permute time) the value is
 // masked as well (0 * 0 = +0), so an Inf / NaN never leaks into a neighbouring
 // row (Alg. 1).  The value mask costs 9 % on C2 whichever way it is written
-// (r62/r63: 0.0964 vs 0.0883 ms), hence the two variants.
+// (r62/r63: 0.0964 vs 0.0883 ms), hence the two variants.  EF & 8 (plan
+// decision, lane_pred): the x of a foreign slot is not gathered at all -- the
+// same sum, fewer L1 wavefronts where rows straddle chunks (stencil).
 template <typename OT, int EF>
 __device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
                                               const float* __restrict__ val,
@@ -751,8 +793,12 @@ __device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
     }
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
-      const float xv = gx(x, cc[i]);
       const bool in = k + i >= lo && k + i < hi;
+      float xv;
+      if constexpr ((EF & 8) != 0)  // plan decision: no gather for a foreign slot
+        xv = in ? gx(x, cc[i]) : 0.f;
+      else  // branch-free: every slot gathered (valid column), foreign ones zeroed
+        xv = gx(x, cc[i]);
       if constexpr ((EF & 4) != 0)  // the plan holds a non-finite value: 0 * 0 = +0
         res = __fadd_rn(res, __fmul_rn(in ? vv[i] : 0.f, in ? xv : 0.f));
       else  // finite values: v * 0 = +-0 exactly (the faster schedule, r62)
@@ -864,7 +910,7 @@ __global__ void __launch_bounds__(LN_THREADS)
     const int64_t q = (blk - B_lane) * 8 + warp;
     if (q < n_mid) {
       const int r = mid_rows[q];
-      const float s = warp_row_sum<OT, SM>(rp, col, val, x, r, lane, stream_policy<SM>());
+      const float s = warp_row_sum<OT, SM, SPMV_SMALL_UNR>(rp, col, val, x, r, lane, stream_policy<SM>());
       if (lane == 0) {
         const float v = __fmul_rn(s, alpha);
         store_y<SS>(y, dst, r, v);
@@ -875,7 +921,7 @@ __global__ void __launch_bounds__(LN_THREADS)
     const int64_t i = blk - B_lane - B_mid;
     const int r = cta_rows[i];
     const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
-    const float s = cta_sum256<SM>(col, val, x, b, L, red);
+    const float s = cta_sum256<SM, SPMV_SMALL_UNR>(col, val, x, b, L, red);
     if (tid == 0) {
       const float v = __fmul_rn(s, alpha);
       store_y<SS>(y, dst, r, v);
@@ -905,6 +951,11 @@ int lane_ef_mode(const spmv_plan_s* p) {
   return p->opts.evict_first && p->stream_ef ? 1 : 0;
 }
 
+int lane_pred_mode(const spmv_plan_s* p) {
+  if (const char* e = getenv("SPMV_LANE_PRED")) return atoi(e) != 0;  // dev knob (A/B)
+  return p->lane_pred ? 1 : 0;
+}
+
 namespace {
 
 template <typename OT, bool SS>
@@ -915,15 +966,18 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
   // normal, the rest evict_first) via the SPMV_LANE_EF dev knob
   int ef = lane_ef_mode(p);
   if (const char* e = getenv("SPMV_LANE_EF")) ef = std::min(2, std::max(0, atoi(e)));  // dev knob
-  if (p->val_nonfinite) {
-    if (ef == 1) launch_lane_t<OT, SS, 1 | 4>(p, x, y, ss_in, s, dst);
-    else if (ef == 2) launch_lane_t<OT, SS, 2 | 4>(p, x, y, ss_in, s, dst);
-    else launch_lane_t<OT, SS, 0 | 4>(p, x, y, ss_in, s, dst);
-  } else {
-    if (ef == 1) launch_lane_t<OT, SS, 1>(p, x, y, ss_in, s, dst);
-    else if (ef == 2) launch_lane_t<OT, SS, 2>(p, x, y, ss_in, s, dst);
-    else launch_lane_t<OT, SS, 0>(p, x, y, ss_in, s, dst);
-  }
+  const int m = (p->val_nonfinite ? 4 : 0) | (lane_pred_mode(p) ? 8 : 0);
+#define SPMV_LANE_M(M)                                                        \
+  do {                                                                        \
+    if (ef == 1) launch_lane_t<OT, SS, 1 | (M)>(p, x, y, ss_in, s, dst);      \
+    else if (ef == 2) launch_lane_t<OT, SS, 2 | (M)>(p, x, y, ss_in, s, dst); \
+    else launch_lane_t<OT, SS, 0 | (M)>(p, x, y, ss_in, s, dst);              \
+  } while (0)
+  if (m == 12) SPMV_LANE_M(12);
+  else if (m == 8) SPMV_LANE_M(8);
+  else if (m == 4) SPMV_LANE_M(4);
+  else SPMV_LANE_M(0);
+#undef SPMV_LANE_M
 }
 
 // Row-class kernels other than the short-row one: MID rows (warp per row),
@@ -991,20 +1045,29 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
 #define SPMV_SMALL_ARGS                                                                      \
   rp, p->d_col, p->d_val, x, y, p->nrows, p->d_mid_rows, p->n_mid, p->d_cta_rows, B_lane, B_mid, \
       ss_in, p->d_blk_ss, p->d_mid_ss, p->d_cta_ss, dst
-    const int ef = (lane_ef_mode(p) == 1 ? 1 : 0) | (p->val_nonfinite ? 4 : 0);
+    const int ef = (lane_ef_mode(p) == 1 ? 1 : 0) | (p->val_nonfinite ? 4 : 0) |
+                   (lane_pred_mode(p) ? 8 : 0);
+#define SPMV_SMALL_EF(SSV)                                                                 \
+  do {                                                                                     \
+    switch (ef) {                                                                          \
+      case 1: k_small<OT, SSV, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS); break;   \
+      case 4: k_small<OT, SSV, 4, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS); break;   \
+      case 5: k_small<OT, SSV, 5, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS); break;   \
+      case 8: k_small<OT, SSV, 8, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS); break;   \
+      case 9: k_small<OT, SSV, 9, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS); break;   \
+      case 12: k_small<OT, SSV, 12, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS); break; \
+      case 13: k_small<OT, SSV, 13, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS); break; \
+      default: k_small<OT, SSV, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);         \
+    }                                                                                      \
+  } while (0)
     if (SS) {
-      if (ef == 1) k_small<OT, true, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
-      else if (ef == 4) k_small<OT, true, 4, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
-      else if (ef == 5) k_small<OT, true, 5, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
-      else k_small<OT, true, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      SPMV_SMALL_EF(true);
       ss_reduce(p, p->d_blk_ss, B_lane * LN_WARPS, p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta,
                 p->d_hub_ss, 0, ss_out, s);
     } else {
-      if (ef == 1) k_small<OT, false, 1, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
-      else if (ef == 4) k_small<OT, false, 4, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
-      else if (ef == 5) k_small<OT, false, 5, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
-      else k_small<OT, false, 0, SM><<<g, LN_THREADS, 0, s>>>(SPMV_SMALL_ARGS);
+      SPMV_SMALL_EF(false);
     }
+#undef SPMV_SMALL_EF
 #undef SPMV_SMALL_ARGS
     SPMV_LAUNCH_CHECK();
     return;

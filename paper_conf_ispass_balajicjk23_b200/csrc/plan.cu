@@ -248,25 +248,35 @@ __global__ void k_tile_desc(const OT* rp, const int32_t* tiles, int64_t K, TileD
   }
 }
 
-// short rows (1 <= L <= SHORT_MAX) and those whose first or last 8-entry
-// chunk is shared with a neighbouring row (start or end not a multiple of 8)
+// short rows (1 <= L <= SHORT_MAX), those whose first or last 8-entry chunk
+// is shared with a neighbouring row (start or end not a multiple of 8), their
+// entries, and the chunk slots outside the row that k_lane reads in rows
+// spanning >= 2 chunks (a lane gathers every slot of a chunk; slots of a
+// neighbour read at another iteration are not merged with the owner's gather)
 template <typename OT>
 __global__ void k_chunk_share(const OT* rp, int64_t nrows, unsigned long long* cnt) {
-  unsigned long long sh = 0, all = 0;
+  unsigned long long sh = 0, all = 0, ent = 0, waste = 0;
   GRID_STRIDE(r, nrows) {
     const int64_t a = (int64_t)rp[r], e = (int64_t)rp[r + 1];
     if (e - a >= 1 && e - a <= SHORT_MAX) {
       ++all;
       sh += ((a | e) & 7) != 0;
+      ent += (unsigned long long)(e - a);
+      const int64_t ch = ((e + 7) >> 3) - (a >> 3);
+      if (ch >= 2) waste += (unsigned long long)(8 * ch - (e - a));
     }
   }
   for (int o = 16; o > 0; o >>= 1) {
     sh += __shfl_xor_sync(0xffffffffu, sh, o);
     all += __shfl_xor_sync(0xffffffffu, all, o);
+    ent += __shfl_xor_sync(0xffffffffu, ent, o);
+    waste += __shfl_xor_sync(0xffffffffu, waste, o);
   }
   if ((threadIdx.x & 31) == 0 && all) {
     atomicAdd(cnt, sh);
     atomicAdd(cnt + 1, all);
+    atomicAdd(cnt + 2, ent);
+    atomicAdd(cnt + 3, waste);
   }
 }
 
@@ -808,17 +818,25 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
 
   // stream cache policy of the short-row kernel: L2
   // evict_first only when no 8-entry chunk is read by two lanes (<= 1 % of the
-  // short rows share one), else a shared chunk evicted early is refetched
+  // short rows share one), else a shared chunk evicted early is refetched.
+  // Gather policy: k_lane gathers x only for a row's own slots when the short
+  // rows carry at least half of the entries and >= 20 % extra slot gathers
+  // would be wasted in rows spanning several chunks (27-point stencil: 28 %;
+  // r68: 5.68 vs 6.78 ms), else every slot (branch-free, cheaper when chunks
+  // are row-aligned: SBM 0.088 vs 0.0996 ms).
   {
-    unsigned long long* dc = dalloc<unsigned long long>(2);
-    SPMV_CUDA(cudaMemsetAsync(dc, 0, 16, s));
+    unsigned long long* dc = dalloc<unsigned long long>(4);
+    SPMV_CUDA(cudaMemsetAsync(dc, 0, 32, s));
     if (nr) k_chunk_share<OT><<<grid_for(nr), TPB, 0, s>>>(rp, nr, dc);
     SPMV_LAUNCH_CHECK();
-    unsigned long long hc[2] = {0, 0};
-    SPMV_CUDA(cudaMemcpyAsync(hc, dc, 16, cudaMemcpyDeviceToHost, s));
+    unsigned long long hc[4] = {0, 0, 0, 0};
+    SPMV_CUDA(cudaMemcpyAsync(hc, dc, 32, cudaMemcpyDeviceToHost, s));
     SPMV_CUDA(cudaStreamSynchronize(s));
     dfree(dc);
     p->stream_ef = hc[0] * 100 <= hc[1];
+    p->lane_nnz = (int64_t)hc[2];
+    p->lane_waste = (int64_t)hc[3];
+    p->lane_pred = p->lane_nnz > 0 && 2 * p->lane_nnz >= p->nnz_local && 5 * p->lane_waste >= p->lane_nnz;
   }
 
   // row classes + sort buckets

@@ -95,6 +95,9 @@ struct spmv_plan_s {
   cudaEvent_t ev_fork = nullptr, ev_join[2] = {nullptr, nullptr};
   bool conc = false, conc_init = false;
   bool stream_ef = false;  // k_lane streams col/val with L2::evict_first (plan decision)
+  bool lane_pred = false;  // k_lane gathers x only for a row's own slots (plan decision)
+  int64_t lane_nnz = 0;    // entries in short rows (1 <= L <= SHORT_MAX)
+  int64_t lane_waste = 0;  // foreign chunk slots k_lane reads in short rows spanning >= 2 chunks
   bool val_nonfinite = false;  // B holds an Inf / NaN value: lane kernels mask values too
 
   // power iteration across ranks (iterate.cu): collective backend
@@ -136,6 +139,7 @@ int exec_launches(const spmv_plan_s* p, bool ss);
 void exec_spmm4(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s);
 int spmm4_launches(const spmv_plan_s* p);
 int lane_ef_mode(const spmv_plan_s* p);
+int lane_pred_mode(const spmv_plan_s* p);
 void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s);
 void export_coo_rows(spmv_plan_s* p, int32_t* rows, cudaStream_t s);
 void coo_free(spmv_plan_s* p);

@@ -69,7 +69,9 @@ class _Info(ctypes.Structure):
         "hot_prefix", "ideal_bytes")] + \
         [(n, ctypes.c_int32) for n in ("offset_bytes", "world", "rank", "permuted",
                                        "l2_window_bytes", "stream_evict_first", "exec_launches", "spmm4_launches")] + \
-        [("hot_prefix_nnz", ctypes.c_int64)]
+        [("hot_prefix_nnz", ctypes.c_int64), ("lane_nnz", ctypes.c_int64),
+         ("lane_waste_slots", ctypes.c_int64), ("lane_pred_gather", ctypes.c_int32),
+         ("reserved0", ctypes.c_int32)]
 
 
 class _Stats(ctypes.Structure):

@@ -94,13 +94,14 @@ __global__ void __launch_bounds__(256) k_gather_smem(const int32_t* __restrict__
 __device__ __forceinline__ uint32_t su32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
 // 128 threads per CTA; a stage = 32 gather4 (one per lane of warp 0) = 128
-// rows of 16 B = 2 KB; NST stages in a ring.  Every thread then reads the
-// float its row needs (row r's element idx & 3).
-constexpr int NST = 8;
+// rows of 16 B; each lane's 4 rows land in its own 128-byte-aligned slot
+// (tensor copies need a 128-B aligned destination); NST stages in a ring.
+// Every thread then reads the float its row needs (row r's element idx & 3).
+constexpr int NST = 4;
 __global__ void __launch_bounds__(128) k_gather_tma4(const __grid_constant__ CUtensorMap tm,
                                                      const int32_t* __restrict__ idx, int64_t m,
                                                      float* out, int* err) {
-  __shared__ alignas(128) float4 buf[NST][128];
+  __shared__ __align__(128) float4 buf[NST][32][8];  // [stage][lane][row 0..3 used]
   __shared__ alignas(8) uint64_t full[NST];
   __shared__ alignas(8) uint64_t empty[NST];
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
@@ -131,7 +132,7 @@ __global__ void __launch_bounds__(128) k_gather_tma4(const __grid_constant__ CUt
                 r3 = __ldcs(ip + 3) >> 2;
       asm volatile(
           "cp.async.bulk.tensor.2d.shared::cluster.global.tile::gather4.mbarrier::complete_tx::bytes"
-          " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(su32(&buf[st][lane * 4])),
+          " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(su32(&buf[st][lane][0])),
           "l"(&tm), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(su32(&full[st]))
           : "memory");
     }
@@ -155,7 +156,7 @@ __global__ void __launch_bounds__(128) k_gather_tma4(const __grid_constant__ CUt
     }
     const int64_t base = (blockIdx.x + k * (int64_t)gridDim.x) * per;
     const int c = __ldcs(idx + base + tid);
-    s += reinterpret_cast<const float*>(&buf[st][tid])[c & 3];
+    s += reinterpret_cast<const float*>(&buf[st][tid >> 2][tid & 3])[c & 3];
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&empty[st])) : "memory");
     // the producer reuses stage (k + NST - 1) % NST = (k - 1) % NST: wait until it is drained
     const int64_t j = k + NST - 1;
@@ -203,7 +204,8 @@ float time_ms(F f, int reps) {
   return ms / reps;
 }
 
-int main() {
+int main(int argc, char** argv) {
+  const bool only_tma = argc > 1 && argv[1][0] == 't';
   int sms;
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
   const int64_t m = int64_t(1) << 28;           // 268 M gathers per launch
@@ -219,6 +221,7 @@ int main() {
   k_fill_x<<<sms * 8, 256>>>(x, xn);
   const int64_t ranges[] = {int64_t(1) << 22, int64_t(1) << 24, int64_t(1) << 26, xn};  // 16 MB .. 1 GB
   for (int64_t R : ranges) {
+    if (only_tma) break;
     k_fill_idx<<<sms * 8, 256>>>(idx, m, (uint64_t)R, 12345);
     CK(cudaDeviceSynchronize());
     auto rep = [&](const char* mode, int U, int cps, float ms) {
@@ -236,7 +239,7 @@ int main() {
     }
   }
   // idx-stream-only control (gather the index's own position: coalesced)
-  {
+  if (!only_tma) {
     int32_t* seq;
     CK(cudaMalloc(&seq, m * 4));
     k_fill_idx<<<sms * 8, 256>>>(seq, m, 1, 0);  // all zero -> every lane the same word
@@ -249,6 +252,7 @@ int main() {
   k_fill_idx<<<sms * 8, 256>>>(idx, m, (uint64_t)TAB, 777);
   CK(cudaFuncSetAttribute(k_gather_smem<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, TAB * 4));
   for (int cps : {1, 2}) {
+    if (only_tma) break;
     const float ms = time_ms([&] { k_gather_smem<8><<<sms * cps, 256, TAB * 4>>>(idx, m, x, out); }, 5);
     printf("{\"mode\": \"lds\", \"U\": 8, \"ctas_per_sm\": %d, \"ms\": %.3f, \"ggather_per_s\": %.1f}\n", cps, ms,
            m / ms / 1e6);

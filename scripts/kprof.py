@@ -33,7 +33,10 @@ ap.add_argument("--ncu", type=int, default=0)
 ap.add_argument("--env", nargs="*", default=[])
 ap.add_argument("--sequential-reorder", action="store_true")
 ap.add_argument("--no-reset", action="store_true", help="flush without the persisting-L2 reset")
+ap.add_argument("--so", default=None, help="load this libspmv build instead of the in-tree one (A/B)")
 a = ap.parse_args()
+if a.so:
+    spmv.SO_PATH = os.path.abspath(a.so)
 for kv in a.env:
     k, v = kv.split("=", 1)
     os.environ[k] = v
@@ -142,6 +145,7 @@ if a.iterate:
 h = hashlib.sha1(y.cpu().numpy().tobytes()).hexdigest()[:16]
 hbm = json.load(open("MEASURED_PEAKS.json"))["hbm_gbs"] if os.path.exists("MEASURED_PEAKS.json") else 6548.8
 print(json.dumps({"workload": name, "ordering": a.ordering, "env": a.env + (["no-reset"] if a.no_reset else []),
+                  "so": a.so,
                   "n": n, "nnz": nnz,
                   "cold_ms": round(cold_ms, 4), "warm_ms": round(warm_ms, 4), "iterate_ms": it_ms, "scaled_fixed_ms": sc_ms,
                   "x_ideal_cold": round(cold_ms * 1e-3 * hbm * 1e9 / ideal, 3),
@@ -149,6 +153,7 @@ print(json.dumps({"workload": name, "ordering": a.ordering, "env": a.env + (["no
                   "mid_rows": info["n_mid_rows"], "cta_rows": info["n_cta_rows"],
                   "hub_rows": info["n_hub_rows"], "H": info["hot_prefix"],
                   "win": P.info()["l2_window_bytes"], "ef": info["stream_evict_first"],
+                  "lane_pred": info.get("lane_pred_gather"), "lane_waste": info.get("lane_waste_slots"), "lane_nnz": info.get("lane_nnz"),
                   "y_sha": h,
                   "peak_rss_gb": round(resource.getrusage(resource.RUSAGE_SELF).ru_maxrss / 2**20, 1)}),
       flush=True)
