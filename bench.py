@@ -128,6 +128,24 @@ def ncu_traffic(workload: str, ordering: str):
     return e if isinstance(e, dict) else None
 
 
+GATHER_CEILING = os.path.join("profiles", "r67_gather_ceiling.jsonl")
+
+
+def gather_ceiling():
+    """Measured random 4-byte LDG gathers per second on this GPU type, x range
+    L2-resident (scripts/gather_ceiling.cu, r67): the L1TEX rate of one 128-B
+    line per clock per SM that a gather touching its own line costs."""
+    p = os.path.join(ROOT, GATHER_CEILING)
+    if not os.path.exists(p):
+        return None
+    best = 0.0
+    for ln in open(p):
+        d = json.loads(ln)
+        if d.get("mode") == "ldg" and d.get("range_mb", 1e9) <= 64:
+            best = max(best, float(d["ggather_per_s"]))
+    return best * 1e9 if best else None
+
+
 def ideal_bytes(n, nnz):
     """PAPER.md:96 with the real row-offset width (reading c2)."""
     return 2 * n * 4 + (n + 1) * (8 if nnz >= 2**31 else 4) + 2 * nnz * 4
@@ -405,6 +423,18 @@ def run_gpu(args):
                           "k_hub_fix on three streams (one launch sequence per step)",
                 "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": ideal}
+            gc = gather_ceiling()
+            if gc:
+                # the step gathers x once per entry; an L2-resident gather that
+                # touches its own 128-B line costs one L1TEX wavefront, so
+                # nnz / ceiling is the step's floor unless lanes share lines
+                floor_ms = inp.nnz / gc * 1e3
+                line["gather_roofline"] = {
+                    "bound": "l1tex wavefronts of the x gathers", "gathers_per_step": inp.nnz,
+                    "ceiling_gathers_per_s": round(gc), "floor_ms": round(floor_ms, 4),
+                    "frac": round(floor_ms / ms, 4), "measured_in_run": False,
+                    "source": GATHER_CEILING + " (scripts/gather_ceiling.cu, random 4-B LDG, "
+                                               "L2-resident range, 4-16 in flight)"}
             line["e2e"] = e2e
             line["gpu_launches"] = launches_per_step * K + (1 if iterate_mode else 0)
             line["clocks"] = ck

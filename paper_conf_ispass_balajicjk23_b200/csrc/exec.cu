@@ -427,21 +427,18 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 }
 
 // ------------------------------------------------------------- long rows
-#ifndef SPMV_WARP_PIPE  // A/B build knobs of the warp-per-row sum
-#define SPMV_WARP_PIPE 1
-#endif
-#ifndef SPMV_WARP_MINB
-#define SPMV_WARP_MINB 8
-#endif
 // Strided partial sum of the entries t0, t0 + S, t0 + 2S, ... < L of a row
 // (S = 32: a lane of the warp-per-row sum; S = 256: a thread of the CTA sum),
-// UNR entries in flight, software-pipelined: the col / val of the next UNR
-// entries are loaded before the x gathers of the current ones are consumed, so
-// an iteration costs one memory round trip (the gathers), not two (stream,
-// then gather).  The ragged end is guarded: a slot past the row has v = x = 0
-// and adds +0, which leaves s unchanged (s starts at +0 and is never -0), so
-// the association is exactly t0, t0 + S, t0 + 2S, ... for every UNR.
-template <int SM, int S, int UNR, bool PIPE = true>
+// UNR entries in flight.  PIPE: software-pipelined, the col / val of the next
+// UNR entries are loaded before the x gathers of the current ones are
+// consumed, so an iteration costs one memory round trip (the gathers), not
+// two -- what a latency-bound launch needs (k_small: RMAT-16 16.3 -> 14.2 us,
+// r68/r69); the throughput-bound class kernels keep the plain loop (r69: the
+// pipelined warp rows cost 4 % on Kronecker-28, within noise on RMAT-26).
+// The ragged end is guarded: a slot past the row has v = x = 0 and adds +0,
+// which leaves s unchanged (s starts at +0 and is never -0), so the
+// association is exactly t0, t0 + S, t0 + 2S, ... for every UNR and PIPE.
+template <int SM, int S, int UNR, bool PIPE>
 __device__ __forceinline__ float strided_sum(const int32_t* __restrict__ cc,
                                              const float* __restrict__ vv,
                                              const float* __restrict__ x, int64_t t0, int64_t L,
@@ -498,28 +495,27 @@ __device__ __forceinline__ float strided_sum(const int32_t* __restrict__ cc,
 
 // canonical W = 32 sum of row r (32 strided partials + xor tree), valid in
 // every lane
-template <int SM, int UNR = 4>
+template <int SM, int UNR = 4, bool PIPE = false>
 __device__ __forceinline__ float warp_row_sum_bl(const int32_t* __restrict__ col,
                                                  const float* __restrict__ val,
                                                  const float* __restrict__ x, int64_t b, int L,
                                                  int lane, uint64_t pol) {
-  return warp_tree(strided_sum<SM, 32, UNR, SPMV_WARP_PIPE>(col + b, val + b, x, lane, L, pol));
+  return warp_tree(strided_sum<SM, 32, UNR, PIPE>(col + b, val + b, x, lane, L, pol));
 }
 
-template <typename OT, int SM, int UNR = 4>
+template <typename OT, int SM, int UNR = 4, bool PIPE = false>
 __device__ __forceinline__ float warp_row_sum(const OT* __restrict__ rp,
                                               const int32_t* __restrict__ col,
                                               const float* __restrict__ val,
                                               const float* __restrict__ x, int r, int lane,
                                               uint64_t pol) {
   const int64_t b = (int64_t)rp[r];
-  return warp_row_sum_bl<SM, UNR>(col, val, x, b, (int)((int64_t)rp[r + 1] - b), lane, pol);
+  return warp_row_sum_bl<SM, UNR, PIPE>(col, val, x, b, (int)((int64_t)rp[r + 1] - b), lane, pol);
 }
 
-// 8 CTAs (64 warps) per SM: held to 32 registers (the SS / int64 variant took
-// 34, which the 8-register allocation granularity rounds to 6 CTAs per SM)
+// (holding it to 32 registers for 8 CTAs per SM cost 4 % on Kronecker-28, r69)
 template <typename OT, bool SS, int SM, int UNR = 4>
-__global__ void __launch_bounds__(256, SPMV_WARP_MINB)
+__global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
                 float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
@@ -541,14 +537,14 @@ __global__ void __launch_bounds__(256, SPMV_WARP_MINB)
 }
 
 // canonical W = 256 sum of entries [b, b + L) of a row
-template <int SM, int UNR = 4>
+template <int SM, int UNR = 4, bool PIPE = false>
 __device__ __forceinline__ float cta_sum256(const int32_t* __restrict__ col,
                                             const float* __restrict__ val,
                                             const float* __restrict__ x, int64_t b, int64_t L,
                                             float* red) {
   const int tid = threadIdx.x;
   const uint64_t pol = stream_policy<SM>();
-  const float s = strided_sum<SM, 256, UNR>(col + b, val + b, x, tid, L, pol);
+  const float s = strided_sum<SM, 256, UNR, PIPE>(col + b, val + b, x, tid, L, pol);
   red[tid] = s;
   __syncthreads();
 #pragma unroll
@@ -716,9 +712,6 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 // Design note (profiles/r01_summary.md, r26): a persistent variant with a
 // sliding shared-memory x window, one barrier per block and evict_first
 // stream hints ran 1.25x slower than this plain form on SBM 4M/64M.
-#ifndef SPMV_SMALL_UNR  // A/B: entries in flight per thread in k_small's MID / CTA rows
-#define SPMV_SMALL_UNR 4
-#endif
 constexpr int LN_THREADS = 256;
 constexpr int MID_STREAM_DEFAULT = 0;  // stream-load mode of the MID / CTA / hub kernels (lds)
 constexpr int LN_WARPS = LN_THREADS / 32;
@@ -910,7 +903,7 @@ __global__ void __launch_bounds__(LN_THREADS)
     const int64_t q = (blk - B_lane) * 8 + warp;
     if (q < n_mid) {
       const int r = mid_rows[q];
-      const float s = warp_row_sum<OT, SM, SPMV_SMALL_UNR>(rp, col, val, x, r, lane, stream_policy<SM>());
+      const float s = warp_row_sum<OT, SM, 8, true>(rp, col, val, x, r, lane, stream_policy<SM>());
       if (lane == 0) {
         const float v = __fmul_rn(s, alpha);
         store_y<SS>(y, dst, r, v);
@@ -921,7 +914,7 @@ __global__ void __launch_bounds__(LN_THREADS)
     const int64_t i = blk - B_lane - B_mid;
     const int r = cta_rows[i];
     const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
-    const float s = cta_sum256<SM, SPMV_SMALL_UNR>(col, val, x, b, L, red);
+    const float s = cta_sum256<SM, 8, true>(col, val, x, b, L, red);
     if (tid == 0) {
       const float v = __fmul_rn(s, alpha);
       store_y<SS>(y, dst, r, v);
