@@ -19,6 +19,11 @@ constexpr int CTA_MAX = 16384;      // CTA-per-row class upper bound
 constexpr int HUB_CHUNK = 16384;    // merge-path chunk of a hub row
 constexpr int CTA_THREADS = 256;    // canonical width of CTA / hub-chunk sums
 constexpr int TILE_BUF = TILE_D + STREAM_MAX + 8;  // max entries of a tile (+ alignment slack)
+// Scheduling only (never a row's value): plans of at most SMALL_NNZ entries
+// and no hub rows run every class in one launch (k_small), where MID rows
+// longer than MID_WIDE get a whole CTA (products staged in shared memory).
+constexpr int64_t SMALL_NNZ = int64_t(1) << 24;
+constexpr int MID_WIDE = 512;
 
 void set_error(const std::string& msg);
 const char* get_error();

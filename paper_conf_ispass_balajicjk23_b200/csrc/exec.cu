@@ -25,6 +25,10 @@
 
 #include "plan.cuh"
 
+#ifndef SPMV_PRED_MINB4  // A/B: hold the predicated-gather k_lane to 64 registers
+#define SPMV_PRED_MINB4 0
+#endif
+
 namespace spmv {
 namespace {
 
@@ -817,7 +821,7 @@ __device__ __forceinline__ void warp_ss(double ssacc, double* out) {
 // 3 CTAs per SM and costs 22 % (r66: 4.45 vs 3.64 ms on C5): both variants
 // are held to 64 registers, 4 CTAs per SM
 template <typename OT, bool SS, int EF>
-__global__ void __launch_bounds__(LN_THREADS, SS ? 4 : 1)
+__global__ void __launch_bounds__(LN_THREADS, (SS || SPMV_PRED_MINB4 && (EF & 8)) ? 4 : 1)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
            int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss,
@@ -871,21 +875,30 @@ __global__ void __launch_bounds__(LN_THREADS, SS ? 4 : 1)
 
 // Small plans (no hub rows, few entries): every row class in ONE launch, no
 // fork / join -- CTA i < B_lane computes the 256-row lane block i, the next
-// B_mid CTAs eight MID rows each (warp per row), the last n_cta CTAs one CTA
-// row each.  Same per-row association as the separate kernels (bitwise equal
-// y); launch and fork/join latency dominate such plans (RMAT-16: 8 MB).
+// B_mid CTAs eight MID rows each (warp per row, rows with L <= MID_WIDE), the
+// next n_wide CTAs one wide MID row each (L > MID_WIDE), the last n_cta CTAs
+// one CTA row each.  Same per-row association as the separate kernels
+// (bitwise equal y); launch and dependent-load latency dominate such plans
+// (RMAT-16: 8 MB), so the long rows' loads are all put in flight at once: a
+// wide MID row's 256 threads each form up to eight products p_e = v_e * x_e
+// (fp32, rounded once, as the warp sum does) into shared memory, then lane j
+// of warp 0 adds p_j, p_{j+32}, ... in that order -- exactly the W = 32
+// strided association of warp_row_sum -- and the xor tree.
 template <typename OT, bool SS, int EF, int SM>
 __global__ void __launch_bounds__(LN_THREADS)
     k_small(const OT* __restrict__ rp, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
             int64_t nrows, const int32_t* __restrict__ mid_rows, int64_t n_mid,
+            const int32_t* __restrict__ mid_wide, int64_t n_wide,
             const int32_t* __restrict__ cta_rows, int64_t B_lane, int64_t B_mid,
             const double* __restrict__ ss_in, double* __restrict__ blk_ss,
             double* __restrict__ mid_ss, double* __restrict__ cta_ss, const YDst dst) {
   __shared__ float red[256];
+  __shared__ float prod[WARP_MAX];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const float alpha = alpha_of(ss_in);
   const int64_t blk = blockIdx.x;
+  const uint64_t pol = stream_policy<SM>();
   if (blk < B_lane) {  // block-uniform branches
     const int64_t r = blk * LN_THREADS + tid;
     double ssacc = 0.0;
@@ -903,15 +916,55 @@ __global__ void __launch_bounds__(LN_THREADS)
     const int64_t q = (blk - B_lane) * 8 + warp;
     if (q < n_mid) {
       const int r = mid_rows[q];
-      const float s = warp_row_sum<OT, SM, 8, true>(rp, col, val, x, r, lane, stream_policy<SM>());
+      const int64_t b = (int64_t)rp[r];
+      const int L = (int)((int64_t)rp[r + 1] - b);
+      if (L <= MID_WIDE) {  // (wide rows: their own CTA below)
+        const float s = warp_row_sum_bl<SM, 8, true>(col, val, x, b, L, lane, pol);
+        if (lane == 0) {
+          const float v = __fmul_rn(s, alpha);
+          store_y<SS>(y, dst, r, v);
+          if (SS) mid_ss[q] = (double)v * (double)v;
+        }
+      }
+    }
+  } else if (blk < B_lane + B_mid + n_wide) {
+    const int64_t q = mid_wide[blk - B_lane - B_mid];
+    const int r = mid_rows[q];
+    const int64_t b = (int64_t)rp[r];
+    const int L = (int)((int64_t)rp[r + 1] - b);  // MID_WIDE < L <= WARP_MAX
+    constexpr int PER = WARP_MAX / LN_THREADS;       // 8 entries per thread
+    int c[PER];
+    float v[PER];
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int e = tid + LN_THREADS * k;
+      c[k] = e < L ? lds<SM>(col + b + e, pol) : 0;
+      v[k] = e < L ? lds<SM>(val + b + e, pol) : 0.f;
+    }
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int e = tid + LN_THREADS * k;
+      if (e < L) prod[e] = __fmul_rn(v[k], gx(x, c[k]));
+    }
+    __syncthreads();
+    if (warp == 0) {
+      float s = 0.f;
+      for (int j0 = lane; j0 < L; j0 += 32 * 8) {  // 8 products read ahead, added in order
+        float pv[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) pv[u] = j0 + 32 * u < L ? prod[j0 + 32 * u] : 0.f;
+#pragma unroll
+        for (int u = 0; u < 8; ++u) s = __fadd_rn(s, pv[u]);
+      }
+      s = warp_tree(s);
       if (lane == 0) {
-        const float v = __fmul_rn(s, alpha);
-        store_y<SS>(y, dst, r, v);
-        if (SS) mid_ss[q] = (double)v * (double)v;
+        const float o = __fmul_rn(s, alpha);
+        store_y<SS>(y, dst, r, o);
+        if (SS) mid_ss[q] = (double)o * (double)o;
       }
     }
   } else {
-    const int64_t i = blk - B_lane - B_mid;
+    const int64_t i = blk - B_lane - B_mid - n_wide;
     const int r = cta_rows[i];
     const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
     const float s = cta_sum256<SM, 8, true>(col, val, x, b, L, red);
@@ -1032,11 +1085,12 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   // launch (SPMV_FORK_EARLY=0: the other classes start when it has finished).
   if (lane_mode && small_plan(p)) {  // one launch for every row class
     const int64_t B_lane = (p->nrows + LN_THREADS - 1) / LN_THREADS, B_mid = (p->n_mid + 7) / 8;
-    const unsigned g = (unsigned)(B_lane + B_mid + p->n_cta);
+    const unsigned g = (unsigned)(B_lane + B_mid + p->n_mid_wide + p->n_cta);
     const OT* rp = (const OT*)p->d_rp;
     constexpr int SM = MID_STREAM_DEFAULT;
 #define SPMV_SMALL_ARGS                                                                      \
-  rp, p->d_col, p->d_val, x, y, p->nrows, p->d_mid_rows, p->n_mid, p->d_cta_rows, B_lane, B_mid, \
+  rp, p->d_col, p->d_val, x, y, p->nrows, p->d_mid_rows, p->n_mid, p->d_mid_wide, p->n_mid_wide,  \
+      p->d_cta_rows, B_lane, B_mid,                                                                \
       ss_in, p->d_blk_ss, p->d_mid_ss, p->d_cta_ss, dst
     const int ef = (lane_ef_mode(p) == 1 ? 1 : 0) | (p->val_nonfinite ? 4 : 0) |
                    (lane_pred_mode(p) ? 8 : 0);
@@ -1137,7 +1191,9 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   }
   // spmv_iterate reads x from two buffers in turn: both windows must fit the
   // persisting carve-out at once, or each step evicts the other's lines
-  if (p->win_alternating) bytes = std::min<int64_t>(bytes, (int64_t)maxpers / 2);
+  bool halve = p->win_alternating;
+  if (const char* e = getenv("SPMV_WIN_ALT_FULL")) if (atoi(e)) halve = false;  // dev knob (A/B)
+  if (halve) bytes = std::min<int64_t>(bytes, (int64_t)maxpers / 2);
   if (const char* e = getenv("SPMV_WIN_HIT")) hit = std::min(1.0, std::max(0.0, atof(e)));  // dev knob
   if (bytes <= 0) return;
   size_t cur = 0;

@@ -300,6 +300,15 @@ __global__ void k_compact(const int32_t* f, const int64_t* pos, int64_t n, int32
   GRID_STRIDE(i, n) if (f[i]) out[pos[i]] = (int32_t)i;
 }
 
+// MID-list positions q whose row is longer than MID_WIDE (k_small's wide rows)
+template <typename OT>
+__global__ void k_mid_wide_flag(const OT* rp, const int32_t* mid_rows, int64_t n_mid, int32_t* f) {
+  GRID_STRIDE(q, n_mid) {
+    const int r = mid_rows[q];
+    f[q] = (int64_t)rp[r + 1] - (int64_t)rp[r] > MID_WIDE;
+  }
+}
+
 template <typename OT>
 __global__ void k_nchunks(const OT* rp, const int32_t* hub_rows, int64_t nh, int32_t* nch) {
   GRID_STRIDE(h, nh) {
@@ -369,6 +378,9 @@ __global__ void k_first_cold(const uint32_t* cnt, int64_t n, int64_t nnz,
 // ------------------------------------------------------------- P A P^T data
 // Key (col_B << 32 | position in row) is unique inside a row, so any correct
 // sort by key is the stable sort by col_B (duplicates keep A's order).
+// rows up to this length are relabelled and sorted in registers (one pass)
+constexpr int64_t REG_SORT_MAX = 256;
+
 __device__ __forceinline__ uint64_t mkkey(int32_t c, int64_t rel) {
   return ((uint64_t)(uint32_t)c << 32) | (uint64_t)(uint32_t)rel;
 }
@@ -392,11 +404,91 @@ __device__ __forceinline__ void lane_bitonic(uint64_t& key, float& v, int gl) {
   }
 }
 
+// Warp bitonic sort of up to 32 * E keys in registers: element i = k * 32 +
+// lane lives in register k of lane `lane`; partners i ^ j with j >= 32 are in
+// the same lane (registers k, k ^ j/32), with j < 32 in lane ^ j (shuffles).
+// Ascending within blocks of size kk where (i & kk) == 0, as lane_bitonic.
+template <int E>
+__device__ __forceinline__ void warp_bitonic(uint64_t (&key)[E], float (&v)[E], int lane) {
+  constexpr int LOG = E == 4 ? 7 : 8;  // 32 * E = 2^LOG keys
+  static_assert(E == 4 || E == 8, "warp_bitonic: 4 or 8 keys per lane");
+#pragma unroll
+  for (int lk = 1; lk <= LOG; ++lk) {  // counted loops: fully unrolled, registers stay registers
+    const int kk = 1 << lk;
+#pragma unroll
+    for (int lj = lk - 1; lj >= 0; --lj) {
+      const int j = 1 << lj;
+      if (j >= 32) {
+        const int jr = j >> 5;
+#pragma unroll
+        for (int k = 0; k < E; ++k) {
+          const int pk = k ^ jr;
+          if (pk > k) {
+            const bool asc = (((k << 5) | lane) & kk) == 0;
+            if ((key[k] > key[pk]) == asc) {
+              const uint64_t tk = key[k];
+              key[k] = key[pk];
+              key[pk] = tk;
+              const float tv = v[k];
+              v[k] = v[pk];
+              v[pk] = tv;
+            }
+          }
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < E; ++k) {
+          const uint64_t ok = __shfl_xor_sync(0xffffffffu, key[k], j);
+          const float ov = __shfl_xor_sync(0xffffffffu, v[k], j);
+          const int i = (k << 5) | lane;
+          const bool take_min = ((i & j) == 0) == ((i & kk) == 0);
+          if (take_min == (ok < key[k])) {
+            key[k] = ok;
+            v[k] = ov;
+          }
+        }
+      }
+    }
+  }
+}
+
+// one row with L <= 32 * E relabelled and sorted by the whole warp in registers
+template <int E, typename OT>
+__device__ __forceinline__ void warp_relabel_sort(const int32_t* __restrict__ colA,
+                                                  const float* __restrict__ valA,
+                                                  const int32_t* __restrict__ perm, int64_t a,
+                                                  int64_t L, int64_t d, int lane,
+                                                  int32_t* __restrict__ colB,
+                                                  float* __restrict__ valB) {
+  uint64_t key[E];
+  float v[E];
+#pragma unroll
+  for (int k = 0; k < E; ++k) {
+    const int i = (k << 5) | lane;
+    key[k] = ~0ull;
+    v[k] = 0.f;
+    if (i < L) {
+      key[k] = mkkey(perm[colA[a + i]], i);
+      v[k] = valA[a + i];
+    }
+  }
+  warp_bitonic<E>(key, v, lane);
+#pragma unroll
+  for (int k = 0; k < E; ++k) {
+    const int i = (k << 5) | lane;
+    if (i < L) {
+      colB[d + i] = (int32_t)(key[k] >> 32);
+      valB[d + i] = v[k];
+    }
+  }
+}
+
 // Rows with L <= 32 relabelled AND sorted in registers: one read of A's row,
 // one gather of perm per entry, one write of B's row.  A warp
 // takes rows 2q and 2q+1: a half-warp each when both have L <= 16 (width-16
-// sort network), else the whole warp on each in turn (width 32).  Longer rows
-// are left to k_relabel_warp / k_relabel_cta and the shared-memory sorts.
+// sort network), else the whole warp on each in turn (width 32).  Rows with
+// 32 < L <= REG_SORT_MAX: k_relabel_sort_mid; longer rows: k_relabel_warp /
+// k_relabel_cta and the shared-memory sorts.
 template <typename AT, typename OT>
 __global__ void __launch_bounds__(256)
     k_relabel_sort_short(const AT* __restrict__ rpA, const int32_t* __restrict__ colA,
@@ -452,7 +544,27 @@ __global__ void __launch_bounds__(256)
   }
 }
 
-// warp per row for rows with 32 < L <= WARP_MAX (relabel only; sorted after)
+// Rows with 32 < L <= REG_SORT_MAX (the plan's list s1): warp per row,
+// relabelled and sorted in registers (4 or 8 keys per lane), one pass -- a
+// kernel of its own so the L <= 32 kernel keeps its occupancy (64 registers)
+template <typename AT, typename OT>
+__global__ void __launch_bounds__(256)
+    k_relabel_sort_mid(const int32_t* __restrict__ rows, int64_t nlist,
+                       const int32_t* __restrict__ colA, const float* __restrict__ valA,
+                       const int32_t* __restrict__ perm, const int64_t* __restrict__ srcA,
+                       const OT* __restrict__ rpB, int32_t* __restrict__ colB,
+                       float* __restrict__ valB) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t t = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; t < nlist; t += nw) {
+    const int64_t r = rows[t];
+    const int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d, a = srcA[r];
+    if (L <= 128) warp_relabel_sort<4, OT>(colA, valA, perm, a, L, d, lane, colB, valB);
+    else warp_relabel_sort<8, OT>(colA, valA, perm, a, L, d, lane, colB, valB);
+  }
+}
+
+// warp per row for rows with REG_SORT_MAX < L <= WARP_MAX (relabel only; sorted after)
 template <typename AT, typename OT>
 __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* valA,
                                const int32_t* perm, const int64_t* srcA,
@@ -462,7 +574,7 @@ __global__ void k_relabel_warp(const AT* rpA, const int32_t* colA, const float* 
   int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t r = w; r < nrows; r += nw) {
     int64_t d = (int64_t)rpB[r], L = (int64_t)rpB[r + 1] - d;
-    if (L <= SHORT_MAX || L > WARP_MAX) continue;  // k_relabel_sort_short / k_relabel_cta
+    if (L <= REG_SORT_MAX || L > WARP_MAX) continue;  // k_relabel_sort_short / k_relabel_cta
     int64_t a = srcA[r];
     for (int64_t k = lane; k < L; k += 32) {
       colB[d + k] = perm[colA[a + k]];
@@ -557,65 +669,140 @@ __global__ void k_big_load(const OT* rp, const int32_t* rows, const int64_t* bof
   }
 }
 
-// sort every BIG_CHUNK-run of every big row in shared memory
-__global__ void k_big_chunk_sort(const int64_t* boff, int64_t nb, uint64_t* K, float* V) {
+// sort every BIG_CHUNK-run of every big row in shared memory (one CTA per
+// tile of the plan's tile list: no empty CTAs for the short big rows)
+__global__ void k_big_chunk_sort(const BigTile* tiles, uint64_t* K, float* V) {
   extern __shared__ __align__(16) unsigned char sm[];
   uint64_t* keys = (uint64_t*)sm;
   float* vals = (float*)(keys + BIG_CHUNK);
-  int64_t b = blockIdx.x;
-  if (b >= nb) return;
-  int64_t o = boff[b], L = boff[b + 1] - o;
-  int64_t c0 = (int64_t)blockIdx.y * BIG_CHUNK;
-  if (c0 >= L) return;
-  int64_t m = min((int64_t)BIG_CHUNK, L - c0);
+  const BigTile t = tiles[blockIdx.x];
+  const int64_t e0 = t.o + t.q;
+  const int64_t m = min((int64_t)BIG_CHUNK, t.L - t.q);
   for (int i = threadIdx.x; i < BIG_CHUNK; i += blockDim.x) {
-    keys[i] = i < m ? K[o + c0 + i] : ~0ull;
-    vals[i] = i < m ? V[o + c0 + i] : 0.f;
+    keys[i] = i < m ? K[e0 + i] : ~0ull;
+    vals[i] = i < m ? V[e0 + i] : 0.f;
   }
   __syncthreads();
   smem_bitonic<BIG_CHUNK>(keys, vals, BIG_CHUNK);
   for (int i = threadIdx.x; i < m; i += blockDim.x) {
-    K[o + c0 + i] = keys[i];
-    V[o + c0 + i] = vals[i];
+    K[e0 + i] = keys[i];
+    V[e0 + i] = vals[i];
   }
 }
 
-// one merge pass of width w over all big rows: element-wise rank merge
-__global__ void k_big_merge(const int64_t* boff, int64_t nb, int64_t total, int64_t w,
-                            const uint64_t* K, const float* V, uint64_t* K2, float* V2) {
-  GRID_STRIDE(e, total) {
-    int64_t lo = 0, hi = nb;  // find b with boff[b] <= e < boff[b+1]
-    while (hi - lo > 1) {
-      int64_t mid = (lo + hi) >> 1;
-      if (boff[mid] <= e) lo = mid; else hi = mid;
+// One merge pass of width w over every big row, merge path per output tile.
+// Runs [base, base + w) = A and [base + w, base + 2w) = B of a row (base a
+// multiple of 2w) merge into the same positions of the output; keys are
+// unique (column << 32 | position), so "A before B on ties" never arises.
+// The tile at diagonal d (its first output, relative to base) takes
+// split(d) = #A among the first d outputs = the smallest i with
+// A[i] > B[d - i - 1]; k_big_split finds it for every tile (one thread each,
+// binary search in global memory), k_big_merge_tile loads the tile's A and B
+// pieces into shared memory and merges them (16 outputs per thread, their own
+// merge-path search in shared memory), staging the outputs for a coalesced
+// store.  Tiles never straddle a pair: 2w is a multiple of BIG_CHUNK.
+__device__ __forceinline__ void big_pair(const BigTile& t, int64_t w, int64_t& base, int64_t& nA,
+                                         int64_t& nB) {
+  base = t.q / (2 * w) * (2 * w);
+  nA = min(w, t.L - base);
+  nB = max((int64_t)0, min(t.L, base + 2 * w) - (base + w));
+}
+
+__global__ void k_big_split(const BigTile* tiles, int64_t nt, int64_t w, const uint64_t* K,
+                            int64_t* split) {
+  GRID_STRIDE(i, nt) {
+    const BigTile t = tiles[i];
+    int64_t base, nA, nB;
+    big_pair(t, w, base, nA, nB);
+    const int64_t d = t.q - base;
+    const uint64_t* A = K + t.o + base;
+    const uint64_t* B = A + w;
+    int64_t lo = max((int64_t)0, d - nB), hi = min(d, nA);
+    while (lo < hi) {
+      const int64_t mid = (lo + hi) >> 1;
+      if (A[mid] < B[d - mid - 1]) lo = mid + 1;
+      else hi = mid;
     }
-    int64_t o = boff[lo], L = boff[lo + 1] - o, rel = e - o;
-    int64_t run = rel / w, base = (run & ~1ll) * w;
-    uint64_t key = K[e];
-    int64_t out;
-    if ((run & 1) == 0) {
-      int64_t b0 = base + w, b1 = min(base + 2 * w, L);
-      int64_t cnt = 0;
-      if (b0 < b1) {  // count keys in B less than key
-        int64_t l = b0, h = b1;
-        while (l < h) {
-          int64_t mid = (l + h) >> 1;
-          if (K[o + mid] < key) l = mid + 1; else h = mid;
-        }
-        cnt = l - b0;
-      }
-      out = base + (rel - base) + cnt;
-    } else {
-      int64_t a0 = base, a1 = base + w;
-      int64_t l = a0, h = a1;
-      while (l < h) {
-        int64_t mid = (l + h) >> 1;
-        if (K[o + mid] < key) l = mid + 1; else h = mid;
-      }
-      out = base + (rel - base - w) + (l - a0);
+    split[i] = lo;
+  }
+}
+
+constexpr int MT_THREADS = 256, MT_PER = BIG_CHUNK / MT_THREADS;  // 16 outputs per thread
+static_assert(MT_PER * MT_THREADS == BIG_CHUNK, "merge tile = BIG_CHUNK outputs");
+
+__global__ void __launch_bounds__(MT_THREADS)
+    k_big_merge_tile(const BigTile* tiles, int64_t nt, int64_t w, const int64_t* split,
+                     const uint64_t* K, const float* V, uint64_t* K2, float* V2) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  uint64_t* sk = (uint64_t*)sm;                // [BIG_CHUNK]: A piece then B piece, then outputs
+  float* sv = (float*)(sk + BIG_CHUNK);
+  const int64_t ti = blockIdx.x;
+  const BigTile t = tiles[ti];
+  int64_t base, nA, nB;
+  big_pair(t, w, base, nA, nB);
+  const int64_t d = t.q - base, d1 = min(d + (int64_t)BIG_CHUNK, nA + nB);
+  const int64_t m = d1 - d;
+  const int64_t out0 = t.o + base + d;
+  if (nB == 0) {  // unpaired last run: already sorted, copy
+    for (int64_t k = threadIdx.x; k < m; k += MT_THREADS) {
+      K2[out0 + k] = K[out0 + k];
+      V2[out0 + k] = V[out0 + k];
     }
-    K2[o + out] = key;
-    V2[o + out] = V[e];
+    return;
+  }
+  const int64_t i0 = split[ti];
+  const bool next_same = ti + 1 < nt && tiles[ti + 1].o == t.o && tiles[ti + 1].q < base + 2 * w;
+  const int64_t i1 = next_same ? split[ti + 1] : nA;
+  const int64_t j0 = d - i0, j1 = d1 - i1;
+  const int na = (int)(i1 - i0), nb = (int)(j1 - j0);
+  const uint64_t* A = K + t.o + base;
+  const float* AV = V + t.o + base;
+  for (int k = threadIdx.x; k < na; k += MT_THREADS) {
+    sk[k] = A[i0 + k];
+    sv[k] = AV[i0 + k];
+  }
+  for (int k = threadIdx.x; k < nb; k += MT_THREADS) {
+    sk[na + k] = A[w + j0 + k];
+    sv[na + k] = AV[w + j0 + k];
+  }
+  __syncthreads();
+  const uint64_t* sA = sk;
+  const uint64_t* sB = sk + na;
+  uint64_t ok[MT_PER];
+  float ov[MT_PER];
+  const int dk = threadIdx.x * MT_PER;
+  if (dk < m) {
+    int lo = max(0, dk - nb), hi = min(dk, na);
+    while (lo < hi) {
+      const int mid = (lo + hi) >> 1;
+      if (sA[mid] < sB[dk - mid - 1]) lo = mid + 1;
+      else hi = mid;
+    }
+    int ia = lo, ib = dk - lo;
+#pragma unroll
+    for (int u = 0; u < MT_PER; ++u) {
+      const bool takeA = ib >= nb || (ia < na && sA[ia] < sB[ib]);
+      const int src = takeA ? ia : na + ib;
+      ok[u] = sk[src];
+      ov[u] = sv[src];
+      ia += takeA;
+      ib += !takeA;
+    }
+  }
+  __syncthreads();
+  if (dk < m) {
+#pragma unroll
+    for (int u = 0; u < MT_PER; ++u) {
+      if (dk + u < m) {
+        sk[dk + u] = ok[u];
+        sv[dk + u] = ov[u];
+      }
+    }
+  }
+  __syncthreads();
+  for (int64_t k = threadIdx.x; k < m; k += MT_THREADS) {
+    K2[out0 + k] = sk[k];
+    V2[out0 + k] = sv[k];
   }
 }
 
@@ -848,9 +1035,17 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   p->n_mid = class_list<OT>(rp, nr, SHORT_MAX, WARP_MAX, &p->d_mid_rows, f, pos, tmp, s);
   p->n_cta = class_list<OT>(rp, nr, WARP_MAX, CTA_MAX, &p->d_cta_rows, f, pos, tmp, s);
   p->n_hub = class_list<OT>(rp, nr, CTA_MAX, INT64_MAX, &p->d_hub_rows, f, pos, tmp, s);
+  if (p->n_hub == 0 && p->n_mid) {  // k_small's wide MID rows (any hub-free plan: SPMV_SMALL=1 forces k_small)
+    k_mid_wide_flag<OT><<<grid_for(p->n_mid), TPB, 0, s>>>(rp, p->d_mid_rows, p->n_mid, f);
+    exclusive_scan<int32_t>(f, p->n_mid, pos, tmp, s);
+    p->n_mid_wide = d2h_one(pos + p->n_mid, s);
+    p->d_mid_wide = dalloc<int32_t>(p->n_mid_wide);
+    if (p->n_mid_wide) k_compact<<<grid_for(p->n_mid), TPB, 0, s>>>(f, pos, p->n_mid, p->d_mid_wide);
+    SPMV_LAUNCH_CHECK();
+  }
   spmv_plan_s* ps = p;
-  ps->n1 = class_list<OT>(rp, nr, 32, 128, &ps->s1, f, pos, tmp, s);
-  ps->n2 = class_list<OT>(rp, nr, 128, 1024, &ps->s2, f, pos, tmp, s);
+  ps->n1 = class_list<OT>(rp, nr, 32, REG_SORT_MAX, &ps->s1, f, pos, tmp, s);  // k_relabel_sort_mid
+  ps->n2 = class_list<OT>(rp, nr, REG_SORT_MAX, 1024, &ps->s2, f, pos, tmp, s);
   ps->n3 = class_list<OT>(rp, nr, 1024, BIG_CHUNK, &ps->s3, f, pos, tmp, s);
   ps->nbig = class_list<OT>(rp, nr, BIG_CHUNK, INT64_MAX, &ps->big, f, pos, tmp, s);
   ps->nlong = class_list<OT>(rp, nr, WARP_MAX, INT64_MAX, &ps->longrows, f, pos, tmp, s);
@@ -864,7 +1059,17 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
     std::vector<int64_t> hl(ps->nbig);
     SPMV_CUDA(cudaMemcpyAsync(hl.data(), blen, 8 * ps->nbig, cudaMemcpyDeviceToHost, s));
     SPMV_CUDA(cudaStreamSynchronize(s));
-    for (int64_t L : hl) { ps->big_total += L; ps->big_max = std::max(ps->big_max, L); }
+    std::vector<BigTile> tiles;
+    for (int64_t L : hl) {
+      for (int64_t q = 0; q < L; q += BIG_CHUNK) tiles.push_back({ps->big_total, L, q});
+      ps->big_total += L;
+      ps->big_max = std::max(ps->big_max, L);
+    }
+    ps->nbtile = (int64_t)tiles.size();
+    ps->btile = dalloc<BigTile>(ps->nbtile);
+    SPMV_CUDA(cudaMemcpyAsync(ps->btile, tiles.data(), sizeof(BigTile) * tiles.size(),
+                              cudaMemcpyHostToDevice, s));
+    SPMV_CUDA(cudaStreamSynchronize(s));  // host vector lifetime
     dfree(blen);
     dfree(t3);
   } else {
@@ -924,7 +1129,10 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
   if (nr) {
     k_relabel_sort_short<AT, OT><<<grid_for((nr + 1) / 2 * 32), 256, 0, s>>>(
         rpA, p->A_col, p->A_val, p->d_perm, p->d_srcA, nr, rp, p->d_col, p->d_val);
-    if (ps->n1 + ps->n2 + ps->n3 + ps->nbig)  // rows with L > 32 exist
+    if (ps->n1)
+      k_relabel_sort_mid<AT, OT><<<grid_for(ps->n1 * 32), 256, 0, s>>>(
+          ps->s1, ps->n1, p->A_col, p->A_val, p->d_perm, p->d_srcA, rp, p->d_col, p->d_val);
+    if (ps->n2 + ps->n3 + ps->nbig)  // rows with L > REG_SORT_MAX exist
       k_relabel_warp<AT, OT><<<grid_for(nr * 32), TPB, 0, s>>>(
           rpA, p->A_col, p->A_val, p->d_perm, p->d_srcA, nr, rp, p->d_col, p->d_val);
     if (ps->nlong)
@@ -932,10 +1140,6 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
           rpA, p->A_col, p->A_val, p->d_perm, p->d_srcA, ps->longrows, ps->nlong,
           rp, p->d_col, p->d_val);
     SPMV_LAUNCH_CHECK();
-    if (ps->n1) {
-      k_sort_cta<128, OT><<<(unsigned)std::min<int64_t>(ps->n1, 148 * 64), 64, 128 * 12, s>>>(
-          rp, ps->s1, ps->n1, p->d_col, p->d_val);
-    }
     if (ps->n2) {
       k_sort_cta<1024, OT><<<(unsigned)std::min<int64_t>(ps->n2, 148 * 16), 256, 1024 * 12, s>>>(
           rp, ps->s2, ps->n2, p->d_col, p->d_val);
@@ -952,19 +1156,21 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
       float* V2 = dalloc<float>(ps->big_total);
       unsigned nb = (unsigned)std::min<int64_t>(ps->nbig, 148 * 8);
       k_big_load<OT><<<nb, 512, 0, s>>>(rp, ps->big, ps->boff, ps->nbig, p->d_col, p->d_val, K1, V1);
-      dim3 g((unsigned)ps->nbig, (unsigned)((ps->big_max + BIG_CHUNK - 1) / BIG_CHUNK));
-      k_big_chunk_sort<<<g, 512, BIG_CHUNK * 12, s>>>(ps->boff, ps->nbig, K1, V1);
+      k_big_chunk_sort<<<(unsigned)ps->nbtile, 512, BIG_CHUNK * 12, s>>>(ps->btile, K1, V1);
       SPMV_LAUNCH_CHECK();
+      int64_t* split = dalloc<int64_t>(ps->nbtile);
       for (int64_t w = BIG_CHUNK; w < ps->big_max; w *= 2) {
-        k_big_merge<<<grid_for(ps->big_total), TPB, 0, s>>>(ps->boff, ps->nbig, ps->big_total, w,
-                                                            K1, V1, K2, V2);
+        k_big_split<<<grid_for(ps->nbtile), TPB, 0, s>>>(ps->btile, ps->nbtile, w, K1, split);
+        k_big_merge_tile<<<(unsigned)ps->nbtile, MT_THREADS, BIG_CHUNK * 12, s>>>(
+            ps->btile, ps->nbtile, w, split, K1, V1, K2, V2);
+        SPMV_LAUNCH_CHECK();
         std::swap(K1, K2);
         std::swap(V1, V2);
       }
       k_big_store<OT><<<nb, 512, 0, s>>>(rp, ps->big, ps->boff, ps->nbig, K1, V1, p->d_col, p->d_val);
       SPMV_LAUNCH_CHECK();
       SPMV_CUDA(cudaStreamSynchronize(s));  // scratch lifetime
-      dfree(K1); dfree(K2); dfree(V1); dfree(V2);
+      dfree(K1); dfree(K2); dfree(V1); dfree(V2); dfree(split);
     }
   }
   if (p->nnz_local) {
@@ -1142,12 +1348,13 @@ void pad_vec(spmv_plan_s* p, const float* in, float* out, int to_padded, cudaStr
 
 void plan_free(spmv_plan_s* p) {
   coo_free(p);
-  dfree(p->s1); dfree(p->s2); dfree(p->s3); dfree(p->big); dfree(p->boff);
+  dfree(p->s1); dfree(p->s2); dfree(p->s3); dfree(p->big); dfree(p->boff); dfree(p->btile);
   dfree(p->longrows);
   dfree(p->d_perm); dfree(p->d_inv); dfree(p->d_srcA);
   if (p->d_rp) { cudaFree(p->d_rp); p->d_rp = nullptr; }
   dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows); dfree(p->d_desc);
   dfree(p->d_warp_rows); dfree(p->d_warp_ss); dfree(p->d_mid_rows); dfree(p->d_mid_ss);
+  dfree(p->d_mid_wide);
   dfree(p->d_chunk_part4);
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
   dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_blk_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);

@@ -12,6 +12,12 @@ struct TileDesc {
   uint32_t packed;
 };
 
+// a BIG_CHUNK-aligned tile of a big row in the key scratch of spmv_permute:
+// row start o, row length L, tile start q within the row
+struct BigTile {
+  int64_t o, L, q;
+};
+
 struct spmv_plan_s {
   int device = 0;
   spmv_opts_t opts{};
@@ -52,6 +58,8 @@ struct spmv_plan_s {
   int32_t* d_warp_rows = nullptr;  // [n_warp] k_panel: last-in-tile rows, 1024 < L <= 2048
   int64_t n_mid = 0;
   int32_t* d_mid_rows = nullptr;   // [n_mid] k_lane: all rows with 32 < L <= 2048
+  int64_t n_mid_wide = 0;          // small plans: MID-list positions q of rows with L > MID_WIDE
+  int32_t* d_mid_wide = nullptr;   // [n_mid_wide] (k_small gives each a CTA)
   int32_t* d_cta_rows = nullptr;   // [n_cta]
   int32_t* d_hub_rows = nullptr;   // [n_hub]
   int32_t* d_hub_choff = nullptr;  // [n_hub+1] first chunk of each hub row
@@ -87,6 +95,7 @@ struct spmv_plan_s {
   int32_t* s3 = nullptr; int64_t n3 = 0;        // 1024 < L <= 4096
   int32_t* big = nullptr; int64_t nbig = 0;     // L > 4096 (chunk sort + merges)
   int64_t* boff = nullptr; int64_t big_total = 0, big_max = 0;
+  BigTile* btile = nullptr; int64_t nbtile = 0;  // BIG_CHUNK-aligned tiles of the big rows
   int32_t* longrows = nullptr; int64_t nlong = 0;  // L > STREAM_MAX
 
   // exec concurrency: the row-class kernels other than the short-row kernel

@@ -30,6 +30,7 @@ ap.add_argument("--ordering", default="rabbitpp")
 ap.add_argument("--steps", type=int, default=10)
 ap.add_argument("--iterate", action="store_true", help="time spmv_iterate steps instead of execs")
 ap.add_argument("--ncu", type=int, default=0)
+ap.add_argument("--ncu-scaled", action="store_true", help="--ncu N: N execs, then N exec_scaled (fixed x)")
 ap.add_argument("--env", nargs="*", default=[])
 ap.add_argument("--sequential-reorder", action="store_true")
 ap.add_argument("--no-reset", action="store_true", help="flush without the persisting-L2 reset")
@@ -74,7 +75,16 @@ else:
     perm, _ = spmv.reorder(host_rp, host_col, a.ordering, parallel=not a.sequential_reorder)
     np.save(f, perm)
 reorder_s = time.time() - t0
-P = spmv.Plan(rp_d, col_d, val_d, torch.from_numpy(perm).to(dev))
+perm_d = torch.from_numpy(perm).to(dev)
+torch.cuda.synchronize()
+t0 = time.time()
+P = spmv.Plan(rp_d, col_d, val_d, perm_d, permute=False)
+torch.cuda.synchronize()
+plan_s = time.time() - t0
+t0 = time.time()
+P.permute()
+torch.cuda.synchronize()
+permute_s = time.time() - t0
 info = P.info()
 xB = P.permute_vec(torch.from_numpy(np.ascontiguousarray(x, np.float32)).to(dev))
 y = torch.empty(n, dtype=torch.float32, device=dev)
@@ -95,6 +105,12 @@ if a.ncu:
     for _ in range(a.ncu):
         fl()
         P.exec(xB, y)
+    if a.ncu_scaled:
+        ss = torch.zeros(2, dtype=torch.float64, device=dev)
+        P.exec_scaled(xB, y, None, ss[:1])
+        for _ in range(a.ncu):
+            fl()
+            P.exec_scaled(xB, y, ss[:1], ss[1:])
     torch.cuda.synchronize()
     print(json.dumps({"ncu_execs": a.ncu, "workload": name, "ordering": a.ordering}))
     sys.exit(0)
@@ -150,6 +166,7 @@ print(json.dumps({"workload": name, "ordering": a.ordering, "env": a.env + (["no
                   "cold_ms": round(cold_ms, 4), "warm_ms": round(warm_ms, 4), "iterate_ms": it_ms, "scaled_fixed_ms": sc_ms,
                   "x_ideal_cold": round(cold_ms * 1e-3 * hbm * 1e9 / ideal, 3),
                   "gen_s": round(gen_s, 2), "reorder_s": round(reorder_s, 1),
+                  "plan_s": round(plan_s, 3), "permute_ms": round(permute_s * 1e3, 1),
                   "mid_rows": info["n_mid_rows"], "cta_rows": info["n_cta_rows"],
                   "hub_rows": info["n_hub_rows"], "H": info["hot_prefix"],
                   "win": P.info()["l2_window_bytes"], "ef": info["stream_evict_first"],
