@@ -15,9 +15,9 @@
 //   k_cta_rows   one CTA per row, 2048 < L <= 16384 (256 strided partials + tree).
 //   k_hub_chunk  one CTA per 16384-entry chunk of a hub row (merge-path split);
 //   k_hub_fix    fp64 combine of the chunk sums in chunk order.
-//   k_ss_part / k_ss_final  fixed-order fp64 sum of per-block / per-row y^2
-//                partials (fixed segments, then the segment sums in order)
-//                (power-iteration norm; deterministic).
+//   k_ss_y / k_ss_final  power-iteration norm: fp64 sum of y^2 over fixed
+//                16384-row segments of y, then the segment sums in order
+//                (deterministic, independent of grid and row classes).
 // No tensor cores: SpMV is not a dense contraction (AI <= 0.25 flop/B).
 #include <atomic>
 #include <cmath>
@@ -25,12 +25,11 @@
 
 #include "plan.cuh"
 
-#ifndef SPMV_PRED_MINB4  // A/B: hold the predicated-gather k_lane to 64 registers
-#define SPMV_PRED_MINB4 0
-#endif
+
 
 namespace spmv {
 namespace {
+
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -62,10 +61,6 @@ __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
                "r"(bytes)
                : "memory");
-}
-
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes,
@@ -210,7 +205,6 @@ struct alignas(16) PanelSmem {
   uint64_t bar[PT_STAGES];
   int32_t mid[MID_CAP];
   int mid_n;
-  double wss[PT_THREADS / 32];
 };
 static_assert((TILE_BUF * 4) % 16 == 0, "stage buffers must stay 16-byte aligned");
 static_assert(TILE_D <= TILE_BUF, "row results reuse a col stage");
@@ -252,7 +246,7 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
     k_panel(const OT* __restrict__ rp, const int32_t* __restrict__ col,
             const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
             const TileDesc* __restrict__ desc, int64_t K, int64_t diag, int64_t xlen,
-            int use_win_i, const double* __restrict__ ss_in, double* __restrict__ tile_ss,
+            int use_win_i, const double* __restrict__ ss_in,
             int evict_first) {
   constexpr int SEGW = 1;  // window advance prefetched per thread (512 floats)
   constexpr int RPF = 1;   // row pointers prefetched per thread
@@ -398,12 +392,10 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
       if (lane == 0) res[q] = acc;
     }
     __syncthreads();
-    double ssacc = 0.0;
     auto emit = [&](int q, OT p0, OT p1) {
       if ((int64_t)(p1 - p0) > WARP_MAX) return;  // written by k_cta_rows / k_hub_fix
       const float o = __fmul_rn(res[q], alpha);
       y[v.r0 + q] = o;
-      if (SS) ssacc += (double)o * (double)o;
     };
 #pragma unroll
     for (int u = 0; u < RPF; ++u) {
@@ -412,16 +404,6 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
     }
     for (int q = tid + RPF * PT_THREADS; q < nr; q += PT_THREADS)
       emit(q, rp[v.r0 + q], rp[v.r0 + q + 1]);
-    if (SS) {
-      ssacc = warp_sum_d(ssacc);
-      if (lane == 0) S.wss[warp] = ssacc;
-      __syncthreads();
-      if (tid == 0) {
-        double a = 0.0;
-        for (int w = 0; w < PT_THREADS / 32; ++w) a += S.wss[w];
-        tile_ss[t] = a;
-      }
-    }
     __syncthreads();
     v = vn;
     if (t + 2 < k1) vn = view(desc[t + 2]);
@@ -463,35 +445,35 @@ __device__ __forceinline__ float strided_sum(const int32_t* __restrict__ cc,
 #pragma unroll
       for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
     }
-    return s;
-  }
-  int c[UNR];
-  float v[UNR];
-#pragma unroll
-  for (int u = 0; u < UNR; ++u) {
-    const bool pu = t0 + S * u < L;
-    c[u] = pu ? lds<SM>(cc + t0 + S * u, pol) : 0;
-    v[u] = pu ? lds<SM>(vv + t0 + S * u, pol) : 0.f;
-  }
-  for (int64_t t = t0; t < L; t += S * UNR) {
-    float xv[UNR];
-#pragma unroll
-    for (int u = 0; u < UNR; ++u) xv[u] = (t + S * u < L) ? gx(x, c[u]) : 0.f;
-    const int64_t tn = t + S * UNR;
-    int cn[UNR];
-    float vn[UNR];
+  } else {
+    int c[UNR];
+    float v[UNR];
 #pragma unroll
     for (int u = 0; u < UNR; ++u) {
-      const bool pu = tn + S * u < L;
-      cn[u] = pu ? lds<SM>(cc + tn + S * u, pol) : 0;
-      vn[u] = pu ? lds<SM>(vv + tn + S * u, pol) : 0.f;
+      const bool pu = t0 + S * u < L;
+      c[u] = pu ? lds<SM>(cc + t0 + S * u, pol) : 0;
+      v[u] = pu ? lds<SM>(vv + t0 + S * u, pol) : 0.f;
     }
+    for (int64_t t = t0; t < L; t += S * UNR) {
+      float xv[UNR];
 #pragma unroll
-    for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
+      for (int u = 0; u < UNR; ++u) xv[u] = (t + S * u < L) ? gx(x, c[u]) : 0.f;
+      const int64_t tn = t + S * UNR;
+      int cn[UNR];
+      float vn[UNR];
 #pragma unroll
-    for (int u = 0; u < UNR; ++u) {
-      c[u] = cn[u];
-      v[u] = vn[u];
+      for (int u = 0; u < UNR; ++u) {
+        const bool pu = tn + S * u < L;
+        cn[u] = pu ? lds<SM>(cc + tn + S * u, pol) : 0;
+        vn[u] = pu ? lds<SM>(vv + tn + S * u, pol) : 0.f;
+      }
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) s = __fadd_rn(s, __fmul_rn(v[u], xv[u]));
+#pragma unroll
+      for (int u = 0; u < UNR; ++u) {
+        c[u] = cn[u];
+        v[u] = vn[u];
+      }
     }
   }
   return s;
@@ -523,7 +505,7 @@ __global__ void __launch_bounds__(256)
     k_warp_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                 const float* __restrict__ val, const float* __restrict__ x,
                 float* __restrict__ y, const int32_t* __restrict__ rows, int64_t nrows,
-                const double* __restrict__ ss_in, double* __restrict__ row_ss, const YDst dst) {
+                const double* __restrict__ ss_in, const YDst dst) {
   const int lane = threadIdx.x & 31;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float alpha = alpha_of(ss_in);
@@ -534,7 +516,6 @@ __global__ void __launch_bounds__(256)
     if (lane == 0) {
       const float v = __fmul_rn(s, alpha);
       store_y<SS>(y, dst, r, v);
-      if (SS) row_ss[q] = (double)v * (double)v;
     }
   }
   fence_bcast<SS>(dst);
@@ -566,7 +547,7 @@ __global__ void __launch_bounds__(256)
     k_cta_rows(const OT* __restrict__ rp, const int32_t* __restrict__ col,
                const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
                const int32_t* __restrict__ rows, const double* __restrict__ ss_in,
-               double* __restrict__ row_ss, const YDst dst) {
+               const YDst dst) {
   __shared__ float red[256];
   const int r = rows[blockIdx.x];
   const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
@@ -574,7 +555,6 @@ __global__ void __launch_bounds__(256)
   if (threadIdx.x == 0) {
     const float v = __fmul_rn(s, alpha_of(ss_in));
     store_y<SS>(y, dst, r, v);
-    if (SS) row_ss[blockIdx.x] = (double)v * (double)v;
     fence_bcast<SS>(dst);
   }
 }
@@ -599,32 +579,14 @@ template <bool SS>
 __global__ void k_hub_fix(const int32_t* __restrict__ hub_rows, const int32_t* __restrict__ choff,
                           int64_t nh, const double* __restrict__ part,
                           const double* __restrict__ ss_in, float* __restrict__ y,
-                          double* __restrict__ hub_ss, const YDst dst) {
+                          const YDst dst) {
   const int64_t h = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (h >= nh) return;
   double acc = 0.0;
   for (int c = choff[h]; c < choff[h + 1]; ++c) acc += part[c];
   const float v = __fmul_rn((float)acc, alpha_of(ss_in));
   store_y<SS>(y, dst, hub_rows[h], v);
-  if (SS) hub_ss[h] = (double)v * (double)v;
   fence_bcast<SS>(dst);
-}
-
-// Fixed-order fp64 sum of the y^2 partials (power-iteration norm).  The
-// partial arrays a | b | c | d form one virtual sequence cut into segments of
-// SS_SEG entries; CTA s sums segment s (strided per thread, then a fixed
-// tree), k_ss_final sums the segment sums in order.  The association depends
-// only on the plan's row classes, never on the grid: bitwise repeatable.
-constexpr int64_t SS_SEG = 16384;
-
-__device__ __forceinline__ double ss_at(int64_t v, const double* a, int64_t na, const double* b,
-                                        int64_t nb, const double* c, int64_t nc, const double* d) {
-  if (v < na) return a[v];
-  v -= na;
-  if (v < nb) return b[v];
-  v -= nb;
-  if (v < nc) return c[v];
-  return d[v - nc];
 }
 
 __device__ __forceinline__ double block_sum_1024(double acc, double* wss) {
@@ -639,19 +601,6 @@ __device__ __forceinline__ double block_sum_1024(double acc, double* wss) {
 }
 
 __global__ void __launch_bounds__(1024)
-    k_ss_part(const double* __restrict__ a, int64_t na, const double* __restrict__ b, int64_t nb,
-              const double* __restrict__ c, int64_t nc, const double* __restrict__ d, int64_t nd,
-              double* __restrict__ part) {
-  __shared__ double wss[32];
-  const int64_t tot = na + nb + nc + nd;
-  const int64_t v0 = (int64_t)blockIdx.x * SS_SEG, v1 = min(tot, v0 + SS_SEG);
-  double acc = 0.0;
-  for (int64_t v = v0 + threadIdx.x; v < v1; v += 1024) acc += ss_at(v, a, na, b, nb, c, nc, d);
-  const double sblk = block_sum_1024(acc, wss);
-  if (threadIdx.x == 0) part[blockIdx.x] = sblk;
-}
-
-__global__ void __launch_bounds__(1024)
     k_ss_final(const double* __restrict__ part, int64_t np, double* __restrict__ out) {
   __shared__ double wss[32];
   double acc = 0.0;
@@ -660,11 +609,31 @@ __global__ void __launch_bounds__(1024)
   if (threadIdx.x == 0) *out = s;
 }
 
-void ss_reduce(spmv_plan_s* p, const double* a, int64_t na, const double* b, int64_t nb,
-               const double* c, int64_t nc, const double* d, int64_t nd, double* out,
-               cudaStream_t s) {
-  const int64_t np = std::max<int64_t>(1, (na + nb + nc + nd + SS_SEG - 1) / SS_SEG);
-  k_ss_part<<<(unsigned)np, 1024, 0, s>>>(a, na, b, nb, c, nc, d, nd, p->d_ss_part);
+// Power-iteration norm (reading c22): sum of y^2 in fp64 over this rank's y
+// slice in fixed segments of SS_ROWS rows (one CTA each: strided per thread,
+// then a fixed tree), then the segment sums in order -- the association
+// depends only on the row count, never on the grid or the row classes, so
+// the norm is bitwise repeatable.  One coalesced read of y (4 B per row)
+// replaces round 1's fp64 partial per row / warp stored by the SpMV kernels,
+// whose scattered 8-byte stores cost the step ~0.7 ms on Kronecker-28 (r72).
+constexpr int64_t SS_ROWS = 16384;
+
+__global__ void __launch_bounds__(1024)
+    k_ss_y(const float* __restrict__ y, int64_t n, double* __restrict__ part) {
+  __shared__ double wss[32];
+  const int64_t v0 = (int64_t)blockIdx.x * SS_ROWS, v1 = min(n, v0 + SS_ROWS);
+  double acc = 0.0;
+  for (int64_t v = v0 + threadIdx.x; v < v1; v += 1024) {
+    const double t = (double)y[v];
+    acc += t * t;
+  }
+  const double sblk = block_sum_1024(acc, wss);
+  if (threadIdx.x == 0) part[blockIdx.x] = sblk;
+}
+
+void ss_reduce_y(spmv_plan_s* p, const float* y, double* out, cudaStream_t s) {
+  const int64_t np = std::max<int64_t>(1, (p->nrows + SS_ROWS - 1) / SS_ROWS);
+  k_ss_y<<<(unsigned)np, 1024, 0, s>>>(y, p->nrows, p->d_ss_part);
   k_ss_final<<<1, 1024, 0, s>>>(p->d_ss_part, np, out);
 }
 
@@ -701,7 +670,7 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
   const int use_win = p->opts.smem_window ? 1 : 0;
   k_panel<OT, SS><<<grid, PT_THREADS, smem, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
                                                  p->d_desc, p->K, p->y_offset, p->x_len, use_win,
-                                                 ss_in, p->d_tile_ss, p->opts.evict_first);
+                                                 ss_in, p->opts.evict_first);
 }
 
 // --------------------------------------------------------- lane-per-row
@@ -718,7 +687,6 @@ void launch_panel(spmv_plan_s* p, const float* x, float* y, const double* ss_in,
 // stream hints ran 1.25x slower than this plain form on SBM 4M/64M.
 constexpr int LN_THREADS = 256;
 constexpr int MID_STREAM_DEFAULT = 0;  // stream-load mode of the MID / CTA / hub kernels (lds)
-constexpr int LN_WARPS = LN_THREADS / 32;
 constexpr int LN_CTAS_PER_SM = 32;  // grid = min(blocks, SMs x this)
 
 // 256-bit streaming loads of one 8-entry chunk, not allocated in L1.
@@ -805,14 +773,6 @@ __device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
   return res;
 }
 
-// fixed-order sum of y^2 of one warp's 32 rows (xor tree), stored as partial
-// (blk, warp) -- no CTA barrier in the lane kernels; the partials of a
-// 256-row block are then eight consecutive entries of the plan's partial
-// array, summed with everything else by ss_reduce in a grid-independent order
-__device__ __forceinline__ void warp_ss(double ssacc, double* out) {
-  ssacc = warp_sum_d(ssacc);
-  if ((threadIdx.x & 31) == 0) out[threadIdx.x >> 5] = ssacc;
-}
 
 // minBlocksPerSM = 1 lets ptxas keep both chunks and all 16 gathers of a
 // 16-entry row in flight per lane (64 registers, 4 CTAs/SM); capping registers
@@ -821,10 +781,10 @@ __device__ __forceinline__ void warp_ss(double ssacc, double* out) {
 // 3 CTAs per SM and costs 22 % (r66: 4.45 vs 3.64 ms on C5): both variants
 // are held to 64 registers, 4 CTAs per SM
 template <typename OT, bool SS, int EF>
-__global__ void __launch_bounds__(LN_THREADS, (SS || SPMV_PRED_MINB4 && (EF & 8)) ? 4 : 1)
+__global__ void __launch_bounds__(LN_THREADS, SS ? 4 : 1)
     k_lane(const OT* __restrict__ rp, const int32_t* __restrict__ col,
            const float* __restrict__ val, const float* __restrict__ x, float* __restrict__ y,
-           int64_t nrows, const double* __restrict__ ss_in, double* __restrict__ blk_ss,
+           int64_t nrows, const double* __restrict__ ss_in,
            const YDst dst) {
   const int tid = threadIdx.x;
   const int64_t NB = (nrows + LN_THREADS - 1) / LN_THREADS;
@@ -862,13 +822,7 @@ __global__ void __launch_bounds__(LN_THREADS, (SS || SPMV_PRED_MINB4 && (EF & 8)
         res = lane_row_sum<OT, EF>(col, val, x, a, L);
       }
     }
-    double ssacc = 0.0;
-    if (mine) {
-      const float o = __fmul_rn(res, alpha);
-      store_y<SS>(y, dst, r, o);
-      if (SS) ssacc = (double)o * (double)o;
-    }
-    if (SS) warp_ss(ssacc, blk_ss + blk * LN_WARPS);
+    if (mine) store_y<SS>(y, dst, r, __fmul_rn(res, alpha));
   }
   fence_bcast<SS>(dst);
 }
@@ -891,27 +845,25 @@ __global__ void __launch_bounds__(LN_THREADS)
             int64_t nrows, const int32_t* __restrict__ mid_rows, int64_t n_mid,
             const int32_t* __restrict__ mid_wide, int64_t n_wide,
             const int32_t* __restrict__ cta_rows, int64_t B_lane, int64_t B_mid,
-            const double* __restrict__ ss_in, double* __restrict__ blk_ss,
-            double* __restrict__ mid_ss, double* __restrict__ cta_ss, const YDst dst) {
+            const double* __restrict__ ss_in, const YDst dst) {
   __shared__ float red[256];
   __shared__ float prod[WARP_MAX];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const float alpha = alpha_of(ss_in);
-  const int64_t blk = blockIdx.x;
+  // the long rows (wide MID, CTA rows) are dispatched first: blocks
+  // [0, n_long) take roles B_lane + B_mid + ..., so the critical path starts
+  // in the first wave instead of after the lane and MID blocks
+  const int64_t tail0 = B_lane + B_mid, n_long = (int64_t)gridDim.x - tail0;
+  const int64_t blk = (int64_t)blockIdx.x < n_long ? tail0 + blockIdx.x : blockIdx.x - n_long;
   const uint64_t pol = stream_policy<SM>();
   if (blk < B_lane) {  // block-uniform branches
     const int64_t r = blk * LN_THREADS + tid;
-    double ssacc = 0.0;
     if (r < nrows) {
       const OT a = rp[r];
       const int L = (int)(rp[r + 1] - a);
-      if (L <= SHORT_MAX) {
-        const float o = __fmul_rn(lane_row_sum<OT, EF>(col, val, x, a, L), alpha);
-        store_y<SS>(y, dst, r, o);
-        if (SS) ssacc = (double)o * (double)o;
-      }
+      if (L <= SHORT_MAX)
+        store_y<SS>(y, dst, r, __fmul_rn(lane_row_sum<OT, EF>(col, val, x, a, L), alpha));
     }
-    if (SS) warp_ss(ssacc, blk_ss + blk * LN_WARPS);
   } else if (blk < B_lane + B_mid) {
     const int64_t q = (blk - B_lane) * 8 + warp;
     if (q < n_mid) {
@@ -920,11 +872,7 @@ __global__ void __launch_bounds__(LN_THREADS)
       const int L = (int)((int64_t)rp[r + 1] - b);
       if (L <= MID_WIDE) {  // (wide rows: their own CTA below)
         const float s = warp_row_sum_bl<SM, 8, true>(col, val, x, b, L, lane, pol);
-        if (lane == 0) {
-          const float v = __fmul_rn(s, alpha);
-          store_y<SS>(y, dst, r, v);
-          if (SS) mid_ss[q] = (double)v * (double)v;
-        }
+        if (lane == 0) store_y<SS>(y, dst, r, __fmul_rn(s, alpha));
       }
     }
   } else if (blk < B_lane + B_mid + n_wide) {
@@ -957,22 +905,14 @@ __global__ void __launch_bounds__(LN_THREADS)
         for (int u = 0; u < 8; ++u) s = __fadd_rn(s, pv[u]);
       }
       s = warp_tree(s);
-      if (lane == 0) {
-        const float o = __fmul_rn(s, alpha);
-        store_y<SS>(y, dst, r, o);
-        if (SS) mid_ss[q] = (double)o * (double)o;
-      }
+      if (lane == 0) store_y<SS>(y, dst, r, __fmul_rn(s, alpha));
     }
   } else {
     const int64_t i = blk - B_lane - B_mid - n_wide;
     const int r = cta_rows[i];
     const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
     const float s = cta_sum256<SM, 8, true>(col, val, x, b, L, red);
-    if (tid == 0) {
-      const float v = __fmul_rn(s, alpha);
-      store_y<SS>(y, dst, r, v);
-      if (SS) cta_ss[i] = (double)v * (double)v;
-    }
+    if (tid == 0) store_y<SS>(y, dst, r, __fmul_rn(s, alpha));
   }
   fence_bcast<SS>(dst);
 }
@@ -988,7 +928,7 @@ void launch_lane_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in
   const int64_t cap = (int64_t)num_sms(p->device) * per_sm;
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min(NB, cap));
   k_lane<OT, SS, EF><<<grid, LN_THREADS, 0, s>>>((const OT*)p->d_rp, p->d_col, p->d_val, x, y,
-                                                   p->nrows, ss_in, p->d_blk_ss, dst);
+                                                   p->nrows, ss_in, dst);
 }
 
 }  // namespace
@@ -1035,20 +975,19 @@ void launch_rows_t(spmv_plan_s* p, const float* x, float* y, const double* ss_in
   const int32_t* col = p->d_col;
   const int64_t nw = lane_mode ? p->n_mid : p->n_warp;
   const int32_t* wr = lane_mode ? p->d_mid_rows : p->d_warp_rows;
-  double* wss = lane_mode ? p->d_mid_ss : p->d_warp_ss;
   if (nw) {
     const unsigned g = (unsigned)std::min<int64_t>((nw + 7) / 8, (int64_t)num_sms(p->device) * 16);
-    k_warp_rows<OT, SS, SM><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, wss, dst);
+    k_warp_rows<OT, SS, SM><<<g, 256, 0, s1>>>(rp, col, p->d_val, x, y, wr, nw, ss_in, dst);
   }
   if (p->n_cta)
     k_cta_rows<OT, SS, SM><<<(unsigned)p->n_cta, 256, 0, s2>>>(rp, col, p->d_val, x, y,
-                                                              p->d_cta_rows, ss_in, p->d_cta_ss, dst);
+                                                              p->d_cta_rows, ss_in, dst);
   if (p->n_chunks) {
     k_hub_chunk<OT, SM><<<(unsigned)p->n_chunks, 256, 0, s2>>>(
         rp, col, p->d_val, x, p->d_chunk_row, p->d_chunk_idx, p->d_chunk_part);
     const unsigned g = (unsigned)((p->n_hub + 127) / 128);
     k_hub_fix<SS><<<g, 128, 0, s2>>>(p->d_hub_rows, p->d_hub_choff, p->n_hub, p->d_chunk_part,
-                                      ss_in, y, p->d_hub_ss, dst);
+                                      ss_in, y, dst);
   }
 }
 
@@ -1091,7 +1030,7 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
 #define SPMV_SMALL_ARGS                                                                      \
   rp, p->d_col, p->d_val, x, y, p->nrows, p->d_mid_rows, p->n_mid, p->d_mid_wide, p->n_mid_wide,  \
       p->d_cta_rows, B_lane, B_mid,                                                                \
-      ss_in, p->d_blk_ss, p->d_mid_ss, p->d_cta_ss, dst
+      ss_in, dst
     const int ef = (lane_ef_mode(p) == 1 ? 1 : 0) | (p->val_nonfinite ? 4 : 0) |
                    (lane_pred_mode(p) ? 8 : 0);
 #define SPMV_SMALL_EF(SSV)                                                                 \
@@ -1109,8 +1048,7 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
   } while (0)
     if (SS) {
       SPMV_SMALL_EF(true);
-      ss_reduce(p, p->d_blk_ss, B_lane * LN_WARPS, p->d_mid_ss, p->n_mid, p->d_cta_ss, p->n_cta,
-                p->d_hub_ss, 0, ss_out, s);
+      ss_reduce_y(p, dst.n ? dst.p[p->rank] : y, ss_out, s);
     } else {
       SPMV_SMALL_EF(false);
     }
@@ -1151,14 +1089,7 @@ void exec_typed(spmv_plan_s* p, const float* x, float* y, const double* ss_in, d
     SPMV_CUDA(cudaStreamWaitEvent(s, p->ev_join[0], 0));
     SPMV_CUDA(cudaStreamWaitEvent(s, p->ev_join[1], 0));
   }
-  if (SS) {
-    if (lane_mode)
-      ss_reduce(p, p->d_blk_ss, (p->nrows + LN_THREADS - 1) / LN_THREADS * LN_WARPS, p->d_mid_ss,
-                p->n_mid, p->d_cta_ss, p->n_cta, p->d_hub_ss, p->n_hub, ss_out, s);
-    else
-      ss_reduce(p, p->d_tile_ss, p->K, p->d_warp_ss, p->n_warp, p->d_cta_ss, p->n_cta,
-                p->d_hub_ss, p->n_hub, ss_out, s);
-  }
+  if (SS) ss_reduce_y(p, dst.n ? dst.p[p->rank] : y, ss_out, s);
   SPMV_LAUNCH_CHECK();
 }
 
@@ -1293,6 +1224,8 @@ void exec(spmv_plan_s* p, const float* x, float* y, const double* ss_in, double*
       dst.p[k] = bcast[k] + p->y_offset;
     }
     dst.n = nbcast;
+    if (ss_out && p->rank >= nbcast)
+      SPMV_FAIL(SPMV_EINVAL, "bcast: x_next[rank] must be this rank's own buffer (the norm reads it)");
   }
   ensure_aux(p);
   set_window(p, x, s);

@@ -404,51 +404,94 @@ __device__ __forceinline__ void lane_bitonic(uint64_t& key, float& v, int gl) {
   }
 }
 
-// Warp bitonic sort of up to 32 * E keys in registers: element i = k * 32 +
-// lane lives in register k of lane `lane`; partners i ^ j with j >= 32 are in
-// the same lane (registers k, k ^ j/32), with j < 32 in lane ^ j (shuffles).
-// Ascending within blocks of size kk where (i & kk) == 0, as lane_bitonic.
+// Register bitonic networks.  Element g = base + k * 32 + lane lives in
+// register k of lane `lane` of a warp; a warp holds 32 * E consecutive
+// elements.  A compare-exchange stage (block size kk, distance j) orders the
+// pair (g, g ^ j) ascending when (g & kk) == 0: partners j >= 32 are in the
+// same lane (registers k, k ^ j/32), j < 32 in lane ^ j (shuffles).
 template <int E>
-__device__ __forceinline__ void warp_bitonic(uint64_t (&key)[E], float (&v)[E], int lane) {
+__device__ __forceinline__ void warp_stage(uint64_t (&key)[E], float (&v)[E], int lane, int base,
+                                           int kk, int j) {
+  if (j >= 32) {
+    const int jr = j >> 5;
+#pragma unroll
+    for (int k = 0; k < E; ++k) {
+      const int pk = k ^ jr;
+      if (pk > k) {
+        const bool asc = ((base + (k << 5) + lane) & kk) == 0;
+        if ((key[k] > key[pk]) == asc) {
+          const uint64_t tk = key[k];
+          key[k] = key[pk];
+          key[pk] = tk;
+          const float tv = v[k];
+          v[k] = v[pk];
+          v[pk] = tv;
+        }
+      }
+    }
+  } else {
+#pragma unroll
+    for (int k = 0; k < E; ++k) {
+      const uint64_t ok = __shfl_xor_sync(0xffffffffu, key[k], j);
+      const float ov = __shfl_xor_sync(0xffffffffu, v[k], j);
+      const int g = base + (k << 5) + lane;
+      const bool take_min = ((g & j) == 0) == ((g & kk) == 0);
+      if (take_min == (ok < key[k])) {
+        key[k] = ok;
+        v[k] = ov;
+      }
+    }
+  }
+}
+
+// full bitonic sort of a warp's 32 * E keys (blocks up to 32 * E; with a
+// nonzero base, blocks alternate direction by (g & kk) as in a CTA-wide sort)
+template <int E>
+__device__ __forceinline__ void warp_bitonic(uint64_t (&key)[E], float (&v)[E], int lane,
+                                             int base = 0) {
   constexpr int LOG = E == 4 ? 7 : 8;  // 32 * E = 2^LOG keys
   static_assert(E == 4 || E == 8, "warp_bitonic: 4 or 8 keys per lane");
 #pragma unroll
   for (int lk = 1; lk <= LOG; ++lk) {  // counted loops: fully unrolled, registers stay registers
-    const int kk = 1 << lk;
 #pragma unroll
-    for (int lj = lk - 1; lj >= 0; --lj) {
-      const int j = 1 << lj;
-      if (j >= 32) {
-        const int jr = j >> 5;
+    for (int lj = lk - 1; lj >= 0; --lj) warp_stage<E>(key, v, lane, base, 1 << lk, 1 << lj);
+  }
+}
+
+// CTA bitonic sort of NW * 256 keys (NW warps of 8 keys per lane): blocks up
+// to 256 inside each warp, then for every larger block size kk the distances
+// j >= 256 through shared memory (each thread keeps min or max of its element
+// and the partner's, two barriers per stage) and j < 256 inside the warp.
+// ~10 barriers for 4096 keys instead of the 78 of a shared-memory network.
+template <int NW>
+__device__ __forceinline__ void cta_bitonic_regs(uint64_t (&key)[8], float (&v)[8],
+                                                 uint64_t* sk, float* sv) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, base = w * 256;
+  warp_bitonic<8>(key, v, lane, base);
+#pragma unroll 1
+  for (int kk = 512; kk <= NW * 256; kk <<= 1) {
+#pragma unroll 1
+    for (int j = kk >> 1; j >= 256; j >>= 1) {
 #pragma unroll
-        for (int k = 0; k < E; ++k) {
-          const int pk = k ^ jr;
-          if (pk > k) {
-            const bool asc = (((k << 5) | lane) & kk) == 0;
-            if ((key[k] > key[pk]) == asc) {
-              const uint64_t tk = key[k];
-              key[k] = key[pk];
-              key[pk] = tk;
-              const float tv = v[k];
-              v[k] = v[pk];
-              v[pk] = tv;
-            }
-          }
-        }
-      } else {
+      for (int k = 0; k < 8; ++k) {
+        sk[base + (k << 5) + lane] = key[k];
+        sv[base + (k << 5) + lane] = v[k];
+      }
+      __syncthreads();
 #pragma unroll
-        for (int k = 0; k < E; ++k) {
-          const uint64_t ok = __shfl_xor_sync(0xffffffffu, key[k], j);
-          const float ov = __shfl_xor_sync(0xffffffffu, v[k], j);
-          const int i = (k << 5) | lane;
-          const bool take_min = ((i & j) == 0) == ((i & kk) == 0);
-          if (take_min == (ok < key[k])) {
-            key[k] = ok;
-            v[k] = ov;
-          }
+      for (int k = 0; k < 8; ++k) {
+        const int g = base + (k << 5) + lane;
+        const uint64_t ok = sk[g ^ j];
+        const bool take_min = ((g & j) == 0) == ((g & kk) == 0);
+        if (take_min == (ok < key[k])) {
+          key[k] = ok;
+          v[k] = sv[g ^ j];
         }
       }
+      __syncthreads();
     }
+#pragma unroll
+    for (int lj = 7; lj >= 0; --lj) warp_stage<8>(key, v, lane, base, kk, 1 << lj);
   }
 }
 
@@ -601,56 +644,37 @@ __global__ void k_relabel_cta(const AT* rpA, const int32_t* colA, const float* v
 }
 
 // ----------------------------------------------------------------- row sort
-// CTA bitonic sort of one row of length L <= pe held in shared memory, pe =
-// the next power of two >= L (>= 64), <= P: the network is sized to the row,
-// not to the class bound (a 130-entry row sorts 256 keys, not 1024).
-template <int P>
-__device__ void smem_bitonic(uint64_t* keys, float* vals, int pe) {
-#pragma unroll 1
-  for (int k = 2; k <= pe; k <<= 1) {
-#pragma unroll 1
-    for (int j = k >> 1; j > 0; j >>= 1) {
-      for (int i = threadIdx.x; i < pe; i += blockDim.x) {
-        int ixj = i ^ j;
-        if (ixj > i) {
-          uint64_t a = keys[i], b = keys[ixj];
-          bool asc = (i & k) == 0;
-          if ((a > b) == asc) {
-            keys[i] = b;
-            keys[ixj] = a;
-            float t = vals[i];
-            vals[i] = vals[ixj];
-            vals[ixj] = t;
-          }
-        }
-      }
-      __syncthreads();
-    }
-  }
-}
-
+// one row of 256 < L <= P keys per CTA iteration, P / 256 warps of 8 keys
+// per lane sorted in registers (cta_bitonic_regs), shared memory only for the
+// cross-warp distances
 template <int P, typename OT>
-__global__ void k_sort_cta(const OT* rp, const int32_t* rows, int64_t nlist, int32_t* col,
-                           float* val) {
+__global__ void __launch_bounds__(P / 8)
+    k_sort_cta(const OT* rp, const int32_t* rows, int64_t nlist, int32_t* col, float* val) {
   extern __shared__ __align__(16) unsigned char sm[];
-  uint64_t* keys = (uint64_t*)sm;
-  float* vals = (float*)(keys + P);
+  uint64_t* sk = (uint64_t*)sm;
+  float* sv = (float*)(sk + P);
+  const int lane = threadIdx.x & 31, base = (threadIdx.x >> 5) * 256;
   for (int64_t t = blockIdx.x; t < nlist; t += gridDim.x) {
-    int64_t r = rows[t];
-    int64_t d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d;
-    int pe = 64;
-    while (pe < L) pe <<= 1;
-    for (int i = threadIdx.x; i < pe; i += blockDim.x) {
-      keys[i] = i < L ? mkkey(col[d + i], i) : ~0ull;
-      vals[i] = i < L ? val[d + i] : 0.f;
+    const int64_t r = rows[t];
+    const int64_t d = (int64_t)rp[r], L = (int64_t)rp[r + 1] - d;
+    uint64_t key[8];
+    float v[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int i = base + (k << 5) + lane;
+      key[k] = i < L ? mkkey(col[d + i], i) : ~0ull;
+      v[k] = i < L ? val[d + i] : 0.f;
     }
-    __syncthreads();
-    smem_bitonic<P>(keys, vals, pe);
-    for (int i = threadIdx.x; i < L; i += blockDim.x) {
-      col[d + i] = (int32_t)(keys[i] >> 32);
-      val[d + i] = vals[i];
+    cta_bitonic_regs<P / 256>(key, v, sk, sv);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int i = base + (k << 5) + lane;
+      if (i < L) {
+        col[d + i] = (int32_t)(key[k] >> 32);
+        val[d + i] = v[k];
+      }
     }
-    __syncthreads();
+    __syncthreads();  // (the next row reuses the exchange buffer)
   }
 }
 
@@ -669,24 +693,33 @@ __global__ void k_big_load(const OT* rp, const int32_t* rows, const int64_t* bof
   }
 }
 
-// sort every BIG_CHUNK-run of every big row in shared memory (one CTA per
-// tile of the plan's tile list: no empty CTAs for the short big rows)
-__global__ void k_big_chunk_sort(const BigTile* tiles, uint64_t* K, float* V) {
+// sort every BIG_CHUNK-run of every big row (one CTA of 16 warps per tile of
+// the plan's tile list: no empty CTAs for the short big rows), in registers
+__global__ void __launch_bounds__(BIG_CHUNK / 8) k_big_chunk_sort(const BigTile* tiles, uint64_t* K,
+                                                                  float* V) {
   extern __shared__ __align__(16) unsigned char sm[];
-  uint64_t* keys = (uint64_t*)sm;
-  float* vals = (float*)(keys + BIG_CHUNK);
+  uint64_t* sk = (uint64_t*)sm;
+  float* sv = (float*)(sk + BIG_CHUNK);
   const BigTile t = tiles[blockIdx.x];
   const int64_t e0 = t.o + t.q;
   const int64_t m = min((int64_t)BIG_CHUNK, t.L - t.q);
-  for (int i = threadIdx.x; i < BIG_CHUNK; i += blockDim.x) {
-    keys[i] = i < m ? K[e0 + i] : ~0ull;
-    vals[i] = i < m ? V[e0 + i] : 0.f;
+  const int lane = threadIdx.x & 31, base = (threadIdx.x >> 5) * 256;
+  uint64_t key[8];
+  float v[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const int i = base + (k << 5) + lane;
+    key[k] = i < m ? K[e0 + i] : ~0ull;
+    v[k] = i < m ? V[e0 + i] : 0.f;
   }
-  __syncthreads();
-  smem_bitonic<BIG_CHUNK>(keys, vals, BIG_CHUNK);
-  for (int i = threadIdx.x; i < m; i += blockDim.x) {
-    K[e0 + i] = keys[i];
-    V[e0 + i] = vals[i];
+  cta_bitonic_regs<BIG_CHUNK / 256>(key, v, sk, sv);
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const int i = base + (k << 5) + lane;
+    if (i < m) {
+      K[e0 + i] = key[k];
+      V[e0 + i] = v[k];
+    }
   }
 }
 
@@ -1106,18 +1139,8 @@ static void build_typed(spmv_plan_s* p, const AT* rpA) {
   SPMV_CUDA(cudaMemsetAsync(p->d_val + p->nnz_local, 0, 32, s));
   // exec scratch
   p->d_chunk_part = dalloc<double>(p->n_chunks);
-  p->d_tile_ss = dalloc<double>(p->K);
-  p->d_blk_ss = dalloc<double>((nr + 255) / 256 * 8 + 8);  // one per warp of each 256-row block
-  p->d_warp_ss = dalloc<double>(p->n_warp);
-  p->d_mid_ss = dalloc<double>(p->n_mid);
-  p->d_cta_ss = dalloc<double>(p->n_cta);
-  p->d_hub_ss = dalloc<double>(p->n_hub);
   p->d_ss = dalloc<double>(4);
-  {  // segment sums of the norm reduction (exec.cu ss_reduce), either row scheme
-    const int64_t lane_parts = (nr + 255) / 256 * 8 + p->n_mid + p->n_cta + p->n_hub;
-    const int64_t tile_parts = p->K + p->n_warp + p->n_cta + p->n_hub;
-    p->d_ss_part = dalloc<double>(std::max(lane_parts, tile_parts) / 16384 + 2);
-  }
+  p->d_ss_part = dalloc<double>(nr / 16384 + 2);  // norm segment sums (exec.cu SS_ROWS rows each)
   SPMV_CUDA(cudaStreamSynchronize(s));
 }
 
@@ -1141,7 +1164,7 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
           rp, p->d_col, p->d_val);
     SPMV_LAUNCH_CHECK();
     if (ps->n2) {
-      k_sort_cta<1024, OT><<<(unsigned)std::min<int64_t>(ps->n2, 148 * 16), 256, 1024 * 12, s>>>(
+      k_sort_cta<1024, OT><<<(unsigned)std::min<int64_t>(ps->n2, 148 * 16), 128, 1024 * 12, s>>>(
           rp, ps->s2, ps->n2, p->d_col, p->d_val);
     }
     if (ps->n3) {
@@ -1156,7 +1179,7 @@ static void permute_typed(spmv_plan_s* p, const AT* rpA, cudaStream_t s) {
       float* V2 = dalloc<float>(ps->big_total);
       unsigned nb = (unsigned)std::min<int64_t>(ps->nbig, 148 * 8);
       k_big_load<OT><<<nb, 512, 0, s>>>(rp, ps->big, ps->boff, ps->nbig, p->d_col, p->d_val, K1, V1);
-      k_big_chunk_sort<<<(unsigned)ps->nbtile, 512, BIG_CHUNK * 12, s>>>(ps->btile, K1, V1);
+      k_big_chunk_sort<<<(unsigned)ps->nbtile, BIG_CHUNK / 8, BIG_CHUNK * 12, s>>>(ps->btile, K1, V1);
       SPMV_LAUNCH_CHECK();
       int64_t* split = dalloc<int64_t>(ps->nbtile);
       for (int64_t w = BIG_CHUNK; w < ps->big_max; w *= 2) {
@@ -1353,11 +1376,11 @@ void plan_free(spmv_plan_s* p) {
   dfree(p->d_perm); dfree(p->d_inv); dfree(p->d_srcA);
   if (p->d_rp) { cudaFree(p->d_rp); p->d_rp = nullptr; }
   dfree(p->d_col); dfree(p->d_val); dfree(p->d_tiles); dfree(p->d_cta_rows); dfree(p->d_desc);
-  dfree(p->d_warp_rows); dfree(p->d_warp_ss); dfree(p->d_mid_rows); dfree(p->d_mid_ss);
+  dfree(p->d_warp_rows); dfree(p->d_mid_rows);
   dfree(p->d_mid_wide);
   dfree(p->d_chunk_part4);
   dfree(p->d_hub_rows); dfree(p->d_hub_choff); dfree(p->d_chunk_row); dfree(p->d_chunk_idx);
-  dfree(p->d_chunk_part); dfree(p->d_tile_ss); dfree(p->d_blk_ss); dfree(p->d_cta_ss); dfree(p->d_hub_ss);
+  dfree(p->d_chunk_part);
   dfree(p->d_ss); dfree(p->d_u); dfree(p->d_ss_part);
   for (int i = 0; i < 2; ++i) {
     if (p->aux[i]) { cudaStreamDestroy(p->aux[i]); p->aux[i] = nullptr; }

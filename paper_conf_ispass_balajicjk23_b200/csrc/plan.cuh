@@ -79,14 +79,8 @@ struct spmv_plan_s {
   double* d_coo_tpart = nullptr;   // [2 coo_tiles] fp64 pieces (first / last row)
   uint8_t* d_coo_tflag = nullptr;  // [coo_tiles]
   bool coo_memset = false;         // a run of > 32 empty rows: memset y, no in-kernel zeroing
-  double* d_tile_ss = nullptr;     // [K]
-  double* d_blk_ss = nullptr;      // [ceil(nrows/64)] per-block sumsq (lane variant)
-  double* d_warp_ss = nullptr;     // [n_warp]
-  double* d_mid_ss = nullptr;      // [n_mid]
-  double* d_cta_ss = nullptr;      // [n_cta]
-  double* d_hub_ss = nullptr;      // [n_hub]
   double* d_ss = nullptr;          // [4] iterate scalars
-  double* d_ss_part = nullptr;     // segment sums of the norm reduction
+  double* d_ss_part = nullptr;     // [nrows / 16384 + 2] segment sums of the norm (Σy² over y)
   float* d_u = nullptr;            // iterate ping-pong [x_len]
 
   // permute-phase sort buckets (ascending local rows)
