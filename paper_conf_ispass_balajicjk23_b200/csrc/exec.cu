@@ -1122,9 +1122,8 @@ void set_window_one(spmv_plan_s* p, const float* x, cudaStream_t s, int slot) {
   }
   // spmv_iterate reads x from two buffers in turn: both windows must fit the
   // persisting carve-out at once, or each step evicts the other's lines
-  bool halve = p->win_alternating;
-  if (const char* e = getenv("SPMV_WIN_ALT_FULL")) if (atoi(e)) halve = false;  // dev knob (A/B)
-  if (halve) bytes = std::min<int64_t>(bytes, (int64_t)maxpers / 2);
+  // (r74: the same step time as one full-size window, within noise)
+  if (p->win_alternating) bytes = std::min<int64_t>(bytes, (int64_t)maxpers / 2);
   if (const char* e = getenv("SPMV_WIN_HIT")) hit = std::min(1.0, std::max(0.0, atof(e)));  // dev knob
   if (bytes <= 0) return;
   size_t cur = 0;
