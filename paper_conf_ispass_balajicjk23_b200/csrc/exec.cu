@@ -419,8 +419,9 @@ __global__ void __launch_bounds__(PT_THREADS, 2)
 // UNR entries are loaded before the x gathers of the current ones are
 // consumed, so an iteration costs one memory round trip (the gathers), not
 // two -- what a latency-bound launch needs (k_small: RMAT-16 16.3 -> 14.2 us,
-// r68/r69); the throughput-bound class kernels keep the plain loop (r69: the
-// pipelined warp rows cost 4 % on Kronecker-28, within noise on RMAT-26).
+// r68/r69) and what the one-CTA-per-row / per-chunk kernels gain from (r76,
+// Kronecker-28 serialised: k_cta_rows 2.79 -> 2.71 ms, k_hub_chunk 3.11 ->
+// 3.05 ms); the warp rows keep the plain loop (r69: pipelined, 4 % slower).
 // The ragged end is guarded: a slot past the row has v = x = 0 and adds +0,
 // which leaves s unchanged (s starts at +0 and is never -0), so the
 // association is exactly t0, t0 + S, t0 + 2S, ... for every UNR and PIPE.
@@ -551,7 +552,7 @@ __global__ void __launch_bounds__(256)
   __shared__ float red[256];
   const int r = rows[blockIdx.x];
   const int64_t b = (int64_t)rp[r], L = (int64_t)rp[r + 1] - b;
-  const float s = cta_sum256<SM, UNR>(col, val, x, b, L, red);
+  const float s = cta_sum256<SM, UNR, true>(col, val, x, b, L, red);
   if (threadIdx.x == 0) {
     const float v = __fmul_rn(s, alpha_of(ss_in));
     store_y<SS>(y, dst, r, v);
@@ -571,7 +572,7 @@ __global__ void __launch_bounds__(256)
   const int64_t rb = (int64_t)rp[r], L = (int64_t)rp[r + 1] - rb;
   const int64_t b = rb + (int64_t)chunk_idx[c] * HUB_CHUNK;
   const int64_t m = min((int64_t)HUB_CHUNK, rb + L - b);
-  const float s = cta_sum256<SM, UNR>(col, val, x, b, m, red);
+  const float s = cta_sum256<SM, UNR, true>(col, val, x, b, m, red);
   if (threadIdx.x == 0) part[c] = (double)s;
 }
 
