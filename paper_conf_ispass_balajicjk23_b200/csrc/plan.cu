@@ -777,9 +777,13 @@ __global__ void __launch_bounds__(MT_THREADS)
   const int64_t m = d1 - d;
   const int64_t out0 = t.o + base + d;
   if (nB == 0) {  // unpaired last run: already sorted, copy
-    for (int64_t k = threadIdx.x; k < m; k += MT_THREADS) {
-      K2[out0 + k] = K[out0 + k];
-      V2[out0 + k] = V[out0 + k];
+#pragma unroll
+    for (int u = 0; u < MT_PER; ++u) {  // (unrolled: every load of the tile in flight)
+      const int k = threadIdx.x + u * MT_THREADS;
+      if (k < m) {
+        K2[out0 + k] = K[out0 + k];
+        V2[out0 + k] = V[out0 + k];
+      }
     }
     return;
   }
@@ -790,13 +794,14 @@ __global__ void __launch_bounds__(MT_THREADS)
   const int na = (int)(i1 - i0), nb = (int)(j1 - j0);
   const uint64_t* A = K + t.o + base;
   const float* AV = V + t.o + base;
-  for (int k = threadIdx.x; k < na; k += MT_THREADS) {
-    sk[k] = A[i0 + k];
-    sv[k] = AV[i0 + k];
-  }
-  for (int k = threadIdx.x; k < nb; k += MT_THREADS) {
-    sk[na + k] = A[w + j0 + k];
-    sv[na + k] = AV[w + j0 + k];
+#pragma unroll
+  for (int u = 0; u < MT_PER; ++u) {  // the A piece then the B piece, all loads in flight
+    const int k = threadIdx.x + u * MT_THREADS;
+    if (k < m) {
+      const int64_t g = k < na ? i0 + k : w + j0 + (k - na);
+      sk[k] = A[g];
+      sv[k] = AV[g];
+    }
   }
   __syncthreads();
   const uint64_t* sA = sk;
@@ -833,9 +838,13 @@ __global__ void __launch_bounds__(MT_THREADS)
     }
   }
   __syncthreads();
-  for (int64_t k = threadIdx.x; k < m; k += MT_THREADS) {
-    K2[out0 + k] = sk[k];
-    V2[out0 + k] = sv[k];
+#pragma unroll
+  for (int u = 0; u < MT_PER; ++u) {
+    const int k = threadIdx.x + u * MT_THREADS;
+    if (k < m) {
+      K2[out0 + k] = sk[k];
+      V2[out0 + k] = sv[k];
+    }
   }
 }
 
