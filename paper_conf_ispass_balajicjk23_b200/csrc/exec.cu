@@ -746,7 +746,7 @@ __device__ __forceinline__ float lane_row_sum(const int32_t* __restrict__ col,
   const int32_t* cp = col + (a & ~(OT)7);
   const float* vp = val + (a & ~(OT)7);
   const int lo = (int)(a & 7), hi = lo + L;
-#pragma unroll((EF & 16) ? 1 : 2)
+#pragma unroll 2
   for (int k = 0; k < hi; k += 8) {
     int cc[8];
     float vv[8];
@@ -938,15 +938,6 @@ int lane_ef_mode(const spmv_plan_s* p) {
   return p->opts.evict_first && p->stream_ef ? 1 : 0;
 }
 
-// one chunk in flight per lane (EF & 16): fewer registers, more rows in
-// flight, for plans whose short rows are mostly one chunk long (dev knob
-// SPMV_LANE_ONE for the A/B; default off until measured)
-bool lane_one_chunk(const spmv_plan_s* p) {
-  if (const char* e = getenv("SPMV_LANE_ONE")) return atoi(e) != 0;
-  (void)p;
-  return false;
-}
-
 int lane_pred_mode(const spmv_plan_s* p) {
   if (const char* e = getenv("SPMV_LANE_PRED")) return atoi(e) != 0;  // dev knob (A/B)
   return p->lane_pred ? 1 : 0;
@@ -969,16 +960,10 @@ void launch_lane(spmv_plan_s* p, const float* x, float* y, const double* ss_in, 
     else if (ef == 2) launch_lane_t<OT, SS, 2 | (M)>(p, x, y, ss_in, s, dst); \
     else launch_lane_t<OT, SS, 0 | (M)>(p, x, y, ss_in, s, dst);              \
   } while (0)
-  switch (m | (lane_one_chunk(p) ? 16 : 0)) {
-    case 12: SPMV_LANE_M(12); break;
-    case 8: SPMV_LANE_M(8); break;
-    case 4: SPMV_LANE_M(4); break;
-    case 28: SPMV_LANE_M(28); break;
-    case 24: SPMV_LANE_M(24); break;
-    case 20: SPMV_LANE_M(20); break;
-    case 16: SPMV_LANE_M(16); break;
-    default: SPMV_LANE_M(0);
-  }
+  if (m == 12) SPMV_LANE_M(12);
+  else if (m == 8) SPMV_LANE_M(8);
+  else if (m == 4) SPMV_LANE_M(4);
+  else SPMV_LANE_M(0);
 #undef SPMV_LANE_M
 }
 

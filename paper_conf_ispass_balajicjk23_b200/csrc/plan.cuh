@@ -143,7 +143,6 @@ void exec_spmm4(spmv_plan_s* p, const float* X, float* Y, cudaStream_t s);
 int spmm4_launches(const spmv_plan_s* p);
 int lane_ef_mode(const spmv_plan_s* p);
 int lane_pred_mode(const spmv_plan_s* p);
-bool lane_one_chunk(const spmv_plan_s* p);
 void exec_coo(spmv_plan_s* p, const float* x, float* y, cudaStream_t s);
 void export_coo_rows(spmv_plan_s* p, int32_t* rows, cudaStream_t s);
 void coo_free(spmv_plan_s* p);
