@@ -643,6 +643,16 @@ def cpu_baseline(inp, perm, budget_s=10.0, steps=None, warmup=0):
     restricted to its rows, per second).  Workloads above 2^28 entries are
     sampled as a contiguous middle block of B's rows (~2^24 entries)."""
     from oracle import cref
+    # give the reorder's freed heap back to the OS first, so the sample's 1 GB
+    # x (random gathers) can be backed by huge pages in either process that
+    # times the oracle (the bench line and the reference arm)
+    import gc
+    gc.collect()
+    try:
+        import ctypes
+        ctypes.CDLL("libc.so.6").malloc_trim(0)
+    except OSError:
+        pass
     big = inp.nnz > 2**28
     rp, col, val, xB, r0, r1 = oracle_sample(inp, perm, target_nnz=2**24 if big else None)
     m, rows = int(rp[-1]), r1 - r0
