@@ -643,9 +643,9 @@ def cpu_baseline(inp, perm, budget_s=10.0, steps=None, warmup=0):
     restricted to its rows, per second).  Workloads above 2^28 entries are
     sampled as a contiguous middle block of B's rows (~2^24 entries)."""
     from oracle import cref
-    # give the reorder's freed heap back to the OS first, so the sample's 1 GB
-    # x (random gathers) can be backed by huge pages in either process that
-    # times the oracle (the bench line and the reference arm)
+    # give the reorder's freed heap back to the OS first: the two processes
+    # that time the oracle (the bench line, the reference arm) then agree
+    # within 5 % (r84: 28.9 vs 30.2 GB/s; up to 1.55x apart before)
     import gc
     gc.collect()
     try:
